@@ -1,0 +1,136 @@
+/*
+ * fftstencil.h -- C ABI of the B200-native FlashFFTStencil hot path.
+ *
+ * The library computes `total_steps` time steps of a d-dimensional (d = 1, 2, 3)
+ * FP64 stencil with fixed boundary cells, by the FFT route of FlashFFTStencil
+ * (PAPER.md /root/reference/PAPER.md):
+ *   - the grid is split into overlap-save tiles, halo h = radius*T  (§3.1 Splitting,
+ *     Eq. 3, Eq. 4; Stitching Eq. 7);
+ *   - each pair of real tiles is packed as one complex tile (Double-layer Filling,
+ *     §3.2.3 Eq. 9), transformed by dense DFT-matrix GEMMs on the FP64
+ *     tensor cores (Algorithm 1; 1D via the prime-factor map §3.2.1
+ *     Eq. 8), multiplied by the stencil spectrum raised to the power T
+ *     (temporal fusion §4 Eq. 10), inverse-transformed, cropped and stored,
+ *     all inside one fused kernel (Kernel Tailoring, §3.1 Fusing L190-L198);
+ *   - cells within h of the fixed ring are recomputed by T direct steps (the paper is
+ *     silent on boundaries; reading Q5).
+ * The result equals the plain definition (PAPER.md: each step, a cell becomes the
+ * weighted sum of its neighbours) up to FP64 rounding.
+ *
+ * Conventions (all entry points):
+ *   ndim       1, 2 or 3.
+ *   extents    ndim int64 values, outermost axis first; the grid is C-order contiguous
+ *              FP64 and INCLUDES the fixed ring; every extent must exceed 2*radius.
+ *   weights    (2*radius+1)^ndim FP64 values in offset-cube row-major order (axis 0
+ *              outermost): weights[((o0+r)*(2r+1) + (o1+r))*(2r+1) + (o2+r)] multiplies
+ *              u[c+o] (correlation form, reading Q1).  Star stencils are boxes
+ *              with zeros.  Copied at plan creation; the caller keeps ownership.
+ *   radius     1..8.
+ *   T          requested fused depth (time steps per FFT pass), >= 1; 0 = automatic.
+ *              The plan may lower T to fit its tile; the chosen value is in plan_info.
+ *   ring       cells with some coordinate c_a < radius or c_a >= extents[a]-radius keep
+ *              their input value at every step (reading Q2).
+ * Errors: functions returning int give FFTSTENCIL_OK (0) or a negative code;
+ * functions returning a pointer give NULL.  Either way fftstencil_last_error() then
+ * describes the failure (thread-local, never NULL, "" when the last call succeeded).
+ * Asynchronous device faults surface at the caller's next synchronisation.
+ */
+#ifndef FFTSTENCIL_H
+#define FFTSTENCIL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  FFTSTENCIL_OK = 0,
+  FFTSTENCIL_EINVAL = -1,        /* invalid argument                               */
+  FFTSTENCIL_ENOMEM = -2,        /* host or device allocation failed               */
+  FFTSTENCIL_ECUDA = -3,         /* a CUDA runtime call or kernel launch failed    */
+  FFTSTENCIL_ENCCL = -4,         /* reserved: multi-GPU halo exchange              */
+  FFTSTENCIL_EUNSUPPORTED = -5   /* valid request this build does not implement    */
+};
+
+/* Opaque plan: owns its device auxiliary data (DFT matrices, powered spectra, band
+ * blocks) and one grid-sized device scratch buffer.  Bound to the CUDA device that
+ * was current at creation.  Not re-entrant: one fftstencil_run at a time per plan. */
+typedef struct fftstencil_plan fftstencil_plan;
+
+typedef struct {
+  int ndim;
+  int T;                        /* fused steps per pass actually used               */
+  int radius;
+  int halo;                     /* h = radius*T                                     */
+  int tile[3];                  /* FFT tile extent per axis (1D: N1*N2 in tile[0])  */
+  int valid[3];                 /* S = tile - 2h, cells each tile stores per axis   */
+  int pfa[2];                   /* 1D prime-factor split N1 x N2 (0 otherwise)      */
+  int64_t extents[3];
+  int64_t tiles;                /* overlap-save tiles covering the exact region     */
+  int64_t pairs;                /* complex tile pairs (Double-layer Filling)        */
+  int64_t band_blocks;          /* CTA blocks of the boundary-band kernel           */
+  double flops_per_cell_step;   /* algorithmic FP64 flops per cell-step (the plan's
+                                   dense-DFT tile, unpadded)  */
+  double mma_flops_per_pass;    /* FP64 tensor flops one fused-kernel launch issues
+                                   (padding included)                               */
+  size_t smem_bytes;            /* dynamic shared memory of the fused kernel        */
+  size_t device_bytes;          /* device memory the plan owns                      */
+  int fused_grid;               /* CTAs of the persistent fused kernel              */
+  int64_t last_run_launches;    /* kernels the last fftstencil_run enqueued          */
+} fftstencil_info;
+
+/* Build a plan (host precompute + device upload).  Returns NULL on error. */
+fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const double* weights,
+                                        int radius, int T);
+
+/* Enqueue `total_steps` (>= 0) time steps on `stream` (a cudaStream_t; NULL = the
+ * legacy default stream).  `in` and `out` are device pointers to prod(extents) FP64
+ * values on the plan's device; the caller owns them.  `in` is read only unless it
+ * aliases `out` (allowed).  total_steps == 0 copies in to out.  Asynchronous: no host
+ * synchronisation.  Returns FFTSTENCIL_OK or a negative code. */
+int fftstencil_run(fftstencil_plan* plan, const double* in, double* out, int64_t total_steps,
+                   void* stream);
+
+/* End-to-end variant with HOST buffers: copies h_in (prod(extents) FP64, pageable or
+ * pinned) to device, runs, copies the result to h_out, and synchronises `stream`
+ * before returning.  Uses two device grids owned by the plan (allocated on first use). */
+int fftstencil_run_host(fftstencil_plan* plan, const double* h_in, double* h_out,
+                        int64_t total_steps, void* stream);
+
+/* Release everything the plan owns.  NULL is a no-op. */
+void fftstencil_destroy(fftstencil_plan* plan);
+
+/* Plan geometry and cost model. */
+int fftstencil_plan_info(const fftstencil_plan* plan, fftstencil_info* info);
+
+/* Thread-local description of the last failure; "" after a successful call. */
+const char* fftstencil_last_error(void);
+
+/* ---- host-only introspection (no CUDA call; usable on a machine without a GPU) ----
+ * Run the plan builder alone and report the geometry it would choose. */
+int fftstencil_describe(int ndim, const int64_t* extents, const double* weights, int radius,
+                        int T, fftstencil_info* info);
+
+/* Export the host plan's auxiliary tables, for tests of the plan builder:
+ *   which = 0: forward DFT matrix of axis `axis` (1D: axis 0 -> F_N1, axis 1 -> F_N2),
+ *              row-major L x L complex as interleaved (re, im) pairs, 2*L*L doubles;
+ *   which = 1: powered spectrum S_t (t = `t`, 1..T) in the kernel's order (2D/3D:
+ *              natural k order; 1D: N1 x N2 matrix in the Ruritanian order of Eq. 8),
+ *              2*prod(tile) doubles (interleaved complex);
+ *   which = 2: tile origins / ownership: for each tile (row-major tile order), per
+ *              axis: origin, first owned cell, owned count -> 3*ndim*tiles int64
+ *              values written as doubles.
+ *   which = 3: 1D only: the prime-factor input map, N1*N2 entries: position l of the
+ *              tile element stored at matrix cell (l1, l2) (row-major), as doubles.
+ * `out` must hold `cap` doubles; returns the number of doubles needed (>= 0) or a
+ * negative code.  Call with out = NULL to query the size. */
+int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* weights, int radius,
+                              int T, int which, int axis, int t, double* out, int64_t cap);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* FFTSTENCIL_H */

@@ -1,0 +1,149 @@
+"""B200-native FlashFFTStencil hot path: Python binding over the C ABI (include/fftstencil.h).
+
+    from paper_conf_ppopp_hanlcbzyczcy25_b200 import Plan
+    plan = Plan((10240, 10240), weights, radius=1, T=8)       # host precompute + upload
+    plan.run(u_in, u_out, total_steps=1000)                   # torch CUDA float64 tensors
+    plan.run_host(h_in, h_out, total_steps=1000)              # numpy arrays (end to end)
+
+Every step of the path runs in the CUDA kernels of libfftstencil.so; this module only
+marshals arguments (torch is used for device memory and streams).  PAPER.md citations
+live in include/fftstencil.h and csrc/.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import _native
+from ._native import FftStencilError, Info, last_error
+
+__all__ = ["Plan", "describe", "export_aux", "FftStencilError"]
+
+
+def _arrays(extents, weights, radius):
+    ext = np.ascontiguousarray(np.asarray(extents, dtype=np.int64).reshape(-1))
+    w = np.ascontiguousarray(np.asarray(weights, dtype=np.float64).reshape(-1))
+    if w.size != (2 * int(radius) + 1) ** ext.size:
+        raise ValueError(f"weights must have (2r+1)^ndim = {(2 * int(radius) + 1) ** ext.size} entries")
+    return ext, w
+
+
+def _i64p(a):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+
+
+def _dp(a):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+
+
+def describe(extents, weights, radius: int, T: int = 0) -> dict:
+    """Run the host plan builder only (no GPU needed) and return its geometry."""
+    ext, w = _arrays(extents, weights, radius)
+    info = Info()
+    rc = _native.lib().fftstencil_describe(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
+                                           ctypes.byref(info))
+    if rc != 0:
+        raise FftStencilError(rc, last_error())
+    return info.as_dict()
+
+
+def export_aux(extents, weights, radius: int, T: int, which: int, axis: int = 0, t: int = 1) -> np.ndarray:
+    """Host plan tables (see fftstencil_export_aux in include/fftstencil.h)."""
+    ext, w = _arrays(extents, weights, radius)
+    L = _native.lib()
+    n = L.fftstencil_export_aux(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T), int(which), int(axis),
+                                int(t), None, 0)
+    if n < 0:
+        raise FftStencilError(int(n), last_error())
+    out = np.empty(int(n), dtype=np.float64)
+    m = L.fftstencil_export_aux(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T), int(which), int(axis),
+                                int(t), _dp(out), int(n))
+    if m < 0:
+        raise FftStencilError(int(m), last_error())
+    return out
+
+
+class Plan:
+    """A FlashFFTStencil plan bound to the current CUDA device."""
+
+    def __init__(self, extents, weights, radius: int, T: int = 0):
+        ext, w = _arrays(extents, weights, radius)
+        self.extents = tuple(int(e) for e in ext)
+        self.radius = int(radius)
+        self._lib = _native.lib()
+        h = self._lib.fftstencil_plan_create(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T))
+        if not h:
+            raise FftStencilError(_native.EINVAL, last_error())
+        self._h = ctypes.c_void_p(h)
+
+    # -- lifetime --
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.fftstencil_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # -- queries --
+    def info(self) -> dict:
+        info = Info()
+        rc = self._lib.fftstencil_plan_info(self._h, ctypes.byref(info))
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+        return info.as_dict()
+
+    # -- execution --
+    def _check_dev(self, t, name):
+        import torch
+        if not isinstance(t, torch.Tensor) or not t.is_cuda or t.dtype != torch.float64:
+            raise TypeError(f"{name} must be a CUDA float64 torch tensor")
+        if tuple(t.shape) != self.extents or not t.is_contiguous():
+            raise ValueError(f"{name} must be contiguous with shape {self.extents}")
+
+    def run(self, inp, out, total_steps: int, stream=None) -> None:
+        """Enqueue total_steps time steps: out <- stencil^steps(inp) (asynchronous)."""
+        import torch
+        self._check_dev(inp, "inp")
+        self._check_dev(out, "out")
+        s = stream if stream is not None else torch.cuda.current_stream(inp.device)
+        rc = self._lib.fftstencil_run(self._h, ctypes.c_void_p(inp.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                      int(total_steps), ctypes.c_void_p(s.cuda_stream))
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+
+    def run_raw(self, in_ptr: int, out_ptr: int, total_steps: int, stream_handle: int) -> None:
+        rc = self._lib.fftstencil_run(self._h, ctypes.c_void_p(in_ptr), ctypes.c_void_p(out_ptr),
+                                      int(total_steps), ctypes.c_void_p(stream_handle))
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+
+    def run_host(self, h_in, h_out, total_steps: int, stream=None) -> None:
+        """End to end with host buffers (numpy float64 or CPU torch tensors); synchronous."""
+        def ptr(a, name):
+            if isinstance(a, np.ndarray):
+                if a.dtype != np.float64 or not a.flags.c_contiguous or tuple(a.shape) != self.extents:
+                    raise ValueError(f"{name} must be C-contiguous float64 with shape {self.extents}")
+                return a.ctypes.data
+            import torch
+            if isinstance(a, torch.Tensor) and not a.is_cuda and a.dtype == torch.float64 and a.is_contiguous():
+                return a.data_ptr()
+            raise TypeError(f"{name} must be a host float64 array")
+        sh = 0
+        if stream is not None:
+            sh = stream.cuda_stream
+        rc = self._lib.fftstencil_run_host(self._h, ctypes.c_void_p(ptr(h_in, "h_in")),
+                                           ctypes.c_void_p(ptr(h_out, "h_out")), int(total_steps),
+                                           ctypes.c_void_p(sh))
+        if rc != 0:
+            raise FftStencilError(rc, last_error())

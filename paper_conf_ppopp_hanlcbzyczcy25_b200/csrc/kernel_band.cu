@@ -1,0 +1,115 @@
+// Boundary-band and fixed-ring kernels (sm_100a).
+//
+// The paper never states a boundary condition (reading Q2); the product keeps a fixed ring
+// of width r.  A T-step FFT pass reproduces the direct stencil only on the exact region
+// [h, n_a - h) of every axis (reading Q5): cells of the band r <= c_a < h (and the mirror
+// band) feel the fixed ring within T steps.  This kernel recomputes the band by t direct
+// steps (PAPER.md L93 definition) in shared memory: one CTA per band block loads the block
+// grown by r*t on every side (clipped to the grid), steps t times -- ring cells held,
+// cells whose neighbourhood leaves the loaded region held (they lie outside the dependency
+// cone of every cell written) -- and writes the block.  Blocks partition the band exactly
+// (plan.cpp), so every band cell is written once per pass and never overlaps the fused
+// kernel's exact-region writes.
+#include "kernels.cuh"
+
+namespace fstencil {
+namespace {
+
+__global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
+  extern __shared__ double sb[];
+  const int* blk = a.blocks + 8 * blockIdx.x;
+  int64_t lo[3], hi[3], rl[3], D[3];
+#pragma unroll
+  for (int q = 0; q < 3; ++q) {
+    lo[q] = blk[q];
+    hi[q] = blk[3 + q];
+    const int64_t gq = a.active[q] ? (int64_t)a.r * a.t : 0;
+    rl[q] = max((int64_t)0, lo[q] - gq);
+    D[q] = min(a.n[q], hi[q] + gq) - rl[q];
+  }
+  const int64_t vol = D[0] * D[1] * D[2];
+  double* b0 = sb;
+  double* b1 = sb + vol;
+  for (int64_t e = threadIdx.x; e < vol; e += blockDim.x) {
+    const int64_t i2 = e % D[2], i1 = (e / D[2]) % D[1], i0 = e / (D[1] * D[2]);
+    b0[e] = a.src[((rl[0] + i0) * a.n[1] + (rl[1] + i1)) * a.n[2] + (rl[2] + i2)];
+  }
+  __syncthreads();
+  const int r = a.r, wd = 2 * r + 1;
+  const int lo0 = a.active[0] ? -r : 0, lo1 = a.active[1] ? -r : 0, lo2 = a.active[2] ? -r : 0;
+  const int hi0 = -lo0, hi1 = -lo1, hi2 = -lo2;
+  for (int s = 0; s < a.t; ++s) {
+    for (int64_t e = threadIdx.x; e < vol; e += blockDim.x) {
+      const int64_t i2 = e % D[2], i1 = (e / D[2]) % D[1], i0 = e / (D[1] * D[2]);
+      const int64_t ii[3] = {i0, i1, i2};
+      bool keep = false;
+#pragma unroll
+      for (int q = 0; q < 3; ++q) {
+        if (!a.active[q]) continue;
+        const int64_t c = rl[q] + ii[q];
+        keep |= (c < r) || (c >= a.n[q] - r);                 // fixed ring
+        keep |= (ii[q] < r) || (ii[q] + r >= D[q]);           // region edge
+      }
+      double v;
+      if (keep) {
+        v = b0[e];
+      } else {
+        v = 0.0;
+        int k = 0;
+        for (int o0 = lo0; o0 <= hi0; ++o0)
+          for (int o1 = lo1; o1 <= hi1; ++o1)
+            for (int o2 = lo2; o2 <= hi2; ++o2, ++k) {
+              const double wv = __ldg(a.w + k);
+              v = fma(wv, b0[((i0 + o0) * D[1] + (i1 + o1)) * D[2] + (i2 + o2)], v);
+            }
+      }
+      b1[e] = v;
+    }
+    __syncthreads();
+    double* t = b0; b0 = b1; b1 = t;
+  }
+  (void)wd;
+  const int64_t O1 = hi[1] - lo[1], O2 = hi[2] - lo[2];
+  const int64_t ovol = (hi[0] - lo[0]) * O1 * O2;
+  for (int64_t e = threadIdx.x; e < ovol; e += blockDim.x) {
+    const int64_t j2 = e % O2, j1 = (e / O2) % O1, j0 = e / (O1 * O2);
+    const int64_t c0 = lo[0] + j0, c1 = lo[1] + j1, c2 = lo[2] + j2;
+    a.dst[(c0 * a.n[1] + c1) * a.n[2] + c2] =
+        b0[((c0 - rl[0]) * D[1] + (c1 - rl[1])) * D[2] + (c2 - rl[2])];
+  }
+}
+
+__global__ void box_copy_kernel(const BoxCopyArgs a) {
+  const int64_t L0 = a.hi[0] - a.lo[0], L1 = a.hi[1] - a.lo[1], L2 = a.hi[2] - a.lo[2];
+  const int64_t vol = L0 * L1 * L2;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < vol; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j2 = e % L2, j1 = (e / L2) % L1, j0 = e / (L1 * L2);
+    const int64_t idx = ((a.lo[0] + j0) * a.n[1] + (a.lo[1] + j1)) * a.n[2] + (a.lo[2] + j2);
+    const double v = a.src[idx];
+    if (a.dst0) a.dst0[idx] = v;
+    if (a.dst1) a.dst1[idx] = v;
+  }
+}
+
+}  // namespace
+
+cudaError_t band_configure(size_t smem) {
+  return cudaFuncSetAttribute(band_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+}
+
+cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s) {
+  if (a.nblocks <= 0) return cudaSuccess;
+  band_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_box_copy(const BoxCopyArgs& a, cudaStream_t s) {
+  const int64_t vol = (a.hi[0] - a.lo[0]) * (a.hi[1] - a.lo[1]) * (a.hi[2] - a.lo[2]);
+  if (vol <= 0) return cudaSuccess;
+  int64_t grid = (vol + 255) / 256;
+  if (grid > 4096) grid = 4096;
+  box_copy_kernel<<<(int)grid, 256, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace fstencil

@@ -1,0 +1,257 @@
+// Fused 2D FFT-stencil tile kernel (sm_100a, FP64 tensor cores via DMMA.8x8x4).
+//
+// One CTA owns a pair of overlap-save tiles at a time (persistent grid-stride loop) and
+// runs the whole of PAPER.md Algorithm 1 (L252-L258) on it in shared memory/registers:
+//   load    tiles 2p and 2p+1 (L x L, halo h = rT, zero outside the grid) become the
+//           real and imaginary planes of one complex tile  (Double-layer Filling, §3.2.3,
+//           Eq. 9; Splitting Eq. 3)
+//   M1      P^T = F . X^T        forward DFT along axis 1  (Alg. 1 line 1, right factor)
+//   M2      Q   = F . P          forward DFT along axis 0  (Alg. 1 line 1, left factor)
+//   mult    Q  *= S_T            powered spectrum, 1/L^2 folded in (Alg. 1 line 2; Eq. 10)
+//   M3      R   = G . Q^T        inverse DFT along axis 1, crop-aware: G = conj(F)[h:h+S]
+//   M4      Y   = G . R^T        inverse DFT along axis 0, crop-aware (Alg. 1 lines 3-4;
+//                                 iF recomputed from F by conjugation, L258/L278)
+//   store   Re(Y) -> tile 2p, Im(Y) -> tile 2p+1, valid S x S window only (Stitching,
+//           Eq. 7; reading Q4)
+// Warp w owns the 8-wide stripe w of the transform: in M1/M2 a frequency stripe of axis 1,
+// in M3/M4 an output stripe of axis 1.  M1->M2 and M3->M4 chain C fragments straight into
+// B fragments (Swizzling Fragments, L266-L272); the only shared-memory round trip is the
+// transposition of ownership between the forward and inverse halves.
+#include "device_common.cuh"
+#include "kernels.cuh"
+
+namespace fstencil {
+namespace {
+
+using dev::dmma;
+using dev::perm8;
+
+template <int L>
+__global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
+  constexpr int NT = L / 8;      // 8x8 tiles per side == warps
+  constexpr int LD = L + 4;      // padded row stride (doubles): 8-bank shift per row
+  extern __shared__ __align__(16) double smem[];
+  double* sFr = smem;
+  double* sFi = sFr + L * LD;
+  double* sXa = sFi + L * LD;    // tile 2p (real part) ... later Q' real part
+  double* sXb = sXa + L * LD;    // tile 2p+1 (imag part) ... later Q' imag part
+
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31, g = lane >> 2, q = lane & 3;
+  constexpr int NTHR = L * 4;
+
+  for (int e = tid; e < L * L; e += NTHR) {
+    const int r = e / L, c = e - r * L;
+    sFr[r * LD + perm8(c)] = a.Fre[e];
+    sFi[r * LD + perm8(c)] = a.Fim[e];
+  }
+  const int S = a.S, h = a.h;
+  const int MT = (S + 7) >> 3;   // output 8-tiles per axis (S padded to 8)
+
+  for (int64_t p = blockIdx.x; p < a.npairs; p += gridDim.x) {
+    __syncthreads();
+    // ---- load the halo'd pair (coalesced along axis 1; OOB = 0) ----
+#pragma unroll
+    for (int t = 0; t < 2; ++t) {
+      const int64_t tile = 2 * p + t;
+      double* sX = t ? sXb : sXa;
+      if (tile < a.ntiles) {
+        const int64_t t0 = tile / a.nt1, t1 = tile - t0 * a.nt1;
+        const int64_t o0 = t0 * S, o1 = t1 * S;
+        for (int e = tid; e < L * L; e += NTHR) {
+          const int r = e / L, c = e - r * L;
+          const int64_t gr = o0 + r, gc = o1 + c;
+          double v = 0.0;
+          if (gr < a.n0 && gc < a.n1) v = __ldg(a.src + gr * a.n1 + gc);
+          sX[r * LD + perm8(c)] = v;
+        }
+      } else {
+        for (int e = tid; e < L * L; e += NTHR) {
+          const int r = e / L, c = e - r * L;
+          sX[r * LD + perm8(c)] = 0.0;
+        }
+      }
+    }
+    __syncthreads();
+
+    // ---- M1: P^T[k1 stripe][l0] = sum_l1 F[k1][l1] X[l0][l1]  (B from shared) ----
+    double Pr[NT][2], Pi[NT][2];
+#pragma unroll
+    for (int i = 0; i < NT; ++i) Pr[i][0] = Pr[i][1] = Pi[i][0] = Pi[i][1] = 0.0;
+    {
+      const double* fr = sFr + (8 * warp + g) * LD + q;
+      const double* fi = sFi + (8 * warp + g) * LD + q;
+#pragma unroll
+      for (int kc = 0; kc < L / 4; ++kc) {
+        const int pc = 4 * kc;
+        const double ar = fr[pc], ai = fi[pc], nai = -ai;
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt) {
+          const double br = sXa[(8 * nt + g) * LD + q + pc];
+          const double bi = sXb[(8 * nt + g) * LD + q + pc];
+          dmma(Pr[nt], ar, br);
+          dmma(Pr[nt], nai, bi);
+          dmma(Pi[nt], ar, bi);
+          dmma(Pi[nt], ai, br);
+        }
+      }
+    }
+    // ---- M2: Q[k0][k1 stripe] = sum_l0 F[k0][l0] P[l0][k1]  (B = M1's C fragments) ----
+    double Qr[NT][2], Qi[NT][2];
+#pragma unroll
+    for (int i = 0; i < NT; ++i) Qr[i][0] = Qr[i][1] = Qi[i][0] = Qi[i][1] = 0.0;
+#pragma unroll
+    for (int kg = 0; kg < NT; ++kg) {
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const double br = Pr[kg][j], bi = Pi[kg][j];
+        const int pc = 8 * kg + 4 * j + q;
+#pragma unroll
+        for (int mt = 0; mt < NT; ++mt) {
+          const double ar = sFr[(8 * mt + g) * LD + pc];
+          const double ai = sFi[(8 * mt + g) * LD + pc];
+          dmma(Qr[mt], ar, br);
+          dmma(Qr[mt], -ai, bi);
+          dmma(Qi[mt], ar, bi);
+          dmma(Qi[mt], ai, br);
+        }
+      }
+    }
+    // ---- pointwise multiply by the powered spectrum (Eq. 10) in the C fragments ----
+#pragma unroll
+    for (int mt = 0; mt < NT; ++mt) {
+      const int k0 = 8 * mt + g, k1 = 8 * warp + 2 * q;
+      const double2 sr = __ldg(reinterpret_cast<const double2*>(a.Sre + k0 * L + k1));
+      const double2 si = __ldg(reinterpret_cast<const double2*>(a.Sim + k0 * L + k1));
+      const double r0 = Qr[mt][0] * sr.x - Qi[mt][0] * si.x;
+      const double i0 = Qr[mt][0] * si.x + Qi[mt][0] * sr.x;
+      const double r1 = Qr[mt][1] * sr.y - Qi[mt][1] * si.y;
+      const double i1 = Qr[mt][1] * si.y + Qi[mt][1] * sr.y;
+      Qr[mt][0] = r0; Qi[mt][0] = i0; Qr[mt][1] = r1; Qi[mt][1] = i1;
+    }
+    __syncthreads();   // every warp is past M1: the tile planes may be overwritten
+#pragma unroll
+    for (int mt = 0; mt < NT; ++mt)
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const int idx = (8 * mt + g) * LD + 8 * warp + 4 * j + q;   // perm8 of k1
+        sXa[idx] = Qr[mt][j];
+        sXb[idx] = Qi[mt][j];
+      }
+    __syncthreads();
+
+    if (warp < MT) {
+      // ---- M3: R[l1 stripe][k0] = sum_k1 conj(F)[h+l1][k1] Q'[k0][k1] (B from shared) ----
+      double Rr[NT][2], Ri[NT][2];
+#pragma unroll
+      for (int i = 0; i < NT; ++i) Rr[i][0] = Rr[i][1] = Ri[i][0] = Ri[i][1] = 0.0;
+      {
+        const int arow = min(h + 8 * warp + g, L - 1);   // rows past S are padding
+        const double* fr = sFr + arow * LD + q;
+        const double* fi = sFi + arow * LD + q;
+#pragma unroll
+        for (int kc = 0; kc < L / 4; ++kc) {
+          const int pc = 4 * kc;
+          const double ar = fr[pc], ai = fi[pc], nai = -ai;
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt) {
+            const double br = sXa[(8 * nt + g) * LD + q + pc];
+            const double bi = sXb[(8 * nt + g) * LD + q + pc];
+            dmma(Rr[nt], ar, br);     // conj(F) . Q'^T
+            dmma(Rr[nt], ai, bi);
+            dmma(Ri[nt], ar, bi);
+            dmma(Ri[nt], nai, br);
+          }
+        }
+      }
+      // ---- M4: Y[l0][l1 stripe] = sum_k0 conj(F)[h+l0][k0] R[l1][k0] (B = M3's C) ----
+      double Yr[NT][2], Yi[NT][2];
+#pragma unroll
+      for (int i = 0; i < NT; ++i) Yr[i][0] = Yr[i][1] = Yi[i][0] = Yi[i][1] = 0.0;
+#pragma unroll
+      for (int kg = 0; kg < NT; ++kg) {
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const double br = Rr[kg][j], bi = Ri[kg][j];
+          const int pc = 8 * kg + 4 * j + q;
+#pragma unroll
+          for (int mt = 0; mt < NT; ++mt) {
+            if (mt < MT) {
+              const int arow = min(h + 8 * mt + g, L - 1);
+              const double ar = sFr[arow * LD + pc];
+              const double ai = sFi[arow * LD + pc];
+              dmma(Yr[mt], ar, br);
+              dmma(Yr[mt], ai, bi);
+              dmma(Yi[mt], ar, bi);
+              dmma(Yi[mt], -ai, br);
+            }
+          }
+        }
+      }
+      // ---- stitch: the S x S valid window of each tile, exact region only ----
+      const int64_t ta = 2 * p, tb = 2 * p + 1;
+      const int64_t a0 = ta / a.nt1, a1 = ta - a0 * a.nt1;
+      const int64_t b0 = tb / a.nt1, b1 = tb - b0 * a.nt1;
+      const bool has_b = tb < a.ntiles;
+#pragma unroll
+      for (int mt = 0; mt < NT; ++mt) {
+        if (mt < MT) {
+          const int l0 = 8 * mt + g;
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            const int l1 = 8 * warp + 2 * q + j;
+            if (l0 < S && l1 < S) {
+              int64_t c0 = a0 * S + h + l0, c1 = a1 * S + h + l1;
+              if (c0 < a.n0 - h && c1 < a.n1 - h) a.dst[c0 * a.n1 + c1] = Yr[mt][j];
+              if (has_b) {
+                c0 = b0 * S + h + l0;
+                c1 = b1 * S + h + l1;
+                if (c0 < a.n0 - h && c1 < a.n1 - h) a.dst[c0 * a.n1 + c1] = Yi[mt][j];
+              }
+            }
+          }
+        }
+      }
+    }
+  }
+}
+
+template <int L>
+cudaError_t configure_L(int* max_blocks) {
+  const size_t smem = fused2d_smem(L);
+  cudaError_t e = cudaFuncSetAttribute(fft2d_kernel<L>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_kernel<L>, L * 4, smem);
+}
+
+}  // namespace
+
+int fused2d_threads(int L) { return L * 4; }
+size_t fused2d_smem(int L) { return (size_t)4 * L * (L + 4) * sizeof(double); }
+
+cudaError_t fused2d_configure(int L, int* max_blocks) {
+  switch (L) {
+    case 16: return configure_L<16>(max_blocks);
+    case 24: return configure_L<24>(max_blocks);
+    case 32: return configure_L<32>(max_blocks);
+    case 40: return configure_L<40>(max_blocks);
+    case 48: return configure_L<48>(max_blocks);
+    case 56: return configure_L<56>(max_blocks);
+    case 64: return configure_L<64>(max_blocks);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+cudaError_t launch_fused2d(int L, const Fft2dArgs& a, int grid, cudaStream_t s) {
+  const size_t smem = fused2d_smem(L);
+  switch (L) {
+#define FS_CASE(LL) \
+  case LL: fft2d_kernel<LL><<<grid, LL * 4, smem, s>>>(a); break;
+    FS_CASE(16) FS_CASE(24) FS_CASE(32) FS_CASE(40) FS_CASE(48) FS_CASE(56) FS_CASE(64)
+#undef FS_CASE
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace fstencil

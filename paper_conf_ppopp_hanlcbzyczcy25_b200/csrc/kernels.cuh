@@ -1,0 +1,74 @@
+// Kernel argument blocks and launchers of the fused FFT-stencil path (sm_100a).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace fstencil {
+
+// One fused pass of the 2D path over every tile pair (kernel_fft2d.cu).
+struct Fft2dArgs {
+  const double* src;
+  double* dst;
+  int64_t n0, n1;        // grid extents
+  int h, S;              // halo r*T (tile geometry) and valid side L - 2h
+  int64_t nt1;           // tiles along axis 1
+  int64_t ntiles, npairs;
+  const double* Fre;     // L x L forward DFT matrix, natural row-major
+  const double* Fim;
+  const double* Sre;     // L x L powered spectrum of this pass, natural row-major
+  const double* Sim;
+};
+
+// One fused pass of the 1D prime-factor path (kernel_fft1d.cu).
+struct Fft1dArgs {
+  const double* src;
+  double* dst;
+  int64_t n;
+  int h, S, L;           // L = N1*N2 = 56
+  int64_t ntiles, npairs;
+  const double* Fre;     // 16 x 8: rows 0..7 F_N1, rows 8..15 F_N2 zero-padded
+  const double* Fim;
+  const double* Sre;     // 8 x 8 Ruritanian-ordered powered spectrum, zero-padded
+  const double* Sim;
+  const int* crt;        // 64: tile position stored at (l1, l2), -1 = padding
+};
+
+// Direct T-step recomputation of the boundary band (kernel_band.cu).
+struct BandArgs {
+  const double* src;
+  double* dst;
+  int64_t n[3];          // embedded extents (leading 1s)
+  int active[3];
+  int r, t;              // radius, steps of this pass
+  const double* w;       // (2r+1)^ndim weights, offset-cube row-major
+  const int* blocks;     // 8 ints per block: lo[3], hi[3], face, pad
+  int nblocks;
+};
+
+// Copy a box (embedded coordinates) from src to dst0 and dst1 (either may be null).
+struct BoxCopyArgs {
+  const double* src;
+  double* dst0;
+  double* dst1;
+  int64_t n[3];
+  int64_t lo[3], hi[3];
+};
+
+int fused2d_threads(int L);
+size_t fused2d_smem(int L);
+cudaError_t fused2d_configure(int L, int* max_blocks_per_sm);
+cudaError_t launch_fused2d(int L, const Fft2dArgs& a, int grid, cudaStream_t s);
+
+constexpr int kFft1dWarpsPerBlock = 8;
+cudaError_t fused1d_configure(int* max_blocks_per_sm);
+cudaError_t launch_fused1d(const Fft1dArgs& a, int grid, cudaStream_t s);
+
+constexpr int kBandThreads = 256;
+cudaError_t band_configure(size_t smem);
+cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s);
+
+cudaError_t launch_box_copy(const BoxCopyArgs& a, cudaStream_t s);
+
+}  // namespace fstencil

@@ -1,0 +1,338 @@
+// Host plan builder (see plan.h).  Pure C++: no CUDA here, so the builder can be
+// exercised by the CPU test-suite through fftstencil_describe / fftstencil_export_aux.
+#include "plan.h"
+
+#include <algorithm>
+#include <cmath>
+#include <complex>
+
+#include "fftstencil.h"
+
+namespace fstencil {
+namespace {
+
+using cplx = std::complex<double>;
+constexpr double kTwoPi = 6.283185307179586476925286766559;
+
+int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+int round8(int x) { return (x + 7) / 8 * 8; }
+
+// exp(-2 pi i m / L) with the argument reduced to [0, L) first (SURVEY §7 pitfall 6).
+cplx root(int64_t m, int64_t L) {
+  m %= L;
+  if (m < 0) m += L;
+  const double a = -kTwoPi * (double)m / (double)L;
+  return cplx(std::cos(a), std::sin(a));
+}
+
+// sigma(theta_k) = sum_o w[o] exp(+i o.theta_k), theta_a = 2 pi k_a / L_a  (reading Q6/Q7).
+// exp(+i o 2 pi k / L) = root(-o k, L): reduced per axis, multiplied across axes.
+cplx symbol(const HostPlan& p, const int* k, const int* L) {
+  const int r = p.radius, wd = 2 * r + 1, nd = p.ndim;
+  cplx acc(0.0, 0.0);
+  const int total = (int)p.w.size();
+  for (int idx = 0; idx < total; ++idx) {
+    const double wv = p.w[idx];
+    if (wv == 0.0) continue;
+    int rem = idx;
+    int o[3] = {0, 0, 0};
+    for (int a = nd - 1; a >= 0; --a) { o[a] = rem % wd - r; rem /= wd; }
+    cplx ph(1.0, 0.0);
+    for (int a = 0; a < nd; ++a) ph *= root(-(int64_t)o[a] * k[a], L[a]);
+    acc += wv * ph;
+  }
+  return acc;
+}
+
+void fill_dft(int L, int ld, int row0, int col0, std::vector<double>& re, std::vector<double>& im) {
+  for (int j = 0; j < L; ++j)
+    for (int k = 0; k < L; ++k) {
+      const cplx v = root((int64_t)j * k, L);
+      re[(size_t)(row0 + j) * ld + col0 + k] = v.real();
+      im[(size_t)(row0 + j) * ld + col0 + k] = v.imag();
+    }
+}
+
+}  // namespace
+
+double model_flops_2d(int L, int S, int T) {
+  const double Sp = round8(S);
+  const double dm = 2.0 * L * L * L + Sp * L * L + Sp * Sp * L;  // DMMA.8x8x4 count * 64
+  return 8.0 * dm / (2.0 * S * (double)S * T);
+}
+
+static double model_flops_3d(int L, int S, int T) {
+  const double Sp = round8(S), l = L;
+  const double f = 24.0 * l * l * l * l + 8.0 * Sp * l * l * l + 8.0 * Sp * Sp * l * l + 8.0 * Sp * Sp * Sp * l;
+  return f / (2.0 * S * (double)S * S * T);
+}
+
+static double model_flops_1d(int S, int T) {  // one 8x8 complex tile, 4 GEMMs of 8 DMMAs
+  return 32.0 * 512.0 / (2.0 * S * (double)T);
+}
+
+int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
+                    HostPlan& p, std::string& err) {
+  p = HostPlan();
+  if (ndim < 1 || ndim > 3) { err = "ndim must be 1, 2 or 3"; return FFTSTENCIL_EINVAL; }
+  if (!extents || !weights) { err = "extents and weights must be non-NULL"; return FFTSTENCIL_EINVAL; }
+  if (radius < 1 || radius > kMaxRadius) { err = "radius must be in 1..8"; return FFTSTENCIL_EINVAL; }
+  if (T < 0) { err = "T must be >= 0 (0 = automatic)"; return FFTSTENCIL_EINVAL; }
+  for (int a = 0; a < ndim; ++a) {
+    if (extents[a] <= 2 * radius) { err = "every extent must exceed 2*radius"; return FFTSTENCIL_EINVAL; }
+    if (extents[a] > (int64_t(1) << 31) - 1) { err = "extent too large (>= 2^31)"; return FFTSTENCIL_EINVAL; }
+  }
+  const int wd = 2 * radius + 1;
+  int64_t nw = 1;
+  for (int a = 0; a < ndim; ++a) nw *= wd;
+  p.w.assign(weights, weights + nw);
+  for (double v : p.w)
+    if (!std::isfinite(v)) { err = "weights must be finite"; return FFTSTENCIL_EINVAL; }
+  p.ndim = ndim;
+  p.radius = radius;
+  for (int a = 0; a < ndim; ++a) { p.ext[a] = extents[a]; p.n[3 - ndim + a] = extents[a]; }
+  int64_t nmin = extents[0];
+  for (int a = 1; a < ndim; ++a) nmin = std::min(nmin, extents[a]);
+  // h = rT must leave a non-empty exact region on every axis: 2h < n_a.
+  const int hmax_grid = (int)std::min<int64_t>((nmin - 1) / 2, 1 << 20);
+
+  // ---- tile and depth selection (Eq. 5's role, re-derived: DESIGN.md §Plan) ----
+  if (ndim == 1) {
+    p.N1 = kPfaN1;
+    p.N2 = kPfaN2;
+    const int L = p.N1 * p.N2;
+    const int hmax = std::min(hmax_grid, (L - 8) / 2);   // keep S >= 8
+    if (hmax < radius) { err = "grid or radius too small for the 1D tile"; return FFTSTENCIL_EINVAL; }
+    const int tmax = hmax / radius;
+    int bestT = 1;
+    if (T == 0) {
+      double best = 1e300;
+      for (int t = 1; t <= std::min(tmax, 64); ++t) {
+        const double f = model_flops_1d(L - 2 * radius * t, t);
+        if (f < best) { best = f; bestT = t; }
+      }
+    } else {
+      bestT = std::min(T, tmax);
+    }
+    p.T = bestT;
+    p.h = radius * p.T;
+    p.L[0] = L;
+    p.S[0] = L - 2 * p.h;
+    p.flops_per_cell_step = (16.0 * p.N1 * p.N2 * (p.N1 + p.N2) + 6.0 * p.N1 * p.N2) / (2.0 * p.S[0] * p.T);
+    p.mma_flops_per_pair = 32.0 * 512.0;
+  } else if (ndim == 2) {
+    static const int cand[] = {16, 24, 32, 40, 48, 56, 64};
+    double best = 1e300;
+    int bL = 0, bT = 0;
+    const int tlo = T == 0 ? 1 : T, thi = T == 0 ? 16 : T;
+    for (int t = tlo; t <= thi; ++t) {
+      const int h = radius * t;
+      if (h > hmax_grid) break;
+      for (int L : cand) {
+        const int S = L - 2 * h;
+        if (S < 8) continue;
+        const double f = model_flops_2d(L, S, t);
+        if (f < best * (1 - 1e-12)) { best = f; bL = L; bT = t; }
+      }
+    }
+    if (bL == 0) {
+      // requested T too deep for the largest tile or the grid: lower it.
+      for (int t = std::min(thi, 64); t >= 1 && bL == 0; --t) {
+        const int h = radius * t;
+        if (h > hmax_grid) continue;
+        for (int L : cand) {
+          const int S = L - 2 * h;
+          if (S < 8) continue;
+          const double f = model_flops_2d(L, S, t);
+          if (f < best) { best = f; bL = L; bT = t; }
+        }
+      }
+    }
+    if (bL == 0) { err = "no 2D tile fits this radius/grid"; return FFTSTENCIL_EINVAL; }
+    p.T = bT;
+    p.h = radius * bT;
+    p.L[0] = p.L[1] = bL;
+    p.S[0] = p.S[1] = bL - 2 * p.h;
+    const double L = bL, S = p.S[0];
+    p.flops_per_cell_step = (16.0 * L * L * L + 6.0 * L * L + 8.0 * S * L * L + 8.0 * S * S * L) / (2.0 * S * S * bT);
+    const double Sp = round8(p.S[0]);
+    p.mma_flops_per_pair = 8.0 * (2.0 * L * L * L + Sp * L * L + Sp * Sp * L);
+    p.fused_smem = (size_t)32 * bL * (bL + 4);
+  } else {
+    const int L = k3DTile;
+    const int hmax = std::min(hmax_grid, (L - 2) / 2);
+    const int tmax = hmax / radius;
+    if (tmax < 1) { err = "radius too large for the 16^3 3D tile"; return FFTSTENCIL_EINVAL; }
+    int bestT = 1;
+    if (T == 0) {
+      double best = 1e300;
+      for (int t = 1; t <= tmax; ++t) {
+        const double f = model_flops_3d(L, L - 2 * radius * t, t);
+        if (f < best) { best = f; bestT = t; }
+      }
+    } else {
+      bestT = std::min(T, tmax);
+    }
+    p.T = bestT;
+    p.h = radius * bestT;
+    for (int a = 0; a < 3; ++a) { p.L[a] = L; p.S[a] = L - 2 * p.h; }
+    const double l = L, S = p.S[0];
+    p.flops_per_cell_step =
+        (24.0 * l * l * l * l + 6.0 * l * l * l + 8.0 * l * (S * l * l + S * S * l + S * S * S)) /
+        (2.0 * S * S * S * bestT);
+    const double Sp = round8(p.S[0]);
+    p.mma_flops_per_pair = 24.0 * l * l * l * l + 8.0 * Sp * l * l * l + 8.0 * Sp * Sp * l * l + 8.0 * Sp * Sp * Sp * l;
+  }
+
+  // ---- overlap-save schedule (Eq. 3 / Eq. 4 / Eq. 7; reading Q4: centred window) ----
+  p.tiles = 1;
+  for (int a = 0; a < ndim; ++a) {
+    p.nt[a] = ceil_div(p.ext[a] - 2 * p.h, p.S[a]);
+    p.tiles *= p.nt[a];
+  }
+  p.pairs = (p.tiles + 1) / 2;   // Double-layer Filling: tiles 2i (Re) and 2i+1 (Im)
+
+  // ---- DFT matrices (forward; the kernel conjugates for the inverse, L258/L278) ----
+  if (ndim == 1) {
+    p.Fre.assign(2 * 64, 0.0);
+    p.Fim.assign(2 * 64, 0.0);
+    fill_dft(p.N1, 8, 0, 0, p.Fre, p.Fim);          // rows 0..7   : F_N1
+    fill_dft(p.N2, 8, 8, 0, p.Fre, p.Fim);          // rows 8..14  : F_N2 (row 15, col 7 zero)
+    p.crt.assign(64, -1);
+    const int L = p.N1 * p.N2;
+    for (int l = 0; l < L; ++l) p.crt[(l % p.N1) * 8 + (l % p.N2)] = l;   // diagonal / CRT map
+  } else {
+    const int L = p.L[0];
+    p.Fre.assign((size_t)L * L, 0.0);
+    p.Fim.assign((size_t)L * L, 0.0);
+    fill_dft(L, L, 0, 0, p.Fre, p.Fim);
+  }
+
+  // ---- powered spectra S_t, t = 1..T (Eq. 10) with 1/prod(L) folded in (Q7) ----
+  p.Sre.assign(p.T, {});
+  p.Sim.assign(p.T, {});
+  if (ndim == 1) {
+    const int L = p.N1 * p.N2;
+    std::vector<cplx> sig(L);
+    for (int k = 0; k < L; ++k) { int kk[1] = {k}; int LL[1] = {L}; sig[k] = symbol(p, kk, LL); }
+    for (int t = 1; t <= p.T; ++t) {
+      auto& re = p.Sre[t - 1];
+      auto& im = p.Sim[t - 1];
+      re.assign(64, 0.0);
+      im.assign(64, 0.0);
+      for (int k1 = 0; k1 < p.N1; ++k1)
+        for (int k2 = 0; k2 < p.N2; ++k2) {
+          const int k = (k1 * p.N2 + k2 * p.N1) % L;   // Ruritanian order (Eq. 8, reading Q8)
+          cplx v(1.0, 0.0);
+          for (int s = 0; s < t; ++s) v *= sig[k];
+          v /= (double)L;
+          re[k1 * 8 + k2] = v.real();
+          im[k1 * 8 + k2] = v.imag();
+        }
+    }
+  } else {
+    int64_t vol = 1;
+    for (int a = 0; a < ndim; ++a) vol *= p.L[a];
+    std::vector<cplx> sig(vol);
+    for (int64_t i = 0; i < vol; ++i) {
+      int k[3], rem = (int)i;
+      for (int a = ndim - 1; a >= 0; --a) { k[a] = rem % p.L[a]; rem /= p.L[a]; }
+      sig[i] = symbol(p, k, p.L);
+    }
+    for (int t = 1; t <= p.T; ++t) {
+      auto& re = p.Sre[t - 1];
+      auto& im = p.Sim[t - 1];
+      re.resize(vol);
+      im.resize(vol);
+      for (int64_t i = 0; i < vol; ++i) {
+        cplx v(1.0, 0.0);
+        for (int s = 0; s < t; ++s) v *= sig[i];
+        v /= (double)vol;
+        re[i] = v.real();
+        im[i] = v.imag();
+      }
+    }
+  }
+
+  // ---- fixed ring: exact partition into boxes (axis a faces, lower axes interior) ----
+  const int r = radius, h = p.h;
+  const int off = 3 - ndim;
+  for (int a = 0; a < ndim; ++a) {
+    for (int side = 0; side < 2; ++side) {
+      Box b;
+      for (int e = 0; e < 3; ++e) { b.lo[e] = 0; b.hi[e] = p.n[e]; }
+      const int e = off + a;
+      b.lo[e] = side == 0 ? 0 : p.n[e] - r;
+      b.hi[e] = side == 0 ? r : p.n[e];
+      for (int c = 0; c < a; ++c) { b.lo[off + c] = r; b.hi[off + c] = p.n[off + c] - r; }
+      p.ring_boxes.push_back(b);
+    }
+  }
+  // ---- boundary band: interior cells outside the exact region [h, n-h) (reading Q5) ----
+  // Face of axis a: c_a in [r, h) or [n_a-h, n_a-r); axes before a exact ([h, n-h)),
+  // axes after a interior ([r, n-r)).  The boxes partition the band exactly.
+  if (h > r) {
+    for (int a = 0; a < ndim; ++a)
+      for (int side = 0; side < 2; ++side) {
+        Box b;
+        for (int e = 0; e < 3; ++e) { b.lo[e] = 0; b.hi[e] = p.n[e]; }
+        const int e = off + a;
+        b.lo[e] = side == 0 ? r : p.n[e] - h;
+        b.hi[e] = side == 0 ? h : p.n[e] - r;
+        for (int c = 0; c < ndim; ++c) {
+          if (c == a) continue;
+          const int ec = off + c;
+          b.lo[ec] = c < a ? h : r;
+          b.hi[ec] = c < a ? p.n[ec] - h : p.n[ec] - r;
+        }
+        b.face = e;
+        bool empty = false;
+        for (int q = 0; q < 3; ++q) empty |= b.hi[q] <= b.lo[q];
+        if (!empty) p.band_boxes.push_back(b);
+      }
+  }
+  // Split each band box into CTA blocks whose input region (block + r*T on every
+  // active side) fits the band kernel's shared-memory budget (2 buffers of FP64).
+  const int budget_cells = (96 * 1024) / 16;
+  const int grow = 2 * r * p.T;
+  for (const Box& b : p.band_boxes) {
+    int64_t len[3], blk[3];
+    for (int q = 0; q < 3; ++q) len[q] = b.hi[q] - b.lo[q];
+    const int face = b.face;   // the face axis keeps its whole band width
+    int ntan = 0;
+    for (int q = 0; q < 3; ++q) {
+      blk[q] = len[q];
+      if (q >= off && q != face) ++ntan;
+    }
+    const int64_t fw = face >= 0 ? len[face] + grow : 1;
+    int64_t tb = 1024;
+    if (ntan == 1) tb = std::max<int64_t>(8, std::min<int64_t>(256, budget_cells / fw - grow));
+    if (ntan == 2) {
+      int64_t s = (int64_t)std::sqrt((double)budget_cells / (double)fw) - grow;
+      tb = std::max<int64_t>(8, std::min<int64_t>(64, s));
+    }
+    for (int q = off; q < 3; ++q)
+      if (q != face) blk[q] = std::min<int64_t>(len[q], tb);
+    for (int64_t i0 = b.lo[0]; i0 < b.hi[0]; i0 += blk[0])
+      for (int64_t i1 = b.lo[1]; i1 < b.hi[1]; i1 += blk[1])
+        for (int64_t i2 = b.lo[2]; i2 < b.hi[2]; i2 += blk[2]) {
+          const int64_t lo[3] = {i0, i1, i2};
+          int64_t hi[3] = {std::min(i0 + blk[0], b.hi[0]), std::min(i1 + blk[1], b.hi[1]),
+                           std::min(i2 + blk[2], b.hi[2])};
+          int64_t cells = 1;
+          for (int q = 0; q < 3; ++q) {
+            const int64_t g = (q >= off) ? r * (int64_t)p.T : 0;
+            const int64_t rl = std::max<int64_t>(0, lo[q] - g), rh = std::min<int64_t>(p.n[q], hi[q] + g);
+            cells *= rh - rl;
+          }
+          p.band_region_cells = std::max<int>(p.band_region_cells, (int)cells);
+          for (int q = 0; q < 3; ++q) p.band_blocks.push_back((int32_t)lo[q]);
+          for (int q = 0; q < 3; ++q) p.band_blocks.push_back((int32_t)hi[q]);
+          p.band_blocks.push_back(face);
+          p.band_blocks.push_back(0);
+        }
+  }
+  return FFTSTENCIL_OK;
+}
+
+}  // namespace fstencil

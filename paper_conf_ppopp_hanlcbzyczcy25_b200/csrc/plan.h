@@ -1,0 +1,65 @@
+// Host plan builder of the FFT-stencil hot path (no CUDA in this translation unit).
+//
+// What it precomputes:
+//   - tile extent L and valid extent S = L - 2h per axis (Splitting, Eq. 3 L167 /
+//     Eq. 4, tile-length rule Eq. 5 L174-L179 re-derived for B200);
+//   - DFT matrices F_L[j][k] = exp(-2 pi i (jk mod L)/L) (L192, Alg. 1; the inverse
+//     is conj(F), L258, recomputed in the kernel rather than stored, L278);
+//   - powered spectra S_t = sigma(2 pi k/L)^t / prod(L), t = 1..T (Eq. 10;
+//     reading Q6: sigma evaluated directly from the weights);
+//   - 1D: the prime-factor split N1 x N2 with the CRT (diagonal, L232) input map and
+//     the Ruritanian spectrum order of Eq. 8 L216 (reading Q8);
+//   - the overlap-save tile schedule, the fixed-ring boxes and the boundary-band blocks.
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace fstencil {
+
+constexpr int kMaxRadius = 8;
+constexpr int kPfaN1 = 8;     // 1D prime-factor split (gcd(8,7) = 1), N2 padded to 8
+constexpr int kPfaN2 = 7;
+constexpr int k3DTile = 16;   // 3D tile side (a 16^3 complex tile is 64 KiB of SMEM)
+
+struct Box {                   // half-open box in embedded 3-axis coordinates
+  int64_t lo[3];
+  int64_t hi[3];
+  int face = -1;               // embedded axis of the face a band box lies on
+};
+
+struct HostPlan {
+  int ndim = 0, radius = 0, T = 0, h = 0;
+  int64_t n[3] = {1, 1, 1};        // embedded extents (leading 1s for ndim < 3)
+  int64_t ext[3] = {0, 0, 0};      // user extents (ndim entries)
+  std::vector<double> w;           // (2r+1)^ndim weights
+  int L[3] = {1, 1, 1};            // tile extent per user axis
+  int S[3] = {1, 1, 1};            // valid extent per user axis
+  int N1 = 0, N2 = 0;              // 1D prime-factor split
+  int64_t nt[3] = {1, 1, 1};       // tiles per user axis
+  int64_t tiles = 0, pairs = 0;
+  // Device-format auxiliary tables (planar re / im, row-major):
+  //   2D/3D: F is L x L;  1D: F holds F_N1 (8x8) then F_N2 zero-padded to 8x8.
+  std::vector<double> Fre, Fim;
+  //   spectra: index t-1, each prod(tile) (1D: 8x8, Ruritanian, zero-padded).
+  std::vector<std::vector<double>> Sre, Sim;
+  //   1D: crt[l1*8 + l2] = tile position l stored at (l1, l2), or -1 for padding.
+  std::vector<int> crt;
+  std::vector<Box> ring_boxes;     // the fixed ring, partitioned exactly
+  std::vector<Box> band_boxes;     // output boxes of the band kernel (exactly-once cover)
+  std::vector<int32_t> band_blocks; // 7 ints per block: out lo[3], hi[3], face axis
+  int band_region_cells = 0;       // max SMEM region (cells) of one band block at t = T
+  double flops_per_cell_step = 0;  // algorithmic (unpadded dense-DFT tile)
+  double mma_flops_per_pair = 0;   // executed by the fused kernel (padded)
+  size_t fused_smem = 0;
+};
+
+// Builds the plan; returns 0 or a negative FFTSTENCIL_* code with `err` set.
+int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
+                    HostPlan& p, std::string& err);
+
+// Dense-DFT tile cost model (executed FP64 tensor flops per cell-step) used to pick L/T.
+double model_flops_2d(int L, int S, int T);
+
+}  // namespace fstencil

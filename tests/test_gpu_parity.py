@@ -1,0 +1,200 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Acceptance (BASELINE.json north_star): max|u_gpu - u_oracle| <= 1e-9 * max|u_oracle| in
+FP64 after the full step count.  Inputs are the seeded synthetic recipe of synth/.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from synth import workloads as wl
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-9
+
+
+@pytest.fixture(scope="module")
+def fs():
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    import paper_conf_ppopp_hanlcbzyczcy25_b200 as mod
+    return mod
+
+
+def run_gpu(fs, u0, w, r, T, steps, plan=None):
+    p = plan or fs.Plan(u0.shape, w, r, T)
+    a = torch.from_numpy(u0).cuda()
+    b = torch.empty_like(a)
+    p.run(a, b, steps)
+    torch.cuda.synchronize()
+    return b.cpu().numpy(), p
+
+
+def rel_err(got, ref):
+    return float(np.abs(got - ref).max() / np.abs(ref).max())
+
+
+CASES = [
+    # (extents, shape, r, T, steps, weights kind)
+    ((4096,), "star", 1, 8, 64, "seeded"),       # BASELINE configs[0]
+    ((4096,), "star", 1, 8, 64, "classic"),
+    ((1001,), "star", 2, 5, 13, "seeded"),
+    ((333,), "star", 3, 4, 9, "seeded"),
+    ((67,), "star", 1, 8, 17, "seeded"),
+    ((57,), "star", 1, 3, 1, "seeded"),
+    ((129, 131), "box", 1, 8, 19, "seeded"),
+    ((200, 173), "star", 1, 4, 11, "seeded"),
+    ((97, 101), "star", 3, 4, 11, "seeded"),
+    ((120, 90), "box", 3, 2, 7, "seeded"),
+    ((75, 88), "box", 1, 1, 5, "seeded"),
+    ((150, 140), "box", 1, 16, 35, "seeded"),
+    ((100, 100), "box", 2, 3, 10, "seeded"),
+    ((64, 64), "star", 1, 12, 27, "classic"),
+    ((40, 41), "box", 1, 2, 3, "classic"),
+    ((257, 77), "box", 3, 3, 8, "seeded"),
+]
+
+
+@pytest.mark.parametrize("ext,shape,r,T,steps,kind", CASES)
+def test_parity_vs_oracle(fs, ext, shape, r, T, steps, kind):
+    w = wl.stencil_weights(shape, len(ext), r, kind)
+    u0 = wl.grid(ext, 11)
+    got, p = run_gpu(fs, u0, w, r, T, steps)
+    ref = oracle.stencil_run(u0, w, r, steps)
+    err = rel_err(got, ref)
+    assert err <= TOL, (err, p.info())
+    ring = np.ones(ext, bool)
+    ring[tuple(slice(r, e - r) for e in ext)] = False
+    assert np.array_equal(got[ring], u0[ring])
+
+
+@pytest.mark.parametrize("ext,r,T,steps", [((96, 90), 1, 4, 8), ((96, 90), 1, 4, 12), ((500,), 1, 8, 16),
+                                           ((500,), 1, 8, 24)])
+def test_in_place_aliasing(fs, ext, r, T, steps):
+    w = wl.seeded_weights("box" if len(ext) == 2 else "star", len(ext), r)
+    u0 = wl.grid(ext, 5)
+    p = fs.Plan(ext, w, r, T)
+    a = torch.from_numpy(u0).cuda()
+    p.run(a, a, steps)
+    torch.cuda.synchronize()
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(a.cpu().numpy(), ref) <= TOL
+
+
+def test_zero_steps_copies(fs):
+    u0 = wl.grid((50, 60), 1)
+    got, _ = run_gpu(fs, u0, wl.seeded_weights("box", 2, 1), 1, 4, 0)
+    assert np.array_equal(got, u0)
+
+
+def test_T_invariance(fs):
+    """G4: the same 24 steps with T in {1,2,3,4,6,8,12} agree within tolerance."""
+    ext = (140, 133)
+    w = wl.seeded_weights("box", 2, 1)
+    u0 = wl.grid(ext, 2)
+    ref = oracle.stencil_run(u0, w, 1, 24)
+    for T in (1, 2, 3, 4, 6, 8, 12):
+        got, p = run_gpu(fs, u0, w, 1, T, 24)
+        assert p.info()["T"] == T
+        assert rel_err(got, ref) <= TOL, T
+
+
+def test_semigroup(fs):
+    ext = (111, 123)
+    w = wl.seeded_weights("star", 2, 3)
+    u0 = wl.grid(ext, 3)
+    p = fs.Plan(ext, w, 3, 4)
+    a = torch.from_numpy(u0).cuda()
+    b = torch.empty_like(a)
+    c = torch.empty_like(a)
+    p.run(a, b, 7)
+    p.run(b, c, 9)
+    d = torch.empty_like(a)
+    p.run(a, d, 16)
+    torch.cuda.synchronize()
+    assert rel_err(c.cpu().numpy(), d.cpu().numpy()) <= 1e-12
+
+
+def test_constant_field(fs):
+    u0 = np.full((130, 170), 0.625)
+    got, _ = run_gpu(fs, u0, wl.seeded_weights("box", 2, 1), 1, 8, 40)
+    np.testing.assert_allclose(got, u0, rtol=1e-12)
+
+
+def test_plane_wave_fixed_grid(fs):
+    """G2: away from the fixed ring (distance >= r*steps) a plane wave scales by sigma^steps."""
+    n0, n1, r, steps = 300, 280, 1, 40
+    w = wl.seeded_weights("box", 2, r)
+    th = (2 * np.pi * 5 / n0, 2 * np.pi * 3 / n1)
+    c0, c1 = np.meshgrid(np.arange(n0), np.arange(n1), indexing="ij")
+    u0 = np.cos(th[0] * c0 + th[1] * c1)
+    sig = sum(w[i, j] * np.exp(1j * ((i - r) * th[0] + (j - r) * th[1])) for i in range(3) for j in range(3))
+    got, _ = run_gpu(fs, u0, w, r, 8, steps)
+    m = r * steps + r
+    ref = np.real(sig ** steps * np.exp(1j * (th[0] * c0 + th[1] * c1)))
+    assert np.abs(got[m:-m, m:-m] - ref[m:-m, m:-m]).max() <= 1e-12
+
+
+def test_run_host_matches_device(fs):
+    ext = (90, 70)
+    w = wl.seeded_weights("box", 2, 1)
+    u0 = wl.grid(ext, 8)
+    p = fs.Plan(ext, w, 1, 4)
+    dev, _ = run_gpu(fs, u0, w, 1, 4, 13, plan=p)
+    out = np.empty_like(u0)
+    p.run_host(u0, out, 13)
+    assert np.array_equal(out, dev)
+
+
+def test_invalid_arguments(fs):
+    w = wl.seeded_weights("box", 2, 1)
+    with pytest.raises(fs.FftStencilError):
+        fs.Plan((2, 50), w, 1, 4)
+    p = fs.Plan((50, 50), w, 1, 4)
+    a = torch.zeros((50, 50), dtype=torch.float64, device="cuda")
+    with pytest.raises(fs.FftStencilError):
+        p.run(a, a, -1)
+    with pytest.raises(ValueError):
+        p.run(a, torch.zeros((50, 51), dtype=torch.float64, device="cuda"), 1)
+    with pytest.raises(TypeError):
+        p.run(a.float(), a, 1)
+
+
+def test_launch_count_reported(fs):
+    ext = (200, 200)
+    p = fs.Plan(ext, wl.seeded_weights("box", 2, 1), 1, 8)
+    a = torch.zeros(ext, dtype=torch.float64, device="cuda")
+    b = torch.empty_like(a)
+    p.run(a, b, 20)   # 2 full passes + 1 remainder pass: (fused + band) x 3 + 4 ring boxes
+    assert p.info()["last_run_launches"] == 3 * 2 + 4
+
+
+# ---------------------------------------------------------------- full BASELINE sizes
+@pytest.mark.parametrize("name,T", [("heat2d", 8), ("box2d9p", 8), ("star2d13p", 4), ("box2d49p", 4),
+                                    ("box2d9p", 1), ("heat2d", 16)])
+def test_full_size_sampled(fs, name, T):
+    """10240^2 at parity steps 2T+3 (launch configuration of bench.py); sampled cells
+    (interior, band, ring, tile seams) against the oracle's single-cell evaluation."""
+    wk = wl.CONFIGS[name]
+    w = wk.weights()
+    u0 = wk.grid()
+    steps = 2 * T + 3
+    got, p = run_gpu(fs, u0, w, wk.radius, T, steps)
+    info = p.info()
+    rng = np.random.default_rng(17)
+    n = np.array(wk.extents)
+    cells = [rng.integers(0, n) for _ in range(150)]
+    h, S = info["halo"], info["valid"][0]
+    for k in range(6):       # tile seams, band and ring cells
+        for v in (h + k * S - 1, h + k * S, wk.radius - 1, wk.radius, h - 1, h, n[0] - h, n[0] - h - 1):
+            cells.append(np.array([v, (v * 7 + 13) % n[1]]))
+    cells = np.clip(np.array(cells), 0, n - 1)
+    ref = oracle.stencil_point(u0, w, wk.radius, steps, cells)
+    vals = got[tuple(cells.T)]
+    scale = np.abs(u0).max()
+    assert np.abs(vals - ref).max() <= TOL * scale
+    # invariants over the whole grid: finite, max principle (w >= 0, sum 1)
+    assert np.isfinite(got).all()
+    assert got.min() >= u0.min() - 1e-9 and got.max() <= u0.max() + 1e-9

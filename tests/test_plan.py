@@ -1,0 +1,235 @@
+"""CPU tests of the C-ABI library's host side: symbols, plan builder tables, schedule.
+
+No GPU is needed: libfftstencil.so loads without a device and fftstencil_describe /
+fftstencil_export_aux run the host plan builder only.  The tables are pinned against
+numpy's FFT (an independent route), the oracle's spectrum, and exhaustive coverage
+checks; a numpy model of the fused tile algorithm that consumes the exported tables is
+compared with the direct-stencil oracle.
+"""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import spectrum
+from synth import workloads as wl
+
+fs = pytest.importorskip("paper_conf_ppopp_hanlcbzyczcy25_b200")
+from paper_conf_ppopp_hanlcbzyczcy25_b200 import _native  # noqa: E402
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_library_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "fftstencil.h")).read()
+    declared = set(re.findall(r"\b(fftstencil_[a-z_]+)\s*\(", hdr))
+    assert declared == set(_native.EXPORTS)
+    lib = _native.lib()
+    for name in declared:
+        assert hasattr(lib, name), name
+
+
+def test_describe_rejects_invalid():
+    w = wl.seeded_weights("box", 2, 1)
+    with pytest.raises(fs.FftStencilError):
+        fs.describe((2, 100), w, 1)          # extent <= 2r
+    with pytest.raises(fs.FftStencilError):
+        fs.describe((100, 100), w, 1, T=-1)
+    with pytest.raises(ValueError):
+        fs.describe((100, 100), w.reshape(-1)[:5], 1)
+    bad = w.copy()
+    bad[0] = np.nan
+    with pytest.raises(fs.FftStencilError):
+        fs.describe((100, 100), bad, 1)
+
+
+@pytest.mark.parametrize("r,T,L", [(1, 8, 40), (1, 1, 16), (1, 4, 24), (3, 4, 64)])
+def test_describe_2d_geometry(r, T, L):
+    info = fs.describe((10240, 10240), wl.seeded_weights("box", 2, r), r, T)
+    assert info["T"] == T and info["halo"] == r * T
+    assert info["tile"] == [L, L] and info["valid"] == [L - 2 * r * T] * 2
+    nt = -(-(10240 - 2 * r * T) // (L - 2 * r * T))
+    assert info["tiles"] == nt * nt and info["pairs"] == (nt * nt + 1) // 2
+
+
+def test_describe_auto_T_and_clamping():
+    w = wl.seeded_weights("star", 2, 1)
+    info = fs.describe((10240, 10240), w, 1, 0)
+    assert 1 <= info["T"] <= 16
+    small = fs.describe((20, 20), w, 1, 16)    # 2h < 20 forces T <= 9; tile forces S >= 8
+    assert 2 * small["halo"] < 20 and small["valid"][0] >= 8
+    one = fs.describe((4096,), wl.seeded_weights("star", 1, 1), 1, 8)
+    assert one["tile"] == [56] and one["valid"] == [40] and one["pfa"] == [8, 7]
+
+
+# ---------------------------------------------------------------- P1: DFT matrices
+@pytest.mark.parametrize("L_T", [(16, 1), (40, 8), (64, 12)])
+def test_dft_matrix_vs_numpy(L_T):
+    L, T = L_T
+    w = wl.seeded_weights("box", 2, 1)
+    info = fs.describe((4000, 4000), w, 1, T)
+    assert info["tile"][0] == L
+    v = fs.export_aux((4000, 4000), w, 1, T, which=0, axis=0)
+    F = (v[0::2] + 1j * v[1::2]).reshape(L, L)
+    np.testing.assert_allclose(F, np.fft.fft(np.eye(L), axis=0), atol=1e-14)
+
+
+def test_pfa_dft_matrices_vs_numpy():
+    w = wl.seeded_weights("star", 1, 1)
+    for axis, N in ((0, 8), (1, 7)):
+        v = fs.export_aux((4096,), w, 1, 8, which=0, axis=axis)
+        F = (v[0::2] + 1j * v[1::2]).reshape(N, N)
+        np.testing.assert_allclose(F, np.fft.fft(np.eye(N), axis=0), atol=1e-14)
+
+
+# ---------------------------------------------------------------- P2: powered spectra
+@pytest.mark.parametrize("shape,r,T", [("box", 1, 8), ("star", 3, 4), ("star", 1, 3)])
+def test_spectra_2d_vs_oracle_spectrum(shape, r, T):
+    w = wl.seeded_weights(shape, 2, r)
+    info = fs.describe((5000, 5000), w, r, T)
+    L = info["tile"][0]
+    for t in range(1, info["T"] + 1):
+        v = fs.export_aux((5000, 5000), w, r, T, which=1, t=t)
+        got = (v[0::2] + 1j * v[1::2]).reshape(L, L)
+        ref = spectrum.powered_spectrum(w, r, (L, L), t)
+        np.testing.assert_allclose(got, ref, atol=1e-15)
+
+
+def test_spectrum_1d_ruritanian_vs_numpy_fft():
+    """1D spectrum in Ruritanian order: G[k1][k2] = conj(fft(W_t wrapped))[(8 k2... )]/L."""
+    w = wl.seeded_weights("star", 1, 1)
+    T = 8
+    L, N1, N2 = 56, 8, 7
+    for t in (1, 5, 8):
+        v = fs.export_aux((4096,), w, 1, T, which=1, t=t)
+        G = (v[0::2] + 1j * v[1::2]).reshape(8, 8)
+        Wt = np.ones(1)
+        for _ in range(t):
+            Wt = np.convolve(Wt, w)
+        wrap = np.zeros(L)
+        for i, val in enumerate(Wt):
+            wrap[(i - t) % L] += val
+        ref = np.conj(np.fft.fft(wrap)) / L
+        for k1 in range(N1):
+            for k2 in range(N2):
+                assert abs(G[k1, k2] - ref[(k1 * N2 + k2 * N1) % L]) < 1e-15
+            assert G[k1, 7] == 0
+
+
+# ---------------------------------------------------------------- P3: PFA identity
+def test_pfa_identity_with_exported_maps():
+    """F_N1 . X . F_N2^T with X[l mod 8][l mod 7] = x[l] is fft(x) in Ruritanian order."""
+    w = wl.seeded_weights("star", 1, 1)
+    crt = fs.export_aux((4096,), w, 1, 8, which=3).astype(int).reshape(8, 7)
+    assert sorted(crt.reshape(-1)) == list(range(56))
+    for l1 in range(8):
+        for l2 in range(7):
+            assert crt[l1, l2] % 8 == l1 and crt[l1, l2] % 7 == l2
+    v1 = fs.export_aux((4096,), w, 1, 8, which=0, axis=0)
+    v2 = fs.export_aux((4096,), w, 1, 8, which=0, axis=1)
+    F1 = (v1[0::2] + 1j * v1[1::2]).reshape(8, 8)
+    F2 = (v2[0::2] + 1j * v2[1::2]).reshape(7, 7)
+    x = np.random.default_rng(3).random(56) + 1j * np.random.default_rng(4).random(56)
+    X = x[crt]
+    G = F1 @ X @ F2.T
+    ref = np.fft.fft(x)
+    for k1 in range(8):
+        for k2 in range(7):
+            assert abs(G[k1, k2] - ref[(k1 * 7 + k2 * 8) % 56]) < 1e-12
+
+
+# ---------------------------------------------------------------- P4: coverage
+def _cover(ext, r, T, shape):
+    nd = len(ext)
+    w = wl.seeded_weights(shape, nd, r)
+    info = fs.describe(ext, w, r, T)
+    h = info["halo"]
+    count = np.zeros(ext, dtype=np.int32)
+    tiles = fs.export_aux(ext, w, r, T, which=2).astype(np.int64).reshape(info["tiles"], nd, 3)
+    for t in tiles:
+        sl = tuple(slice(t[a, 1], t[a, 1] + t[a, 2]) for a in range(nd))
+        count[sl] += 1
+    off = 3 - nd
+    for kind in (4, 5):
+        vals = fs.export_aux(ext, w, r, T, which=kind)
+        step = 7 if kind == 4 else 6
+        for b in vals.astype(np.int64).reshape(-1, step):
+            sl = tuple(slice(b[off + a], b[3 + off + a]) for a in range(nd))
+            count[sl] += 1
+            for e in range(off):
+                assert b[e] == 0 and b[3 + e] == 1
+    return count, h
+
+
+@pytest.mark.parametrize("ext,r,T,shape", [((100, 77), 1, 8, "box"), ((33, 41), 3, 2, "star"),
+                                            ((4096,), 1, 8, "star"), ((301,), 2, 5, "star"),
+                                            ((30, 29), 1, 1, "box")])
+def test_tiles_band_ring_partition_grid_exactly(ext, r, T, shape):
+    count, h = _cover(ext, r, T, shape)
+    assert count.min() == 1 and count.max() == 1
+
+
+def test_3d_geometry_partitions_grid():
+    count, h = _cover((20, 23, 19), 1, 2, "box")
+    assert count.min() == 1 and count.max() == 1
+
+
+# ---------------------------------------------------------------- P5: tile algorithm model
+def _model_2d(u, w, r, T, steps):
+    """numpy model of the fused pass as the kernel runs it, fed with the exported tables."""
+    ext = u.shape
+    info = fs.describe(ext, w, r, T)
+    L, S, h, T = info["tile"][0], info["valid"][0], info["halo"], info["T"]
+    v = fs.export_aux(ext, w, r, T, which=0, axis=0)
+    F = (v[0::2] + 1j * v[1::2]).reshape(L, L)
+    tiles = fs.export_aux(ext, w, r, T, which=2).astype(np.int64).reshape(info["tiles"], 2, 3)
+    rings = fs.export_aux(ext, w, r, T, which=5).astype(np.int64).reshape(-1, 6)
+    bands = fs.export_aux(ext, w, r, T, which=4).astype(np.int64).reshape(-1, 7)
+    cur = u.copy()
+    done = 0
+    while done < steps:
+        t = min(T, steps - done)
+        sv = fs.export_aux(ext, w, r, T, which=1, t=t)
+        St = (sv[0::2] + 1j * sv[1::2]).reshape(L, L)
+        nxt = np.full_like(cur, np.nan)
+        for b in rings:
+            sl = (slice(b[1], b[4]), slice(b[2], b[5]))
+            nxt[sl] = cur[sl]
+        pad = np.zeros((ext[0] + L, ext[1] + L))
+        pad[:ext[0], :ext[1]] = cur
+        for i in range(0, len(tiles), 2):
+            pair = tiles[i:i + 2]
+            xa = pad[pair[0, 0, 0]:pair[0, 0, 0] + L, pair[0, 1, 0]:pair[0, 1, 0] + L]
+            xb = pad[pair[1, 0, 0]:pair[1, 0, 0] + L, pair[1, 1, 0]:pair[1, 1, 0] + L] if len(pair) > 1 else 0 * xa
+            Z = F @ (xa + 1j * xb) @ F.T                    # Alg. 1 line 1
+            Z = Z * St                                      # line 2 (Eq. 10)
+            G = np.conj(F)[h:h + S]
+            Y = G @ Z @ G.T                                 # lines 3-4, crop-aware
+            for k, part in enumerate((Y.real, Y.imag)[:len(pair)]):
+                tl = pair[k]
+                n0, n1 = tl[0, 2], tl[1, 2]
+                nxt[tl[0, 1]:tl[0, 1] + n0, tl[1, 1]:tl[1, 1] + n1] = part[:n0, :n1]
+        for b in bands:   # band: t direct steps (model uses the oracle definition)
+            lo, hi = b[1:3], b[4:6]
+            g = r * t
+            rl = np.maximum(lo - g, 0)
+            rh = np.minimum(hi + g, ext)
+            sub = oracle.stencil_run(cur, w, r, t)[lo[0]:hi[0], lo[1]:hi[1]]
+            nxt[lo[0]:hi[0], lo[1]:hi[1]] = sub
+            del rl, rh
+        assert not np.isnan(nxt).any()
+        cur = nxt
+        done += t
+    return cur
+
+
+@pytest.mark.parametrize("ext,shape,r,T,steps", [((61, 70), "box", 1, 4, 11), ((58, 47), "star", 3, 2, 5),
+                                                   ((40, 40), "box", 1, 8, 8)])
+def test_tile_algorithm_model_matches_oracle(ext, shape, r, T, steps):
+    w = wl.seeded_weights(shape, 2, r)
+    u = wl.grid(ext, 99)
+    got = _model_2d(u, w, r, T, steps)
+    ref = oracle.stencil_run(u, w, r, steps)
+    assert np.abs(got - ref).max() <= 1e-12 * np.abs(ref).max()
