@@ -1,0 +1,321 @@
+#!/usr/bin/env python
+"""Benchmark of the B200-native FlashFFTStencil hot path (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload heat2d] [--T 0] [--time-steps 1000]
+
+One bench "step" = one fftstencil_run over the whole grid for `--time-steps` stencil time
+steps (default: PAPER.md Table 3's 1000), i.e. one pass of every §8(a) row: ring copy,
+floor(steps/T) fused FFT-tile passes + band passes, remainder pass.  The metric is
+GStencils/s = cells x time steps / s / 1e9 (reading Q18), FP64.  Inputs are resident in
+HBM for `value`; `e2e` goes through the C ABI's host-buffer entry point
+(fftstencil_run_host) with the H2D/D2H copies inside the timed region.
+
+--impl reference times the CPU oracle (oracle/, the plain direct stencil) on the host
+cores on a bounded sample of the same workload (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth import workloads as wl  # noqa: E402
+
+FP64_PEAK_TFLOPS = 37.18   # measured DMMA.8x8x4 peak on this pool's B200 (profiles/r01_fp64_peak.txt)
+FP64_PEAK_SOURCE = ("measured: tools/fp64_peak.cu DMMA m8n8k4 microbenchmark, 148 SMs x 64 FMA/clk x 1.965 GHz "
+                    "(profiles/r01_fp64_peak.txt); MEASURED_PEAKS.json carries no FP64 figure")
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", default="heat2d", choices=sorted(wl.CONFIGS))
+    ap.add_argument("--T", type=int, default=0, help="fused depth (0 = plan's automatic choice)")
+    ap.add_argument("--time-steps", type=int, default=0, help="stencil time steps per bench step (0 = workload)")
+    ap.add_argument("--weights", default="seeded", choices=["seeded", "classic"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--json-out", default="")
+    return ap.parse_args()
+
+
+def env_rank():
+    return int(os.environ.get("RANK", "0")), int(os.environ.get("LOCAL_RANK", "0")), int(os.environ.get("WORLD_SIZE", "1"))
+
+
+class ClockSampler:
+    """nvidia-smi sampling of SM clocks and throttle reasons during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.lines = []
+        if self.proc is not None:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+                out = ""
+            self.lines = [ln for ln in out.splitlines() if ln.strip()]
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        for ln in getattr(self, "lines", []):
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+            for name, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(name)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def load_traffic(info: dict, workload: str):
+    """DRAM bytes per fused launch from the committed ncu --set full capture, if it matches."""
+    path = os.path.join(ROOT, "profiles", "ncu_fused_traffic.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        e = d.get(workload)
+        if e and e.get("T") == info["T"] and e.get("tile") == info["tile"]:
+            return float(e["dram_bytes_per_launch"])
+    except Exception:
+        pass
+    return None
+
+
+def cpu_oracle_sample(wk, w, budget_s: float = 12.0):
+    """Time the oracle as it stands on the host cores on a bounded sample."""
+    import oracle
+    u = wk.grid()
+    threads = oracle.max_threads()
+    t0 = time.perf_counter()
+    oracle.stencil_run(u, w, wk.radius, 1, nthreads=threads)
+    t1 = time.perf_counter() - t0
+    steps = 1
+    if t1 < budget_s / 2:
+        steps = int(max(1, min(64, budget_s / t1)))
+        t0 = time.perf_counter()
+        oracle.stencil_run(u, w, wk.radius, steps, nthreads=threads)
+        t1 = time.perf_counter() - t0
+    cells = int(np.prod(wk.extents))
+    return {"value": cells * steps / t1 / 1e9, "unit": "GStencils/s", "cores": threads, "kind": "oracle",
+            "sample": f"full {wk.name} grid {'x'.join(map(str, wk.extents))}, {steps} direct time step(s), "
+                      f"{t1:.1f} s wall, OMP threads={threads}"}
+
+
+def run_reference(args):
+    rank, _, world = env_rank()
+    if rank != 0:
+        return 0
+    import oracle
+    wk = wl.CONFIGS[args.workload]
+    w = wk.weights(args.weights)
+    u = wk.grid()
+    threads = oracle.max_threads()
+    cells = int(np.prod(wk.extents))
+    s_ref = 1   # direct time steps per bench step (bounded sample of the 1000-step run)
+    for _ in range(args.warmup):
+        oracle.stencil_run(u, w, wk.radius, s_ref, nthreads=threads)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.stencil_run(u, w, wk.radius, s_ref, nthreads=threads)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    value = cells * s_ref * args.steps / tot / 1e9
+    line = {
+        "impl": "reference", "metric": "GStencils/s FP64", "value": value, "unit": "GStencils/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{wk.name} {'x'.join(map(str, wk.extents))} (BASELINE configs[1])",
+                   "stencil": f"{wk.points}-point {wk.shape} r={wk.radius}, {args.weights} weights",
+                   "time_steps_per_step": s_ref, "sample": "full grid, 1 direct time step per bench step"},
+        "cpu_baseline": {"value": value, "unit": "GStencils/s", "cores": threads, "kind": "oracle",
+                         "sample": f"full grid, {s_ref} direct time step per bench step, {args.steps} timed"},
+        "e2e": {"value": value, "unit": "GStencils/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_hanlcbzyczcy25_b200 as fs
+
+    rank, local, world = env_rank()
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+
+    wk = wl.CONFIGS[args.workload]
+    w = wk.weights(args.weights)
+    steps_per_run = args.time_steps or wk.bench_steps
+    u0 = wk.grid()
+    cells = int(np.prod(wk.extents))
+
+    plan = fs.Plan(wk.extents, w, wk.radius, args.T)
+    info = plan.info()
+    d_in = torch.from_numpy(u0).to(dev)
+    d_out = torch.empty_like(d_in)
+    stream = torch.cuda.current_stream(dev)
+
+    def barrier():
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+
+    for _ in range(max(args.warmup, 0)):
+        plan.run(d_in, d_out, steps_per_run, stream)
+    barrier()
+
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    plan.set_profiling(True)
+    with ClockSampler(dev.index) as clk:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            plan.run(d_in, d_out, steps_per_run, stream)
+        ev1.record(stream)
+        barrier()
+    prof = plan.profile_read()
+    plan.set_profiling(False)
+    launches_per_run = plan.info()["last_run_launches"]
+    ms = ev0.elapsed_time(ev1)
+    ms_t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms_max = float(ms_t.item())
+    value = world * cells * steps_per_run * args.steps / (ms_max / 1e3) / 1e9
+
+    # ---- roofline of the dominant kernel (the fused FFT-tile kernel) ----
+    h = info["halo"]
+    exact = 1
+    for e in wk.extents:
+        exact *= max(0, e - 2 * h)
+    fl = max(1, prof["fused_launches"])
+    fused_avg_s = prof["fused_ms"] / fl / 1e3
+    alg_flops_launch = info["flops_per_cell_step"] * exact * info["T"]
+    achieved = alg_flops_launch / fused_avg_s / 1e12
+    traffic = load_traffic(info, args.workload)
+    roofline = {"bound": "tensor", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
+                "frac": achieved / FP64_PEAK_TFLOPS, "traffic": traffic,
+                "kernel": f"fft2d_kernel<{info['tile'][0]}>" if info["ndim"] == 2 else "fft1d_kernel",
+                "dtype": "f64 (DMMA.8x8x4)", "peak_source": FP64_PEAK_SOURCE,
+                "alg_flops_per_launch": alg_flops_launch,
+                "flops_per_cell_step": info["flops_per_cell_step"],
+                "mma_flops_per_launch": info["mma_flops_per_pass"],
+                "mma_tflops": info["mma_flops_per_pass"] / fused_avg_s / 1e12,
+                "fused_ms_avg": fused_avg_s * 1e3, "fused_share_of_step": prof["fused_ms"] / max(ms, 1e-9),
+                "band_ms_avg": prof["band_ms"] / max(1, prof["band_launches"])}
+
+    # ---- end to end through the host-buffer C-ABI entry point ----
+    e2e = None
+    if not args.no_e2e:
+        h_in = torch.from_numpy(u0).pin_memory()
+        h_out = torch.empty_like(h_in).pin_memory()
+        plan.run_host(h_in, h_out, steps_per_run, stream)
+        k_e = max(1, min(args.steps, 3))
+        barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(k_e):
+            plan.run_host(h_in, h_out, steps_per_run, stream)
+        e1.record(stream)
+        barrier()
+        ems = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(ems, op=dist.ReduceOp.MAX)
+        e_ms = float(ems.item())
+        e2e = {"value": world * cells * steps_per_run * k_e / (e_ms / 1e3) / 1e9, "unit": "GStencils/s",
+               "h2d_bytes_per_step": int(u0.nbytes), "d2h_bytes_per_step": int(u0.nbytes),
+               "steps": k_e, "ms_per_step": e_ms / k_e, "api": "fftstencil_run_host (pinned host buffers)"}
+        if not np.isfinite(h_out.numpy()).all():
+            raise RuntimeError("non-finite output")
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_oracle_sample(wk, w)
+
+    if rank == 0:
+        line = {
+            "metric": "GStencils/s FP64", "value": value, "unit": "GStencils/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": f"{wk.name} {'x'.join(map(str, wk.extents))}"
+                                   + (" (BASELINE configs[1])" if args.workload in ("heat2d", "box2d9p") else ""),
+                       "stencil": f"{wk.points}-point {wk.shape} r={wk.radius}, {args.weights} weights (seed 20250301)",
+                       "grid": list(wk.extents), "time_steps_per_step": steps_per_run, "T": info["T"],
+                       "tile": info["tile"], "valid": info["valid"],
+                       "parallelism": "single GPU" if world == 1 else f"{world} independent replicas (weak)",
+                       "l2": f"inputs {u0.nbytes / 1e6:.0f} MB > 126 MB L2 (no flush needed)"},
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": int(launches_per_run * args.steps),
+            "clocks": clk.summary(),
+        }
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.json_out:
+            with open(args.json_out, "w") as f:
+                f.write(s + "\n")
+    plan.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -105,6 +105,15 @@ void fftstencil_destroy(fftstencil_plan* plan);
 /* Plan geometry and cost model. */
 int fftstencil_plan_info(const fftstencil_plan* plan, fftstencil_info* info);
 
+/* Per-kernel timing for roofline reporting.  With profiling enabled, fftstencil_run
+ * records a CUDA event pair on its stream around every fused FFT-tile launch and every
+ * band launch (event overhead only; no synchronisation).  fftstencil_profile_read waits
+ * for the recorded events, returns the summed device milliseconds and launch counts since
+ * the last read (any pointer may be NULL), and resets the accumulators. */
+int fftstencil_set_profiling(fftstencil_plan* plan, int enable);
+int fftstencil_profile_read(fftstencil_plan* plan, double* fused_ms, int64_t* fused_launches,
+                            double* band_ms, int64_t* band_launches);
+
 /* Thread-local description of the last failure; "" after a successful call. */
 const char* fftstencil_last_error(void);
 

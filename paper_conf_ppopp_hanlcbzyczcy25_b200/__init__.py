@@ -103,6 +103,20 @@ class Plan:
             raise FftStencilError(rc, last_error())
         return info.as_dict()
 
+    def set_profiling(self, enable: bool) -> None:
+        rc = self._lib.fftstencil_set_profiling(self._h, int(bool(enable)))
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+
+    def profile_read(self) -> dict:
+        fm, bm = ctypes.c_double(), ctypes.c_double()
+        fl, bl = ctypes.c_int64(), ctypes.c_int64()
+        rc = self._lib.fftstencil_profile_read(self._h, ctypes.byref(fm), ctypes.byref(fl), ctypes.byref(bm),
+                                               ctypes.byref(bl))
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+        return {"fused_ms": fm.value, "fused_launches": fl.value, "band_ms": bm.value, "band_launches": bl.value}
+
     # -- execution --
     def _check_dev(self, t, name):
         import torch

@@ -17,7 +17,8 @@ CODES = {OK: "OK", EINVAL: "EINVAL", ENOMEM: "ENOMEM", ECUDA: "ECUDA", ENCCL: "E
 
 # every symbol include/fftstencil.h declares
 EXPORTS = ("fftstencil_plan_create", "fftstencil_run", "fftstencil_run_host", "fftstencil_destroy",
-           "fftstencil_plan_info", "fftstencil_last_error", "fftstencil_describe", "fftstencil_export_aux")
+           "fftstencil_plan_info", "fftstencil_last_error", "fftstencil_describe", "fftstencil_export_aux",
+           "fftstencil_set_profiling", "fftstencil_profile_read")
 
 
 class Info(ctypes.Structure):
@@ -86,6 +87,10 @@ def lib():
     L.fftstencil_export_aux.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                         ctypes.c_int, ctypes.c_int, dp, ctypes.c_int64]
     L.fftstencil_export_aux.restype = ctypes.c_int64
+    L.fftstencil_set_profiling.argtypes = [vp, ctypes.c_int]
+    L.fftstencil_set_profiling.restype = ctypes.c_int
+    L.fftstencil_profile_read.argtypes = [vp, dp, i64p, dp, i64p]
+    L.fftstencil_profile_read.restype = ctypes.c_int
     _lib = L
     return L
 

@@ -27,11 +27,6 @@ thread_local std::string g_last_error;
 void set_error(const std::string& s) { g_last_error = s; }
 void clear_error() { g_last_error.clear(); }
 
-struct DevBuf {
-  void* p = nullptr;
-  size_t bytes = 0;
-};
-
 }  // namespace
 
 struct fftstencil_plan {
@@ -52,6 +47,11 @@ struct fftstencil_plan {
   int fused_grid = 0;
   size_t band_smem = 0;
   int64_t last_launches = 0;
+  // profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run()
+  bool profiling = false;
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<int> ev_kind;
+  size_t ev_used = 0;
 };
 
 namespace {
@@ -77,6 +77,7 @@ void free_plan(fftstencil_plan* p) {
   int cur = 0;
   cudaGetDevice(&cur);
   cudaSetDevice(p->device);
+  for (cudaEvent_t ev : p->ev_pool) cudaEventDestroy(ev);
   cudaFree(p->dF);
   cudaFree(p->dS);
   cudaFree(p->dCrt);
@@ -107,6 +108,28 @@ void fill_info(const HostPlan& hp, fftstencil_info* info) {
   info->smem_bytes = hp.fused_smem;
 }
 
+// Profiling: a (start, end) event pair around one launch; returns the pair index or -1.
+long prof_begin(fftstencil_plan* p, int kind, cudaStream_t s) {
+  if (!p->profiling) return -1;
+  if (p->ev_used + 2 > p->ev_pool.size()) {
+    for (int i = 0; i < 64; ++i) {
+      cudaEvent_t ev;
+      if (cudaEventCreate(&ev) != cudaSuccess) return -1;
+      p->ev_pool.push_back(ev);
+    }
+    p->ev_kind.resize(p->ev_pool.size() / 2, 0);
+  }
+  const size_t i = p->ev_used;
+  p->ev_used += 2;
+  p->ev_kind[i / 2] = kind;
+  cudaEventRecord(p->ev_pool[i], s);
+  return (long)i;
+}
+
+void prof_end(fftstencil_plan* p, long i, cudaStream_t s) {
+  if (i >= 0) cudaEventRecord(p->ev_pool[(size_t)i + 1], s);
+}
+
 // One fused pass: src -> dst with t steps (t <= T), tile geometry of T.
 int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s) {
   const HostPlan& hp = p->hp;
@@ -128,7 +151,9 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
     a.Sre = Sre;
     a.Sim = Sim;
+    const long pe = prof_begin(p, 0, s);
     e = launch_fused2d(hp.L[0], a, p->fused_grid, s);
+    prof_end(p, pe, s);
   } else if (hp.ndim == 1) {
     Fft1dArgs a;
     a.src = src;
@@ -144,7 +169,9 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     a.Sre = Sre;
     a.Sim = Sim;
     a.crt = p->dCrt;
+    const long pe = prof_begin(p, 0, s);
     e = launch_fused1d(a, p->fused_grid, s);
+    prof_end(p, pe, s);
   } else {
     set_error("3D fused kernel not available in this build");
     return FFTSTENCIL_EUNSUPPORTED;
@@ -162,7 +189,9 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     b.w = p->dW;
     b.blocks = p->dBlocks;
     b.nblocks = nb;
+    const long pb = prof_begin(p, 1, s);
     e = launch_band(b, p->band_smem, s);
+    prof_end(p, pb, s);
     if (e != cudaSuccess) return cuda_fail(e, "band launch");
     ++p->last_launches;
   }
@@ -426,6 +455,38 @@ int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, i
 }
 
 void fftstencil_destroy(fftstencil_plan* p) { free_plan(p); }
+
+int fftstencil_set_profiling(fftstencil_plan* p, int enable) {
+  if (!p) { set_error("plan must be non-NULL"); return FFTSTENCIL_EINVAL; }
+  p->profiling = enable != 0;
+  p->ev_used = 0;
+  clear_error();
+  return FFTSTENCIL_OK;
+}
+
+int fftstencil_profile_read(fftstencil_plan* p, double* fused_ms, int64_t* fused_launches, double* band_ms,
+                            int64_t* band_launches) {
+  if (!p) { set_error("plan must be non-NULL"); return FFTSTENCIL_EINVAL; }
+  double ms[2] = {0.0, 0.0};
+  int64_t cnt[2] = {0, 0};
+  for (size_t i = 0; i < p->ev_used; i += 2) {
+    cudaError_t e = cudaEventSynchronize(p->ev_pool[i + 1]);
+    if (e != cudaSuccess) return cuda_fail(e, "profiling event");
+    float v = 0.f;
+    e = cudaEventElapsedTime(&v, p->ev_pool[i], p->ev_pool[i + 1]);
+    if (e != cudaSuccess) return cuda_fail(e, "profiling elapsed time");
+    const int k = p->ev_kind[i / 2];
+    ms[k] += v;
+    cnt[k] += 1;
+  }
+  p->ev_used = 0;
+  if (fused_ms) *fused_ms = ms[0];
+  if (fused_launches) *fused_launches = cnt[0];
+  if (band_ms) *band_ms = ms[1];
+  if (band_launches) *band_launches = cnt[1];
+  clear_error();
+  return FFTSTENCIL_OK;
+}
 
 int fftstencil_plan_info(const fftstencil_plan* p, fftstencil_info* info) {
   if (!p || !info) { set_error("plan and info must be non-NULL"); return FFTSTENCIL_EINVAL; }
