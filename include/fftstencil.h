@@ -125,8 +125,9 @@ int fftstencil_describe(int ndim, const int64_t* extents, const double* weights,
 /* Export the host plan's auxiliary tables, for tests of the plan builder:
  *   which = 0: forward DFT matrix of axis `axis` (1D: axis 0 -> F_N1, axis 1 -> F_N2),
  *              row-major L x L complex as interleaved (re, im) pairs, 2*L*L doubles;
- *   which = 1: powered spectrum S_t (t = `t`, 1..T) in the kernel's order (2D/3D:
- *              natural k order; 1D: N1 x N2 matrix in the Ruritanian order of Eq. 8),
+ *   which = 1: powered spectrum S_t (t = `t`, 1..T) in the kernel's order (2D:
+ *              natural [k0][k1]; 3D: [k1][k2][k0]; 1D: N1 x N2 matrix in the Ruritanian
+ *              order of Eq. 8),
  *              2*prod(tile) doubles (interleaved complex);
  *   which = 2: tile origins / ownership: for each tile (row-major tile order), per
  *              axis: origin, first owned cell, owned count -> 3*ndim*tiles int64

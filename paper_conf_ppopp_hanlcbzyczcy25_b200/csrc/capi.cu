@@ -173,8 +173,25 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     e = launch_fused1d(a, p->fused_grid, s);
     prof_end(p, pe, s);
   } else {
-    set_error("3D fused kernel not available in this build");
-    return FFTSTENCIL_EUNSUPPORTED;
+    Fft3dArgs a;
+    a.src = src;
+    a.dst = dst;
+    a.n0 = hp.ext[0];
+    a.n1 = hp.ext[1];
+    a.n2 = hp.ext[2];
+    a.h = hp.h;
+    a.S = hp.S[0];
+    a.nt1 = hp.nt[1];
+    a.nt2 = hp.nt[2];
+    a.ntiles = hp.tiles;
+    a.npairs = hp.pairs;
+    a.Fre = p->dF;
+    a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
+    a.Sre = Sre;
+    a.Sim = Sim;
+    const long pe = prof_begin(p, 0, s);
+    e = launch_fused3d(a, p->fused_grid, s);
+    prof_end(p, pe, s);
   }
   if (e != cudaSuccess) return cuda_fail(e, "fused FFT-tile launch");
   ++p->last_launches;
@@ -305,11 +322,6 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
   int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err);
   if (rc != FFTSTENCIL_OK) { set_error(err); delete p; return nullptr; }
   HostPlan& hp = p->hp;
-  if (hp.ndim == 3) {
-    set_error("3D fused kernel not available in this build");
-    delete p;
-    return nullptr;
-  }
   cudaError_t e = cudaGetDevice(&p->device);
   if (e != cudaSuccess) { cuda_fail(e, "cudaGetDevice"); delete p; return nullptr; }
   e = cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
@@ -350,6 +362,12 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
     e = fused2d_configure(hp.L[0], &occ);
     if (e != cudaSuccess) { cuda_fail(e, "fused 2D kernel configuration"); free_plan(p); return nullptr; }
     if (occ < 1) { set_error("fused 2D kernel cannot be resident"); free_plan(p); return nullptr; }
+    const int64_t want = (int64_t)p->sm_count * occ;
+    p->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, hp.pairs));
+  } else if (hp.ndim == 3) {
+    e = fused3d_configure(&occ);
+    if (e != cudaSuccess) { cuda_fail(e, "fused 3D kernel configuration"); free_plan(p); return nullptr; }
+    if (occ < 1) { set_error("fused 3D kernel cannot be resident"); free_plan(p); return nullptr; }
     const int64_t want = (int64_t)p->sm_count * occ;
     p->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, hp.pairs));
   } else {

@@ -35,6 +35,20 @@ struct Fft1dArgs {
   const int* crt;        // 64: tile position stored at (l1, l2), -1 = padding
 };
 
+// One fused pass of the 3D path over every tile pair (kernel_fft3d.cu); 16^3 tiles.
+struct Fft3dArgs {
+  const double* src;
+  double* dst;
+  int64_t n0, n1, n2;
+  int h, S;
+  int64_t nt1, nt2;      // tiles along axes 1 and 2
+  int64_t ntiles, npairs;
+  const double* Fre;     // 16 x 16 forward DFT matrix
+  const double* Fim;
+  const double* Sre;     // powered spectrum in [k1][k2][k0] order
+  const double* Sim;
+};
+
 // Direct T-step recomputation of the boundary band (kernel_band.cu).
 struct BandArgs {
   const double* src;
@@ -64,6 +78,10 @@ cudaError_t launch_fused2d(int L, const Fft2dArgs& a, int grid, cudaStream_t s);
 constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused1d(const Fft1dArgs& a, int grid, cudaStream_t s);
+
+size_t fused3d_smem();
+cudaError_t fused3d_configure(int* max_blocks_per_sm);
+cudaError_t launch_fused3d(const Fft3dArgs& a, int grid, cudaStream_t s);
 
 constexpr int kBandThreads = 256;
 cudaError_t band_configure(size_t smem);

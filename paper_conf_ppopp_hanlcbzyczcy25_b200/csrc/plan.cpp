@@ -181,7 +181,11 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         (24.0 * l * l * l * l + 6.0 * l * l * l + 8.0 * l * (S * l * l + S * S * l + S * S * S)) /
         (2.0 * S * S * S * bestT);
     const double Sp = round8(p.S[0]);
-    p.mma_flops_per_pair = 24.0 * l * l * l * l + 8.0 * Sp * l * l * l + 8.0 * Sp * Sp * l * l + 8.0 * Sp * Sp * Sp * l;
+    // executed DMMAs per pair (kernel_fft3d.cu): phase 1 16 slices x 128, phase 2 32 row
+    // blocks x (32 + 16 Sp/8), phase 3 S slices x (64 Sp/8 + 16 (Sp/8)^2)
+    const double mt = Sp / 8.0;
+    p.mma_flops_per_pair = 512.0 * (16 * 128 + 32 * (32 + 16 * mt) + S * (64 * mt + 16 * mt * mt));
+    p.fused_smem = (size_t)(2 * 16 * 20 + 2 * 16 * (16 * 20 + 4)) * sizeof(double);
   }
 
   // ---- overlap-save schedule (Eq. 3 / Eq. 4 / Eq. 7; reading Q4: centred window) ----
@@ -248,8 +252,15 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         cplx v(1.0, 0.0);
         for (int s = 0; s < t; ++s) v *= sig[i];
         v /= (double)vol;
-        re[i] = v.real();
-        im[i] = v.imag();
+        // 2D: natural [k0][k1].  3D: [k1][k2][k0] -- the 3D kernel multiplies in C fragments
+        // whose two adjacent columns are consecutive k0 (kernel_fft3d.cu phase 2).
+        int64_t dst = i;
+        if (ndim == 3) {
+          const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
+          dst = k12 * L + k0;
+        }
+        re[dst] = v.real();
+        im[dst] = v.imag();
       }
     }
   }

@@ -54,6 +54,14 @@ CASES = [
     ((64, 64), "star", 1, 12, 27, "classic"),
     ((40, 41), "box", 1, 2, 3, "classic"),
     ((257, 77), "box", 3, 3, 8, "seeded"),
+    ((20, 23, 19), "box", 1, 2, 5, "seeded"),
+    ((24, 30, 28), "star", 1, 2, 7, "seeded"),
+    ((33, 17, 25), "box", 1, 1, 3, "seeded"),
+    ((40, 40, 40), "star", 1, 3, 7, "classic"),
+    ((36, 29, 31), "box", 2, 3, 7, "seeded"),
+    ((30, 30, 30), "star", 1, 4, 9, "seeded"),
+    ((25, 26, 27), "box", 3, 2, 4, "seeded"),
+    ((45, 38, 41), "box", 1, 2, 2, "classic"),
 ]
 
 
@@ -148,6 +156,20 @@ def test_run_host_matches_device(fs):
     assert np.array_equal(out, dev)
 
 
+def test_3d_T_invariance_and_constant(fs):
+    ext = (34, 31, 29)
+    w = wl.seeded_weights("star", 3, 1)
+    u0 = wl.grid(ext, 21)
+    ref = oracle.stencil_run(u0, w, 1, 12)
+    for T in (1, 2, 3, 4, 6):
+        got, p = run_gpu(fs, u0, w, 1, T, 12)
+        assert p.info()["T"] == T
+        assert rel_err(got, ref) <= TOL, T
+    c = np.full(ext, 1.75)
+    got, _ = run_gpu(fs, c, wl.seeded_weights("box", 3, 1), 1, 2, 9)
+    np.testing.assert_allclose(got, c, rtol=1e-12)
+
+
 def test_invalid_arguments(fs):
     w = wl.seeded_weights("box", 2, 1)
     with pytest.raises(fs.FftStencilError):
@@ -196,5 +218,31 @@ def test_full_size_sampled(fs, name, T):
     scale = np.abs(u0).max()
     assert np.abs(vals - ref).max() <= TOL * scale
     # invariants over the whole grid: finite, max principle (w >= 0, sum 1)
+    assert np.isfinite(got).all()
+    assert got.min() >= u0.min() - 1e-9 and got.max() <= u0.max() + 1e-9
+
+
+@pytest.mark.parametrize("name,T", [("heat3d", 2), ("box3d27p", 2), ("heat3d", 1), ("box3d27p", 3)])
+def test_full_size_3d_sampled(fs, name, T):
+    """1024^3 at parity steps 2T+3; sampled cells against the single-cell oracle."""
+    wk = wl.CONFIGS[name]
+    w = wk.weights()
+    u0 = wk.grid()
+    steps = 2 * T + 3
+    got, p = run_gpu(fs, u0, w, wk.radius, T, steps)
+    info = p.info()
+    rng = np.random.default_rng(23)
+    n = np.array(wk.extents)
+    cells = [rng.integers(0, n) for _ in range(120)]
+    h, S = info["halo"], info["valid"][0]
+    for k in range(4):
+        for v in (h + k * S - 1, h + k * S, 0, 1, h - 1, h, n[0] - h, n[0] - 1):
+            cells.append(np.array([v, (v * 7 + 13) % n[1], (v * 3 + 5) % n[2]]))
+            cells.append(np.array([(v * 5 + 1) % n[0], v, (v * 11 + 2) % n[2]]))
+            cells.append(np.array([(v * 5 + 1) % n[0], (v * 3 + 9) % n[1], v]))
+    cells = np.clip(np.array(cells), 0, n - 1)
+    ref = oracle.stencil_point(u0, w, wk.radius, steps, cells)
+    vals = got[tuple(cells.T)]
+    assert np.abs(vals - ref).max() <= TOL * np.abs(u0).max()
     assert np.isfinite(got).all()
     assert got.min() >= u0.min() - 1e-9 and got.max() <= u0.max() + 1e-9
