@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -45,6 +46,7 @@ struct fftstencil_plan {
   size_t grid_cells = 0;
   size_t device_bytes = 0;
   int fused_grid = 0;
+  int variant = 0;            // fused-kernel variant (2D)
   size_t band_smem = 0;
   int64_t last_launches = 0;
   // profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run()
@@ -152,7 +154,7 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     a.Sre = Sre;
     a.Sim = Sim;
     const long pe = prof_begin(p, 0, s);
-    e = launch_fused2d(hp.L[0], a, p->fused_grid, s);
+    e = launch_fused2d(hp.L[0], p->variant, a, p->fused_grid, s);
     prof_end(p, pe, s);
   } else if (hp.ndim == 1) {
     Fft1dArgs a;
@@ -330,6 +332,15 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
   size_t acc = 0;
   std::vector<double> F(hp.Fre);
   F.insert(F.end(), hp.Fim.begin(), hp.Fim.end());
+  if (hp.ndim == 2) {
+    // the 2D kernel reads F with columns permuted within groups of 8 (device_common.cuh)
+    const int L = hp.L[0];
+    for (int plane = 0; plane < 2; ++plane)
+      for (int r = 0; r < L; ++r)
+        for (int c = 0; c < L; ++c)
+          F[(size_t)plane * L * L + (size_t)r * L + ((c & ~7) | ((c & 1) << 2) | ((c & 7) >> 1))] =
+              (plane ? hp.Fim : hp.Fre)[(size_t)r * L + c];
+  }
   p->spec_vol = hp.Sre[0].size();
   std::vector<double> Sv;
   Sv.reserve((size_t)hp.T * 2 * p->spec_vol);
@@ -359,7 +370,11 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
 
   int occ = 0;
   if (hp.ndim == 2) {
-    e = fused2d_configure(hp.L[0], &occ);
+    // double-buffered prefetch pays only where it does not cost occupancy (profiles/r01_variants.txt)
+    p->variant = hp.L[0] >= 56 ? 1 : 0;
+    if (const char* v = std::getenv("FFTSTENCIL_VARIANT")) p->variant = std::atoi(v);
+    if (p->variant < 0 || p->variant > 2) { set_error("FFTSTENCIL_VARIANT must be 0, 1 or 2"); free_plan(p); return nullptr; }
+    e = fused2d_configure(hp.L[0], p->variant, &occ);
     if (e != cudaSuccess) { cuda_fail(e, "fused 2D kernel configuration"); free_plan(p); return nullptr; }
     if (occ < 1) { set_error("fused 2D kernel cannot be resident"); free_plan(p); return nullptr; }
     const int64_t want = (int64_t)p->sm_count * occ;

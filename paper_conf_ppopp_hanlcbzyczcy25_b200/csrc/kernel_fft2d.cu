@@ -17,6 +17,13 @@
 // in M3/M4 an output stripe of axis 1.  M1->M2 and M3->M4 chain C fragments straight into
 // B fragments (Swizzling Fragments, L266-L272); the only shared-memory round trip is the
 // transposition of ownership between the forward and inverse halves.
+//
+// Variants (template V, selected by the plan; FFTSTENCIL_VARIANT overrides for ablations):
+//   V = 0  single pair buffer, synchronous loads, F in shared memory (first version)
+//   V = 1  double-buffered pair: the next pair is fetched with cp.async (zero-fill OOB)
+//          while the inverse half (M3/M4) of the current pair runs; F in shared memory
+//   V = 2  as V = 1 but F is read through L1 (column-permuted copy in HBM), so a CTA's
+//          shared memory is just the two pair buffers (more CTAs per SM)
 #include "device_common.cuh"
 #include "kernels.cuh"
 
@@ -26,51 +33,90 @@ namespace {
 using dev::dmma;
 using dev::perm8;
 
-template <int L>
+__device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
+template <int L, bool ASYNC>
+__device__ __forceinline__ void load_pair(double* sXa, double* sXb, const Fft2dArgs& a, int64_t p, int tid) {
+  constexpr int LD = L + 4, NTHR = L * 4;
+#pragma unroll
+  for (int t = 0; t < 2; ++t) {
+    const int64_t tile = 2 * p + t;
+    double* sX = t ? sXb : sXa;
+    const bool have = tile < a.ntiles;
+    int64_t o0 = 0, o1 = 0;
+    if (have) {
+      const int64_t t0 = tile / a.nt1;
+      o0 = t0 * a.S;
+      o1 = (tile - t0 * a.nt1) * a.S;
+    }
+    for (int e = tid; e < L * L; e += NTHR) {
+      const int r = e / L, c = e - r * L;
+      const int64_t gr = o0 + r, gc = o1 + c;
+      const bool valid = have && gr < a.n0 && gc < a.n1;
+      double* dst = sX + r * LD + perm8(c);
+      if (ASYNC) {
+        cp_async8(dst, valid ? a.src + gr * a.n1 + gc : a.src, valid);
+      } else {
+        *dst = valid ? __ldg(a.src + gr * a.n1 + gc) : 0.0;
+      }
+    }
+  }
+}
+
+template <bool GLOBAL>
+__device__ __forceinline__ double ldF(const double* p) {
+  if (GLOBAL) return __ldg(p);
+  return *p;
+}
+
+template <int L, int V>
 __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
   constexpr int NT = L / 8;      // 8x8 tiles per side == warps
   constexpr int LD = L + 4;      // padded row stride (doubles): 8-bank shift per row
+  constexpr int NTHR = L * 4;
+  constexpr bool FSM = V != 2;   // F in shared memory
+  constexpr bool DB = V != 0;    // double-buffered pair with cp.async prefetch
+  constexpr int FLD = FSM ? LD : L;
   extern __shared__ __align__(16) double smem[];
-  double* sFr = smem;
-  double* sFi = sFr + L * LD;
-  double* sXa = sFi + L * LD;    // tile 2p (real part) ... later Q' real part
-  double* sXb = sXa + L * LD;    // tile 2p+1 (imag part) ... later Q' imag part
-
+  double* sbuf = smem + (FSM ? 2 * L * LD : 0);
+  const double* Fr;
+  const double* Fi;
   const int tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31, g = lane >> 2, q = lane & 3;
-  constexpr int NTHR = L * 4;
-
-  for (int e = tid; e < L * L; e += NTHR) {
-    const int r = e / L, c = e - r * L;
-    sFr[r * LD + perm8(c)] = a.Fre[e];
-    sFi[r * LD + perm8(c)] = a.Fim[e];
+  if (FSM) {
+    double* sFr = smem;
+    double* sFi = sFr + L * LD;
+    for (int e = tid; e < L * L; e += NTHR) {
+      const int r = e / L, c = e - r * L;     // a.Fre is already column-permuted
+      sFr[r * LD + c] = a.Fre[e];
+      sFi[r * LD + c] = a.Fim[e];
+    }
+    Fr = sFr;
+    Fi = sFi;
+  } else {
+    Fr = a.Fre;
+    Fi = a.Fim;
   }
   const int S = a.S, h = a.h;
   const int MT = (S + 7) >> 3;   // output 8-tiles per axis (S padded to 8)
+  int cur = 0;
 
+  if (DB && blockIdx.x < a.npairs) {
+    load_pair<L, true>(sbuf, sbuf + L * LD, a, blockIdx.x, tid);
+    cp_async_commit();
+    cp_async_wait_all();
+  }
   for (int64_t p = blockIdx.x; p < a.npairs; p += gridDim.x) {
-    __syncthreads();
-    // ---- load the halo'd pair (coalesced along axis 1; OOB = 0) ----
-#pragma unroll
-    for (int t = 0; t < 2; ++t) {
-      const int64_t tile = 2 * p + t;
-      double* sX = t ? sXb : sXa;
-      if (tile < a.ntiles) {
-        const int64_t t0 = tile / a.nt1, t1 = tile - t0 * a.nt1;
-        const int64_t o0 = t0 * S, o1 = t1 * S;
-        for (int e = tid; e < L * L; e += NTHR) {
-          const int r = e / L, c = e - r * L;
-          const int64_t gr = o0 + r, gc = o1 + c;
-          double v = 0.0;
-          if (gr < a.n0 && gc < a.n1) v = __ldg(a.src + gr * a.n1 + gc);
-          sX[r * LD + perm8(c)] = v;
-        }
-      } else {
-        for (int e = tid; e < L * L; e += NTHR) {
-          const int r = e / L, c = e - r * L;
-          sX[r * LD + perm8(c)] = 0.0;
-        }
-      }
+    double* sXa = sbuf + cur * 2 * L * LD;   // tile 2p (real part) ... later Q' real part
+    double* sXb = sXa + L * LD;              // tile 2p+1 (imag part) ... later Q' imag part
+    if (!DB) {
+      __syncthreads();
+      load_pair<L, false>(sXa, sXb, a, p, tid);
     }
     __syncthreads();
 
@@ -79,12 +125,12 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
 #pragma unroll
     for (int i = 0; i < NT; ++i) Pr[i][0] = Pr[i][1] = Pi[i][0] = Pi[i][1] = 0.0;
     {
-      const double* fr = sFr + (8 * warp + g) * LD + q;
-      const double* fi = sFi + (8 * warp + g) * LD + q;
+      const double* fr = Fr + (8 * warp + g) * FLD + q;
+      const double* fi = Fi + (8 * warp + g) * FLD + q;
 #pragma unroll
       for (int kc = 0; kc < L / 4; ++kc) {
         const int pc = 4 * kc;
-        const double ar = fr[pc], ai = fi[pc], nai = -ai;
+        const double ar = ldF<!FSM>(fr + pc), ai = ldF<!FSM>(fi + pc), nai = -ai;
 #pragma unroll
         for (int nt = 0; nt < NT; ++nt) {
           const double br = sXa[(8 * nt + g) * LD + q + pc];
@@ -108,8 +154,8 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
         const int pc = 8 * kg + 4 * j + q;
 #pragma unroll
         for (int mt = 0; mt < NT; ++mt) {
-          const double ar = sFr[(8 * mt + g) * LD + pc];
-          const double ai = sFi[(8 * mt + g) * LD + pc];
+          const double ar = ldF<!FSM>(Fr + (8 * mt + g) * FLD + pc);
+          const double ai = ldF<!FSM>(Fi + (8 * mt + g) * FLD + pc);
           dmma(Qr[mt], ar, br);
           dmma(Qr[mt], -ai, bi);
           dmma(Qi[mt], ar, bi);
@@ -139,6 +185,15 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
         sXb[idx] = Qi[mt][j];
       }
     __syncthreads();
+    // ---- prefetch the next pair into the other buffer while the inverse half runs ----
+    if (DB) {
+      const int64_t pn = p + gridDim.x;
+      if (pn < a.npairs) {
+        double* nb = sbuf + (cur ^ 1) * 2 * L * LD;
+        load_pair<L, true>(nb, nb + L * LD, a, pn, tid);
+      }
+      cp_async_commit();
+    }
 
     if (warp < MT) {
       // ---- M3: R[l1 stripe][k0] = sum_k1 conj(F)[h+l1][k1] Q'[k0][k1] (B from shared) ----
@@ -147,12 +202,12 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
       for (int i = 0; i < NT; ++i) Rr[i][0] = Rr[i][1] = Ri[i][0] = Ri[i][1] = 0.0;
       {
         const int arow = min(h + 8 * warp + g, L - 1);   // rows past S are padding
-        const double* fr = sFr + arow * LD + q;
-        const double* fi = sFi + arow * LD + q;
+        const double* fr = Fr + arow * FLD + q;
+        const double* fi = Fi + arow * FLD + q;
 #pragma unroll
         for (int kc = 0; kc < L / 4; ++kc) {
           const int pc = 4 * kc;
-          const double ar = fr[pc], ai = fi[pc], nai = -ai;
+          const double ar = ldF<!FSM>(fr + pc), ai = ldF<!FSM>(fi + pc), nai = -ai;
 #pragma unroll
           for (int nt = 0; nt < NT; ++nt) {
             const double br = sXa[(8 * nt + g) * LD + q + pc];
@@ -178,8 +233,8 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
           for (int mt = 0; mt < NT; ++mt) {
             if (mt < MT) {
               const int arow = min(h + 8 * mt + g, L - 1);
-              const double ar = sFr[arow * LD + pc];
-              const double ai = sFi[arow * LD + pc];
+              const double ar = ldF<!FSM>(Fr + arow * FLD + pc);
+              const double ai = ldF<!FSM>(Fi + arow * FLD + pc);
               dmma(Yr[mt], ar, br);
               dmma(Yr[mt], ai, bi);
               dmma(Yi[mt], ar, bi);
@@ -213,42 +268,76 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
         }
       }
     }
+    if (DB) {
+      cp_async_wait_all();
+      __syncthreads();   // next pair landed; this pair's Q' reads are done
+      cur ^= 1;
+    }
+  }
+}
+
+template <int L, int V>
+cudaError_t configure_LV(int* max_blocks) {
+  const size_t smem = fused2d_smem(L, V);
+  cudaError_t e = cudaFuncSetAttribute(fft2d_kernel<L, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_kernel<L, V>, L * 4, smem);
+}
+
+template <int L>
+cudaError_t configure_L(int V, int* max_blocks) {
+  switch (V) {
+    case 0: return configure_LV<L, 0>(max_blocks);
+    case 1: return configure_LV<L, 1>(max_blocks);
+    case 2: return configure_LV<L, 2>(max_blocks);
+    default: return cudaErrorInvalidValue;
   }
 }
 
 template <int L>
-cudaError_t configure_L(int* max_blocks) {
-  const size_t smem = fused2d_smem(L);
-  cudaError_t e = cudaFuncSetAttribute(fft2d_kernel<L>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_kernel<L>, L * 4, smem);
+void launch_L(int V, const Fft2dArgs& a, int grid, cudaStream_t s) {
+  const size_t smem = fused2d_smem(L, V);
+  switch (V) {
+    case 0: fft2d_kernel<L, 0><<<grid, L * 4, smem, s>>>(a); break;
+    case 1: fft2d_kernel<L, 1><<<grid, L * 4, smem, s>>>(a); break;
+    default: fft2d_kernel<L, 2><<<grid, L * 4, smem, s>>>(a); break;
+  }
 }
 
 }  // namespace
 
 int fused2d_threads(int L) { return L * 4; }
-size_t fused2d_smem(int L) { return (size_t)4 * L * (L + 4) * sizeof(double); }
 
-cudaError_t fused2d_configure(int L, int* max_blocks) {
+size_t fused2d_smem(int L, int V) {
+  const size_t plane = (size_t)L * (L + 4) * sizeof(double);
+  const size_t f = V == 2 ? 0 : 2 * plane;
+  const size_t bufs = V == 0 ? 2 * plane : 4 * plane;
+  return f + bufs;
+}
+
+cudaError_t fused2d_configure(int L, int V, int* max_blocks) {
   switch (L) {
-    case 16: return configure_L<16>(max_blocks);
-    case 24: return configure_L<24>(max_blocks);
-    case 32: return configure_L<32>(max_blocks);
-    case 40: return configure_L<40>(max_blocks);
-    case 48: return configure_L<48>(max_blocks);
-    case 56: return configure_L<56>(max_blocks);
-    case 64: return configure_L<64>(max_blocks);
+    case 16: return configure_L<16>(V, max_blocks);
+    case 24: return configure_L<24>(V, max_blocks);
+    case 32: return configure_L<32>(V, max_blocks);
+    case 40: return configure_L<40>(V, max_blocks);
+    case 48: return configure_L<48>(V, max_blocks);
+    case 56: return configure_L<56>(V, max_blocks);
+    case 64: return configure_L<64>(V, max_blocks);
     default: return cudaErrorInvalidValue;
   }
 }
 
-cudaError_t launch_fused2d(int L, const Fft2dArgs& a, int grid, cudaStream_t s) {
-  const size_t smem = fused2d_smem(L);
+cudaError_t launch_fused2d(int L, int V, const Fft2dArgs& a, int grid, cudaStream_t s) {
+  if (V < 0 || V > 2) return cudaErrorInvalidValue;
   switch (L) {
-#define FS_CASE(LL) \
-  case LL: fft2d_kernel<LL><<<grid, LL * 4, smem, s>>>(a); break;
-    FS_CASE(16) FS_CASE(24) FS_CASE(32) FS_CASE(40) FS_CASE(48) FS_CASE(56) FS_CASE(64)
-#undef FS_CASE
+    case 16: launch_L<16>(V, a, grid, s); break;
+    case 24: launch_L<24>(V, a, grid, s); break;
+    case 32: launch_L<32>(V, a, grid, s); break;
+    case 40: launch_L<40>(V, a, grid, s); break;
+    case 48: launch_L<48>(V, a, grid, s); break;
+    case 56: launch_L<56>(V, a, grid, s); break;
+    case 64: launch_L<64>(V, a, grid, s); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();

@@ -15,7 +15,7 @@ struct Fft2dArgs {
   int h, S;              // halo r*T (tile geometry) and valid side L - 2h
   int64_t nt1;           // tiles along axis 1
   int64_t ntiles, npairs;
-  const double* Fre;     // L x L forward DFT matrix, natural row-major
+  const double* Fre;     // L x L forward DFT matrix, row-major, columns permuted (perm8)
   const double* Fim;
   const double* Sre;     // L x L powered spectrum of this pass, natural row-major
   const double* Sim;
@@ -70,10 +70,12 @@ struct BoxCopyArgs {
   int64_t lo[3], hi[3];
 };
 
+// V: kernel variant (kernel_fft2d.cu header): 0 sync loads, 1 cp.async double buffer,
+// 2 double buffer + F through L1.  Fre/Fim for the 2D kernel are column-permuted (perm8).
 int fused2d_threads(int L);
-size_t fused2d_smem(int L);
-cudaError_t fused2d_configure(int L, int* max_blocks_per_sm);
-cudaError_t launch_fused2d(int L, const Fft2dArgs& a, int grid, cudaStream_t s);
+size_t fused2d_smem(int L, int V);
+cudaError_t fused2d_configure(int L, int V, int* max_blocks_per_sm);
+cudaError_t launch_fused2d(int L, int V, const Fft2dArgs& a, int grid, cudaStream_t s);
 
 constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);

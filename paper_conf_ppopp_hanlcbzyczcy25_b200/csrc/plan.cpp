@@ -61,6 +61,22 @@ double model_flops_2d(int L, int S, int T) {
   return 8.0 * dm / (2.0 * S * (double)S * T);
 }
 
+// Measured DMMA issue efficiency of the fused 2D kernel per tile side (fraction of the
+// 37.18 TF/s peak, B200, profiles/r01_sweep.txt / r01_variants.txt): the plan minimises
+// executed flops / efficiency, i.e. predicted time per cell-step (the role of Eq. 5's
+// auto-tuning of L, L174).
+static double eff_2d(int L) {
+  switch (L) {
+    case 16: return 0.68;
+    case 24: return 0.66;
+    case 32: return 0.70;
+    case 40: return 0.64;
+    case 48: return 0.74;
+    case 56: return 0.66;
+    default: return 0.70;
+  }
+}
+
 static double model_flops_3d(int L, int S, int T) {
   const double Sp = round8(S), l = L;
   const double f = 24.0 * l * l * l * l + 8.0 * Sp * l * l * l + 8.0 * Sp * Sp * l * l + 8.0 * Sp * Sp * Sp * l;
@@ -131,7 +147,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       for (int L : cand) {
         const int S = L - 2 * h;
         if (S < 8) continue;
-        const double f = model_flops_2d(L, S, t);
+        const double f = model_flops_2d(L, S, t) / eff_2d(L);
         if (f < best * (1 - 1e-12)) { best = f; bL = L; bT = t; }
       }
     }
@@ -143,7 +159,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         for (int L : cand) {
           const int S = L - 2 * h;
           if (S < 8) continue;
-          const double f = model_flops_2d(L, S, t);
+          const double f = model_flops_2d(L, S, t) / eff_2d(L);
           if (f < best) { best = f; bL = L; bT = t; }
         }
       }
@@ -157,7 +173,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     p.flops_per_cell_step = (16.0 * L * L * L + 6.0 * L * L + 8.0 * S * L * L + 8.0 * S * S * L) / (2.0 * S * S * bT);
     const double Sp = round8(p.S[0]);
     p.mma_flops_per_pair = 8.0 * (2.0 * L * L * L + Sp * L * L + Sp * Sp * L);
-    p.fused_smem = (size_t)32 * bL * (bL + 4);
+    p.fused_smem = (size_t)(bL >= 56 ? 48 : 32) * bL * (bL + 4);   // F + pair buffer(s)
   } else {
     const int L = k3DTile;
     const int hmax = std::min(hmax_grid, (L - 2) / 2);
