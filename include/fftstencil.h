@@ -50,7 +50,7 @@ enum {
   FFTSTENCIL_EINVAL = -1,        /* invalid argument                               */
   FFTSTENCIL_ENOMEM = -2,        /* host or device allocation failed               */
   FFTSTENCIL_ECUDA = -3,         /* a CUDA runtime call or kernel launch failed    */
-  FFTSTENCIL_ENCCL = -4,         /* reserved: multi-GPU halo exchange              */
+  FFTSTENCIL_ENCCL = -4,         /* an NCCL call of the multi-GPU halo exchange failed */
   FFTSTENCIL_EUNSUPPORTED = -5   /* valid request this build does not implement    */
 };
 
@@ -79,6 +79,12 @@ typedef struct {
   size_t device_bytes;          /* device memory the plan owns                      */
   int fused_grid;               /* CTAs of the persistent fused kernel              */
   int64_t last_run_launches;    /* kernels the last fftstencil_run enqueued          */
+  /* outer-axis decomposition (single GPU: nranks = 1, the whole grid) */
+  int nranks, rank;
+  int64_t row_begin, row_end;   /* global axis-0 rows this rank owns (its in/out slab)  */
+  int64_t pair_begin, pair_end; /* tile pairs this rank computes                         */
+  int64_t interior_begin, interior_end; /* pairs needing no halo rows (overlap the exchange) */
+  int64_t ghost_lo, ghost_hi;   /* halo rows received from rank-1 / rank+1 per pass     */
 } fftstencil_info;
 
 /* Build a plan (host precompute + device upload).  Returns NULL on error. */
@@ -98,6 +104,37 @@ int fftstencil_run(fftstencil_plan* plan, const double* in, double* out, int64_t
  * before returning.  Uses two device grids owned by the plan (allocated on first use). */
 int fftstencil_run_host(fftstencil_plan* plan, const double* h_in, double* h_out,
                         int64_t total_steps, void* stream);
+
+/* ---- multi-GPU: outer-axis (axis 0) domain decomposition, one process per GPU ----
+ * The grid is cut into nranks slabs of whole overlap-save tile rows (2D/3D) or tile pairs
+ * (1D), so every rank computes exactly the single-GPU tiles and results are bitwise
+ * identical to fftstencil_run on one GPU.  `extents` are GLOBAL; `in`/`out` passed to
+ * fftstencil_run are this rank's slab: rows [row_begin, row_end) of fftstencil_plan_info
+ * (every slab must hold at least radius*T rows).  Before every fused pass each rank swaps
+ * h = radius*T halo rows with rank-1 and rank+1 by NCCL send/recv on a library-owned
+ * stream over NVLink; tile pairs whose inputs need no halo run concurrently with the
+ * exchange.  `nccl_unique_id` is the 128-byte ncclUniqueId of the group (rank 0 creates it
+ * with fftstencil_nccl_unique_id and broadcasts it); creation is collective over the
+ * ranks.  nranks = 1 gives an ordinary plan.  nccl_unique_id = NULL creates a LOOPBACK
+ * rank: no communicator; the ranks of one process are then run together on one device by
+ * fftstencil_run_group, which exchanges halos by device copies (tests the decomposition
+ * without several GPUs).  Returns NULL on error (ENCCL failures included). */
+fftstencil_plan* fftstencil_plan_create_dist(int ndim, const int64_t* extents, const double* weights,
+                                             int radius, int T, int nranks, int rank,
+                                             const void* nccl_unique_id);
+
+/* Writes a new 128-byte ncclUniqueId into `out` (rank 0 of a group). */
+int fftstencil_nccl_unique_id(void* out);
+
+/* Runs loopback ranks 0..nranks-1 (plans[k] created with rank k, nccl_unique_id NULL, on the
+ * current device) for total_steps, in[k]/out[k] being rank k's device slabs; enqueued on
+ * `stream`.  Asynchronous like fftstencil_run. */
+int fftstencil_run_group(fftstencil_plan* const* plans, const double* const* in, double* const* out,
+                         int nranks, int64_t total_steps, void* stream);
+
+/* Host-only: the slab geometry rank `rank` of `nranks` would get (see fftstencil_info). */
+int fftstencil_describe_dist(int ndim, const int64_t* extents, const double* weights, int radius,
+                             int T, int nranks, int rank, fftstencil_info* info);
 
 /* Release everything the plan owns.  NULL is a no-op. */
 void fftstencil_destroy(fftstencil_plan* plan);

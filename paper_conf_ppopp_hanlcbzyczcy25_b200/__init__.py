@@ -18,7 +18,7 @@ import numpy as np
 from . import _native
 from ._native import FftStencilError, Info, last_error
 
-__all__ = ["Plan", "describe", "export_aux", "FftStencilError"]
+__all__ = ["Plan", "describe", "describe_dist", "export_aux", "nccl_unique_id", "run_group", "FftStencilError"]
 
 
 def _arrays(extents, weights, radius):
@@ -48,6 +48,43 @@ def describe(extents, weights, radius: int, T: int = 0) -> dict:
     return info.as_dict()
 
 
+def describe_dist(extents, weights, radius: int, T: int, nranks: int, rank: int) -> dict:
+    """Host-only slab geometry of one rank of the outer-axis decomposition."""
+    ext, w = _arrays(extents, weights, radius)
+    info = Info()
+    rc = _native.lib().fftstencil_describe_dist(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
+                                                int(nranks), int(rank), ctypes.byref(info))
+    if rc != 0:
+        raise FftStencilError(rc, last_error())
+    return info.as_dict()
+
+
+def nccl_unique_id() -> bytes:
+    """A fresh 128-byte ncclUniqueId (rank 0 creates it, then broadcasts it)."""
+    buf = ctypes.create_string_buffer(128)
+    rc = _native.lib().fftstencil_nccl_unique_id(buf)
+    if rc != 0:
+        raise FftStencilError(rc, last_error())
+    return buf.raw
+
+
+def run_group(plans, ins, outs, total_steps: int, stream=None) -> None:
+    """Run loopback ranks (Plan(..., nranks=n, rank=k, nccl_id=None)) together on one GPU."""
+    import torch
+    n = len(plans)
+    vp = ctypes.c_void_p
+    P = (vp * n)(*[p._h.value for p in plans])
+    I = (vp * n)(*[t.data_ptr() for t in ins])
+    O = (vp * n)(*[t.data_ptr() for t in outs])
+    for p, a, b in zip(plans, ins, outs):
+        p._check_dev(a, "in")
+        p._check_dev(b, "out")
+    s = stream if stream is not None else torch.cuda.current_stream(ins[0].device)
+    rc = _native.lib().fftstencil_run_group(P, I, O, n, int(total_steps), vp(s.cuda_stream))
+    if rc != 0:
+        raise FftStencilError(rc, last_error())
+
+
 def export_aux(extents, weights, radius: int, T: int, which: int, axis: int = 0, t: int = 1) -> np.ndarray:
     """Host plan tables (see fftstencil_export_aux in include/fftstencil.h)."""
     ext, w = _arrays(extents, weights, radius)
@@ -67,15 +104,29 @@ def export_aux(extents, weights, radius: int, T: int, which: int, axis: int = 0,
 class Plan:
     """A FlashFFTStencil plan bound to the current CUDA device."""
 
-    def __init__(self, extents, weights, radius: int, T: int = 0):
+    def __init__(self, extents, weights, radius: int, T: int = 0, nranks: int = 1, rank: int = 0,
+                 nccl_id: bytes | None = None, loopback: bool = False):
+        """extents are GLOBAL.  nranks > 1: this process's rank of the outer-axis decomposition;
+        pass the group's nccl_id (bytes from nccl_unique_id()), or loopback=True for a rank
+        run with run_group on one device.  in/out tensors then hold this rank's slab
+        (rows [row_begin, row_end) of info())."""
         ext, w = _arrays(extents, weights, radius)
-        self.extents = tuple(int(e) for e in ext)
+        self.global_extents = tuple(int(e) for e in ext)
         self.radius = int(radius)
         self._lib = _native.lib()
-        h = self._lib.fftstencil_plan_create(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T))
+        if nranks == 1:
+            h = self._lib.fftstencil_plan_create(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T))
+        else:
+            if nccl_id is None and not loopback:
+                raise ValueError("nranks > 1 needs nccl_id (or loopback=True)")
+            idbuf = None if loopback else ctypes.create_string_buffer(bytes(nccl_id), 128)
+            h = self._lib.fftstencil_plan_create_dist(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
+                                                      int(nranks), int(rank), idbuf)
         if not h:
             raise FftStencilError(_native.EINVAL, last_error())
         self._h = ctypes.c_void_p(h)
+        inf = self.info()
+        self.extents = (inf["row_end"] - inf["row_begin"],) + self.global_extents[1:]
 
     # -- lifetime --
     def close(self):

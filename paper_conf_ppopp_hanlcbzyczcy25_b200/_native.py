@@ -18,7 +18,8 @@ CODES = {OK: "OK", EINVAL: "EINVAL", ENOMEM: "ENOMEM", ECUDA: "ECUDA", ENCCL: "E
 # every symbol include/fftstencil.h declares
 EXPORTS = ("fftstencil_plan_create", "fftstencil_run", "fftstencil_run_host", "fftstencil_destroy",
            "fftstencil_plan_info", "fftstencil_last_error", "fftstencil_describe", "fftstencil_export_aux",
-           "fftstencil_set_profiling", "fftstencil_profile_read")
+           "fftstencil_set_profiling", "fftstencil_profile_read", "fftstencil_plan_create_dist",
+           "fftstencil_nccl_unique_id", "fftstencil_run_group", "fftstencil_describe_dist")
 
 
 class Info(ctypes.Structure):
@@ -40,6 +41,16 @@ class Info(ctypes.Structure):
         ("device_bytes", ctypes.c_size_t),
         ("fused_grid", ctypes.c_int),
         ("last_run_launches", ctypes.c_int64),
+        ("nranks", ctypes.c_int),
+        ("rank", ctypes.c_int),
+        ("row_begin", ctypes.c_int64),
+        ("row_end", ctypes.c_int64),
+        ("pair_begin", ctypes.c_int64),
+        ("pair_end", ctypes.c_int64),
+        ("interior_begin", ctypes.c_int64),
+        ("interior_end", ctypes.c_int64),
+        ("ghost_lo", ctypes.c_int64),
+        ("ghost_hi", ctypes.c_int64),
     ]
 
     def as_dict(self) -> dict:
@@ -52,6 +63,9 @@ class Info(ctypes.Structure):
             "mma_flops_per_pass": self.mma_flops_per_pass, "smem_bytes": self.smem_bytes,
             "device_bytes": self.device_bytes, "fused_grid": self.fused_grid,
             "last_run_launches": self.last_run_launches,
+            "nranks": self.nranks, "rank": self.rank, "row_begin": self.row_begin, "row_end": self.row_end,
+            "pair_begin": self.pair_begin, "pair_end": self.pair_end, "interior_begin": self.interior_begin,
+            "interior_end": self.interior_end, "ghost_lo": self.ghost_lo, "ghost_hi": self.ghost_hi,
         }
 
 
@@ -91,6 +105,17 @@ def lib():
     L.fftstencil_set_profiling.restype = ctypes.c_int
     L.fftstencil_profile_read.argtypes = [vp, dp, i64p, dp, i64p]
     L.fftstencil_profile_read.restype = ctypes.c_int
+    L.fftstencil_plan_create_dist.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                              ctypes.c_int, vp]
+    L.fftstencil_plan_create_dist.restype = vp
+    L.fftstencil_nccl_unique_id.argtypes = [vp]
+    L.fftstencil_nccl_unique_id.restype = ctypes.c_int
+    L.fftstencil_run_group.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.c_int,
+                                       ctypes.c_int64, vp]
+    L.fftstencil_run_group.restype = ctypes.c_int
+    L.fftstencil_describe_dist.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                           ctypes.c_int, ctypes.POINTER(Info)]
+    L.fftstencil_describe_dist.restype = ctypes.c_int
     _lib = L
     return L
 

@@ -20,9 +20,26 @@ SO = os.path.join(HERE, "libfftstencil.so")
 INCLUDE = os.path.join(ROOT, "include")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+
+
+def _nccl_dirs():
+    """NCCL headers/library: the copy torch loads (pip nvidia-nccl), else the system one.
+    Both carry the soname libnccl.so.2, so one NCCL is loaded per process."""
+    try:
+        import nvidia.nccl as nn   # noqa: F401
+        base = list(nn.__path__)[0]
+        inc, lib = os.path.join(base, "include"), os.path.join(base, "lib")
+        if os.path.exists(os.path.join(inc, "nccl.h")) and os.path.exists(os.path.join(lib, "libnccl.so.2")):
+            return inc, lib
+    except Exception:
+        pass
+    return "/usr/include", "/usr/lib/x86_64-linux-gnu"
+
+
+NCCL_INC, NCCL_LIB = _nccl_dirs()
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVFLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v", *ARCH,
-           "-I", INCLUDE, "-I", CSRC]
+           "-I", INCLUDE, "-I", CSRC, "-I", NCCL_INC]
 CXXFLAGS = ["-O2", "-std=c++17", "-fPIC", "-I", INCLUDE, "-I", CSRC]
 
 CU = ["capi.cu", "kernel_fft2d.cu", "kernel_fft1d.cu", "kernel_fft3d.cu", "kernel_band.cu"]
@@ -64,7 +81,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
                 sys.stderr.write(log)
     if force or not os.path.exists(SO) or any(os.path.getmtime(o) > os.path.getmtime(SO) for o in objs):
         tmp = SO + f".tmp{os.getpid()}"
-        cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart"]
+        cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart", "-L", NCCL_LIB, "-l:libnccl.so.2",
+               "-Xlinker", "-rpath", "-Xlinker", NCCL_LIB]
         res = subprocess.run(cmd, capture_output=True, text=True)
         if res.returncode != 0:
             raise RuntimeError(f"link failed: {' '.join(cmd)}\n{res.stdout}\n{res.stderr}")

@@ -2,12 +2,18 @@
 //
 // The run driver is the temporal loop of PAPER.md §4 (Eq. 10): floor(steps/T) fused
 // passes with S_T, then one pass with S_T' (T' = steps mod T; reading Q15).  Each pass is
-// one fused FFT-tile launch over the exact region plus one boundary-band launch, both
-// reading `src` and writing disjoint cells of `dst`; buffers ping-pong between `out` and
-// the plan's scratch grid so that the last pass lands in `out`.  The fixed ring is copied
-// once per run into every buffer that is written.
+// fused FFT-tile launch(es) over the exact region plus one boundary-band launch, reading
+// `src` and writing disjoint cells of `dst`.
+//   single GPU: buffers ping-pong between the caller's `out` and the plan's scratch grid so
+//               the last pass lands in `out`; the fixed ring is copied once per run.
+//   multi-GPU:  each rank keeps two slab buffers with r*T halo rows above and below
+//               (DESIGN.md a10); before every pass the halo rows of `src` are exchanged
+//               with the neighbouring ranks (NCCL send/recv on a comm stream, or device
+//               copies for loopback groups) while the pairs that need no halo run.
 #include <cuda_runtime.h>
+#include <nccl.h>
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -34,22 +40,31 @@ struct fftstencil_plan {
   HostPlan hp;
   int device = 0;
   int sm_count = 0;
-  double* dF = nullptr;       // Fre | Fim
-  double* dS = nullptr;       // for t = 1..T: Sre | Sim, each vol
+  double* dF = nullptr;       // Fre | Fim (2D: columns permuted)
+  double* dS = nullptr;       // for t = 1..T: Sre | Sim, each spec_vol
   int* dCrt = nullptr;
   double* dW = nullptr;
   int* dBlocks = nullptr;
-  double* dScratch = nullptr;
+  double* dScratch = nullptr; // single GPU: ping-pong partner of `out`
   double* dHostIn = nullptr;  // run_host staging grids (lazy)
   double* dHostOut = nullptr;
   size_t spec_vol = 0;
-  size_t grid_cells = 0;
+  size_t grid_cells = 0;      // cells of the caller's in/out (the slab for a dist plan)
+  size_t row_cells = 0;       // cells per outer-axis row
   size_t device_bytes = 0;
   int fused_grid = 0;
   int variant = 0;            // fused-kernel variant (2D)
   size_t band_smem = 0;
   int64_t last_launches = 0;
-  // profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run()
+  // ---- decomposition (dist) ----
+  bool dist = false;          // slab plan with halo buffers
+  bool loopback = false;      // no communicator: run by fftstencil_run_group
+  ncclComm_t comm = nullptr;
+  cudaStream_t comm_stream = nullptr;
+  cudaEvent_t ev_ready = nullptr, ev_xchg = nullptr;
+  double* dE[2] = {nullptr, nullptr};   // slab + halo buffers, rows [g0, g1)
+  int ecur = 0;               // index of the buffer holding the current state
+  // ---- profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run() ----
   bool profiling = false;
   std::vector<cudaEvent_t> ev_pool;
   std::vector<int> ev_kind;
@@ -63,6 +78,13 @@ int cuda_fail(cudaError_t e, const char* what) {
   std::snprintf(buf, sizeof buf, "%s: %s", what, cudaGetErrorString(e));
   set_error(buf);
   return FFTSTENCIL_ECUDA;
+}
+
+int nccl_fail(ncclResult_t r, const char* what) {
+  char buf[256];
+  std::snprintf(buf, sizeof buf, "%s: %s", what, ncclGetErrorString(r));
+  set_error(buf);
+  return FFTSTENCIL_ENCCL;
 }
 
 template <typename T>
@@ -79,6 +101,10 @@ void free_plan(fftstencil_plan* p) {
   int cur = 0;
   cudaGetDevice(&cur);
   cudaSetDevice(p->device);
+  if (p->comm) ncclCommDestroy(p->comm);
+  if (p->comm_stream) cudaStreamDestroy(p->comm_stream);
+  if (p->ev_ready) cudaEventDestroy(p->ev_ready);
+  if (p->ev_xchg) cudaEventDestroy(p->ev_xchg);
   for (cudaEvent_t ev : p->ev_pool) cudaEventDestroy(ev);
   cudaFree(p->dF);
   cudaFree(p->dS);
@@ -88,6 +114,8 @@ void free_plan(fftstencil_plan* p) {
   cudaFree(p->dScratch);
   cudaFree(p->dHostIn);
   cudaFree(p->dHostOut);
+  cudaFree(p->dE[0]);
+  cudaFree(p->dE[1]);
   cudaSetDevice(cur);
   delete p;
 }
@@ -106,8 +134,18 @@ void fill_info(const HostPlan& hp, fftstencil_info* info) {
   info->pairs = hp.pairs;
   info->band_blocks = (int64_t)(hp.band_blocks.size() / 8);
   info->flops_per_cell_step = hp.flops_per_cell_step;
-  info->mma_flops_per_pass = hp.mma_flops_per_pair * (double)hp.pairs;
+  info->mma_flops_per_pass = hp.mma_flops_per_pair * (double)(hp.pair_hi - hp.pair_lo);
   info->smem_bytes = hp.fused_smem;
+  info->nranks = hp.nranks;
+  info->rank = hp.rank;
+  info->row_begin = hp.row_lo;
+  info->row_end = hp.row_hi;
+  info->pair_begin = hp.pair_lo;
+  info->pair_end = hp.pair_hi;
+  info->interior_begin = hp.ipair_lo;
+  info->interior_end = hp.ipair_hi;
+  info->ghost_lo = hp.row_lo - hp.g0;
+  info->ghost_hi = hp.g1 - hp.row_hi;
 }
 
 // Profiling: a (start, end) event pair around one launch; returns the pair index or -1.
@@ -132,12 +170,24 @@ void prof_end(fftstencil_plan* p, long i, cudaStream_t s) {
   if (i >= 0) cudaEventRecord(p->ev_pool[(size_t)i + 1], s);
 }
 
-// One fused pass: src -> dst with t steps (t <= T), tile geometry of T.
-int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s) {
+// One fused launch over pairs [pb, pe): src -> dst with t steps (t <= T), tile geometry of
+// T.  The buffers hold global outer rows [g0, g1); only rows [row_lo, row_hi) are written.
+int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int64_t pb, int64_t pe,
+                 cudaStream_t s) {
+  if (pe <= pb) return FFTSTENCIL_OK;
   const HostPlan& hp = p->hp;
   const double* Sre = p->dS + (size_t)(t - 1) * 2 * p->spec_vol;
   const double* Sim = Sre + p->spec_vol;
+  Window win;
+  win.g0 = hp.g0;
+  win.gn = hp.g1 - hp.g0;
+  win.w_lo = hp.row_lo;
+  win.w_hi = hp.row_hi;
+  win.p_begin = pb;
+  win.p_end = pe;
+  const int64_t np = pe - pb;
   cudaError_t e = cudaSuccess;
+  const long pe_ = prof_begin(p, 0, s);
   if (hp.ndim == 2) {
     Fft2dArgs a;
     a.src = src;
@@ -147,15 +197,13 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     a.h = hp.h;
     a.S = hp.S[0];
     a.nt1 = hp.nt[1];
-    a.ntiles = hp.tiles;
-    a.npairs = hp.pairs;
+    a.npr = hp.npr;
+    a.win = win;
     a.Fre = p->dF;
     a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
     a.Sre = Sre;
     a.Sim = Sim;
-    const long pe = prof_begin(p, 0, s);
-    e = launch_fused2d(hp.L[0], p->variant, a, p->fused_grid, s);
-    prof_end(p, pe, s);
+    e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(p->fused_grid, np), s);
   } else if (hp.ndim == 1) {
     Fft1dArgs a;
     a.src = src;
@@ -165,15 +213,14 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     a.S = hp.S[0];
     a.L = hp.L[0];
     a.ntiles = hp.tiles;
-    a.npairs = hp.pairs;
+    a.win = win;
     a.Fre = p->dF;
     a.Fim = p->dF + 128;
     a.Sre = Sre;
     a.Sim = Sim;
     a.crt = p->dCrt;
-    const long pe = prof_begin(p, 0, s);
-    e = launch_fused1d(a, p->fused_grid, s);
-    prof_end(p, pe, s);
+    const int64_t blocks = (np + kFft1dWarpsPerBlock - 1) / kFft1dWarpsPerBlock;
+    e = launch_fused1d(a, (int)std::max<int64_t>(1, std::min<int64_t>(p->fused_grid, blocks)), s);
   } else {
     Fft3dArgs a;
     a.src = src;
@@ -185,48 +232,276 @@ int enqueue_pass(fftstencil_plan* p, const double* src, double* dst, int t, cuda
     a.S = hp.S[0];
     a.nt1 = hp.nt[1];
     a.nt2 = hp.nt[2];
-    a.ntiles = hp.tiles;
-    a.npairs = hp.pairs;
+    a.npr = hp.npr;
+    a.win = win;
     a.Fre = p->dF;
     a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
     a.Sre = Sre;
     a.Sim = Sim;
-    const long pe = prof_begin(p, 0, s);
-    e = launch_fused3d(a, p->fused_grid, s);
-    prof_end(p, pe, s);
+    e = launch_fused3d(a, (int)std::min<int64_t>(p->fused_grid, np), s);
   }
+  prof_end(p, pe_, s);
   if (e != cudaSuccess) return cuda_fail(e, "fused FFT-tile launch");
   ++p->last_launches;
-  const int nb = (int)(hp.band_blocks.size() / 8);
-  if (nb > 0) {
-    BandArgs b;
-    b.src = src;
-    b.dst = dst;
-    for (int q = 0; q < 3; ++q) { b.n[q] = hp.n[q]; b.active[q] = q >= 3 - hp.ndim; }
-    b.r = hp.radius;
-    b.t = t;
-    b.w = p->dW;
-    b.blocks = p->dBlocks;
-    b.nblocks = nb;
-    const long pb = prof_begin(p, 1, s);
-    e = launch_band(b, p->band_smem, s);
-    prof_end(p, pb, s);
-    if (e != cudaSuccess) return cuda_fail(e, "band launch");
-    ++p->last_launches;
-  }
   return FFTSTENCIL_OK;
 }
 
-int copy_ring(fftstencil_plan* p, const double* src, double* d0, double* d1, cudaStream_t s) {
+int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  const int nb = (int)(hp.band_blocks.size() / 8);
+  if (nb == 0) return FFTSTENCIL_OK;
+  BandArgs b;
+  b.src = src;
+  b.dst = dst;
+  for (int q = 0; q < 3; ++q) { b.n[q] = hp.n[q]; b.active[q] = q >= 3 - hp.ndim; }
+  b.r = hp.radius;
+  b.t = t;
+  b.w = p->dW;
+  b.blocks = p->dBlocks;
+  b.nblocks = nb;
+  b.oax = 3 - hp.ndim;
+  b.g0 = hp.g0;
+  b.gn = hp.g1 - hp.g0;
+  const long pb = prof_begin(p, 1, s);
+  cudaError_t e = launch_band(b, p->band_smem, s);
+  prof_end(p, pb, s);
+  if (e != cudaSuccess) return cuda_fail(e, "band launch");
+  ++p->last_launches;
+  return FFTSTENCIL_OK;
+}
+
+// Copy the (rank's) fixed ring from src (buffer rows start at global row src_off) into
+// d0/d1 (buffer rows start at dst_off).
+int copy_ring(fftstencil_plan* p, const double* src, int64_t src_off, double* d0, double* d1, int64_t dst_off,
+              cudaStream_t s) {
   for (const Box& b : p->hp.ring_boxes) {
     BoxCopyArgs a;
     a.src = src;
     a.dst0 = d0;
     a.dst1 = d1;
     for (int q = 0; q < 3; ++q) { a.n[q] = p->hp.n[q]; a.lo[q] = b.lo[q]; a.hi[q] = b.hi[q]; }
+    a.oax = 3 - p->hp.ndim;
+    a.src_off = src_off;
+    a.dst_off = dst_off;
     cudaError_t e = launch_box_copy(a, s);
     if (e != cudaSuccess) return cuda_fail(e, "ring copy launch");
     ++p->last_launches;
+  }
+  return FFTSTENCIL_OK;
+}
+
+// ---------------------------------------------------------------- single-GPU driver
+int run_single(fftstencil_plan* p, const double* in, double* out, int64_t total_steps, cudaStream_t s) {
+  const size_t bytes = p->grid_cells * sizeof(double);
+  if (total_steps == 0) {
+    if (in != out) {
+      cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
+      if (e != cudaSuccess) return cuda_fail(e, "copy");
+    }
+    return FFTSTENCIL_OK;
+  }
+  const int T = p->hp.T;
+  const int64_t nfull = total_steps / T;
+  const int rem = (int)(total_steps % T);
+  const int64_t passes = nfull + (rem ? 1 : 0);
+  // destination sequence: alternate out / scratch so the last pass writes `out`;
+  // with in == out the first destination must be scratch (a final copy if needed).
+  const bool alias = in == out;
+  double* dsts[2];
+  bool final_copy = false;
+  if (!alias) {
+    dsts[0] = (passes % 2) ? out : p->dScratch;
+    dsts[1] = (passes % 2) ? p->dScratch : out;
+  } else {
+    dsts[0] = p->dScratch;
+    dsts[1] = out;
+    final_copy = (passes % 2) == 1;
+  }
+  int rc = copy_ring(p, in, 0, alias ? nullptr : out, passes > 1 || alias ? p->dScratch : nullptr, 0, s);
+  if (rc) return rc;
+  const double* src = in;
+  for (int64_t i = 0; i < passes; ++i) {
+    const int t = i < nfull ? T : rem;
+    double* dst = dsts[i % 2];
+    if ((rc = launch_fused(p, src, dst, t, p->hp.pair_lo, p->hp.pair_hi, s))) return rc;
+    if ((rc = launch_band_pass(p, src, dst, t, s))) return rc;
+    src = dst;
+  }
+  if (final_copy) {
+    cudaError_t e = cudaMemcpyAsync(out, p->dScratch, bytes, cudaMemcpyDeviceToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(e, "final copy");
+  }
+  return FFTSTENCIL_OK;
+}
+
+// ---------------------------------------------------------------- multi-GPU driver pieces
+double* owned_ptr(fftstencil_plan* p, int which) {
+  return p->dE[which] + (size_t)(p->hp.row_lo - p->hp.g0) * p->row_cells;
+}
+
+int dist_begin(fftstencil_plan* p, const double* in, cudaStream_t s) {
+  const size_t bytes = p->grid_cells * sizeof(double);
+  p->ecur = 0;
+  cudaError_t e = cudaMemcpyAsync(owned_ptr(p, 0), in, bytes, cudaMemcpyDeviceToDevice, s);
+  if (e != cudaSuccess) return cuda_fail(e, "slab copy-in");
+  return copy_ring(p, in, p->hp.row_lo, p->dE[1], nullptr, p->hp.g0, s);
+}
+
+int dist_end(fftstencil_plan* p, double* out, cudaStream_t s) {
+  cudaError_t e = cudaMemcpyAsync(out, owned_ptr(p, p->ecur), p->grid_cells * sizeof(double),
+                                  cudaMemcpyDeviceToDevice, s);
+  if (e != cudaSuccess) return cuda_fail(e, "slab copy-out");
+  return FFTSTENCIL_OK;
+}
+
+// NCCL halo exchange of the current buffer on the comm stream (after `s`'s prior work).
+int nccl_exchange(fftstencil_plan* p, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  double* buf = p->dE[p->ecur];
+  const size_t rc_ = p->row_cells;
+  const int64_t glo = hp.row_lo - hp.g0, ghi = hp.g1 - hp.row_hi, own = hp.row_hi - hp.row_lo;
+  cudaError_t e = cudaEventRecord(p->ev_ready, s);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(p->comm_stream, p->ev_ready, 0);
+  if (e != cudaSuccess) return cuda_fail(e, "exchange ordering");
+  ncclResult_t r = ncclGroupStart();
+  if (r == ncclSuccess && hp.rank > 0) {
+    r = ncclSend(buf + (size_t)glo * rc_, (size_t)hp.h * rc_, ncclDouble, hp.rank - 1, p->comm, p->comm_stream);
+    if (r == ncclSuccess) r = ncclRecv(buf, (size_t)glo * rc_, ncclDouble, hp.rank - 1, p->comm, p->comm_stream);
+  }
+  if (r == ncclSuccess && hp.rank < hp.nranks - 1) {
+    r = ncclSend(buf + (size_t)(glo + own - hp.h) * rc_, (size_t)hp.h * rc_, ncclDouble, hp.rank + 1, p->comm,
+                 p->comm_stream);
+    if (r == ncclSuccess)
+      r = ncclRecv(buf + (size_t)(glo + own) * rc_, (size_t)ghi * rc_, ncclDouble, hp.rank + 1, p->comm,
+                   p->comm_stream);
+  }
+  const ncclResult_t r2 = ncclGroupEnd();
+  if (r != ncclSuccess) return nccl_fail(r, "halo send/recv");
+  if (r2 != ncclSuccess) return nccl_fail(r2, "halo group");
+  e = cudaEventRecord(p->ev_xchg, p->comm_stream);
+  if (e != cudaSuccess) return cuda_fail(e, "exchange event");
+  return FFTSTENCIL_OK;
+}
+
+// One pass of a dist rank: interior pairs overlap the exchange (if `xchg`), then the
+// halo-dependent pairs and the band.
+int dist_pass(fftstencil_plan* p, int t, bool xchg, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  const double* src = p->dE[p->ecur];
+  double* dst = p->dE[p->ecur ^ 1];
+  int rc;
+  if (xchg && (rc = nccl_exchange(p, s))) return rc;
+  if ((rc = launch_fused(p, src, dst, t, hp.ipair_lo, hp.ipair_hi, s))) return rc;
+  if (xchg) {
+    cudaError_t e = cudaStreamWaitEvent(s, p->ev_xchg, 0);
+    if (e != cudaSuccess) return cuda_fail(e, "wait for halo exchange");
+  }
+  if ((rc = launch_fused(p, src, dst, t, hp.pair_lo, hp.ipair_lo, s))) return rc;
+  if ((rc = launch_fused(p, src, dst, t, hp.ipair_hi, hp.pair_hi, s))) return rc;
+  if ((rc = launch_band_pass(p, src, dst, t, s))) return rc;
+  p->ecur ^= 1;
+  return FFTSTENCIL_OK;
+}
+
+int run_dist(fftstencil_plan* p, const double* in, double* out, int64_t total_steps, cudaStream_t s) {
+  if (p->loopback) {
+    set_error("a loopback rank runs only through fftstencil_run_group");
+    return FFTSTENCIL_EINVAL;
+  }
+  if (total_steps == 0) {
+    if (in != out) {
+      cudaError_t e = cudaMemcpyAsync(out, in, p->grid_cells * sizeof(double), cudaMemcpyDeviceToDevice, s);
+      if (e != cudaSuccess) return cuda_fail(e, "copy");
+    }
+    return FFTSTENCIL_OK;
+  }
+  int rc = dist_begin(p, in, s);
+  if (rc) return rc;
+  const int T = p->hp.T;
+  const int64_t nfull = total_steps / T;
+  const int rem = (int)(total_steps % T);
+  for (int64_t i = 0; i < nfull + (rem ? 1 : 0); ++i)
+    if ((rc = dist_pass(p, i < nfull ? T : rem, true, s))) return rc;
+  return dist_end(p, out, s);
+}
+
+// Allocates and uploads everything a plan needs after its host plan is built.
+int setup_device(fftstencil_plan* p) {
+  HostPlan& hp = p->hp;
+  cudaError_t e = cudaGetDevice(&p->device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+  e = cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceGetAttribute");
+
+  size_t acc = 0;
+  std::vector<double> F(hp.Fre);
+  F.insert(F.end(), hp.Fim.begin(), hp.Fim.end());
+  if (hp.ndim == 2) {
+    // the 2D kernel reads F with columns permuted within groups of 8 (device_common.cuh)
+    const int L = hp.L[0];
+    for (int plane = 0; plane < 2; ++plane)
+      for (int r = 0; r < L; ++r)
+        for (int c = 0; c < L; ++c)
+          F[(size_t)plane * L * L + (size_t)r * L + ((c & ~7) | ((c & 1) << 2) | ((c & 7) >> 1))] =
+              (plane ? hp.Fim : hp.Fre)[(size_t)r * L + c];
+  }
+  p->spec_vol = hp.Sre[0].size();
+  std::vector<double> Sv;
+  Sv.reserve((size_t)hp.T * 2 * p->spec_vol);
+  for (int t = 0; t < hp.T; ++t) {
+    Sv.insert(Sv.end(), hp.Sre[t].begin(), hp.Sre[t].end());
+    Sv.insert(Sv.end(), hp.Sim[t].begin(), hp.Sim[t].end());
+  }
+  p->row_cells = 1;
+  for (int a = 1; a < hp.ndim; ++a) p->row_cells *= (size_t)hp.ext[a];
+  p->grid_cells = p->row_cells * (size_t)(hp.row_hi - hp.row_lo);
+  if ((e = upload(&p->dF, F.data(), F.size(), acc)) != cudaSuccess ||
+      (e = upload(&p->dS, Sv.data(), Sv.size(), acc)) != cudaSuccess ||
+      (e = upload(&p->dW, hp.w.data(), hp.w.size(), acc)) != cudaSuccess ||
+      (e = upload(&p->dBlocks, hp.band_blocks.data(), hp.band_blocks.size(), acc)) != cudaSuccess ||
+      (hp.ndim == 1 && (e = upload(&p->dCrt, hp.crt.data(), hp.crt.size(), acc)) != cudaSuccess))
+    return cuda_fail(e, "device upload");
+  if (!p->dist) {
+    e = cudaMalloc((void**)&p->dScratch, p->grid_cells * sizeof(double));
+    if (e != cudaSuccess) return cuda_fail(e, "scratch grid allocation");
+    acc += p->grid_cells * sizeof(double);
+  } else {
+    const size_t ecells = p->row_cells * (size_t)(hp.g1 - hp.g0);
+    for (int k = 0; k < 2; ++k) {
+      e = cudaMalloc((void**)&p->dE[k], ecells * sizeof(double));
+      if (e != cudaSuccess) return cuda_fail(e, "slab buffer allocation");
+      acc += ecells * sizeof(double);
+    }
+  }
+  p->device_bytes = acc;
+
+  int occ = 0;
+  if (hp.ndim == 2) {
+    // double-buffered prefetch pays only where it does not cost occupancy (profiles/r01_variants.txt)
+    p->variant = hp.L[0] >= 56 ? 1 : 0;
+    if (const char* v = std::getenv("FFTSTENCIL_VARIANT")) p->variant = std::atoi(v);
+    if (p->variant < 0 || p->variant > 2) {
+      set_error("FFTSTENCIL_VARIANT must be 0, 1 or 2");
+      return FFTSTENCIL_EINVAL;
+    }
+    e = fused2d_configure(hp.L[0], p->variant, &occ);
+    if (e != cudaSuccess) return cuda_fail(e, "fused 2D kernel configuration");
+  } else if (hp.ndim == 3) {
+    e = fused3d_configure(&occ);
+    if (e != cudaSuccess) return cuda_fail(e, "fused 3D kernel configuration");
+  } else {
+    e = fused1d_configure(&occ);
+    if (e != cudaSuccess) return cuda_fail(e, "fused 1D kernel configuration");
+  }
+  if (occ < 1) {
+    set_error("fused kernel cannot be resident on this device");
+    return FFTSTENCIL_EUNSUPPORTED;
+  }
+  p->fused_grid = (int)std::max<int64_t>(1, (int64_t)p->sm_count * occ);
+  p->band_smem = (size_t)2 * hp.band_region_cells * sizeof(double);
+  if (p->band_smem > 0) {
+    e = band_configure(p->band_smem);
+    if (e != cudaSuccess) return cuda_fail(e, "band kernel configuration");
   }
   return FFTSTENCIL_OK;
 }
@@ -239,10 +514,15 @@ const char* fftstencil_last_error(void) { return g_last_error.c_str(); }
 
 int fftstencil_describe(int ndim, const int64_t* extents, const double* weights, int radius, int T,
                         fftstencil_info* info) {
+  return fftstencil_describe_dist(ndim, extents, weights, radius, T, 1, 0, info);
+}
+
+int fftstencil_describe_dist(int ndim, const int64_t* extents, const double* weights, int radius, int T,
+                             int nranks, int rank, fftstencil_info* info) {
   if (!info) { set_error("info must be non-NULL"); return FFTSTENCIL_EINVAL; }
   HostPlan hp;
   std::string err;
-  const int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err);
+  const int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, nranks, rank);
   if (rc != FFTSTENCIL_OK) { set_error(err); return rc; }
   fill_info(hp, info);
   clear_error();
@@ -323,136 +603,113 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
   std::string err;
   int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err);
   if (rc != FFTSTENCIL_OK) { set_error(err); delete p; return nullptr; }
-  HostPlan& hp = p->hp;
-  cudaError_t e = cudaGetDevice(&p->device);
-  if (e != cudaSuccess) { cuda_fail(e, "cudaGetDevice"); delete p; return nullptr; }
-  e = cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
-  if (e != cudaSuccess) { cuda_fail(e, "cudaDeviceGetAttribute"); delete p; return nullptr; }
+  if (setup_device(p) != FFTSTENCIL_OK) { free_plan(p); return nullptr; }
+  clear_error();
+  return p;
+}
 
-  size_t acc = 0;
-  std::vector<double> F(hp.Fre);
-  F.insert(F.end(), hp.Fim.begin(), hp.Fim.end());
-  if (hp.ndim == 2) {
-    // the 2D kernel reads F with columns permuted within groups of 8 (device_common.cuh)
-    const int L = hp.L[0];
-    for (int plane = 0; plane < 2; ++plane)
-      for (int r = 0; r < L; ++r)
-        for (int c = 0; c < L; ++c)
-          F[(size_t)plane * L * L + (size_t)r * L + ((c & ~7) | ((c & 1) << 2) | ((c & 7) >> 1))] =
-              (plane ? hp.Fim : hp.Fre)[(size_t)r * L + c];
-  }
-  p->spec_vol = hp.Sre[0].size();
-  std::vector<double> Sv;
-  Sv.reserve((size_t)hp.T * 2 * p->spec_vol);
-  for (int t = 0; t < hp.T; ++t) {
-    Sv.insert(Sv.end(), hp.Sre[t].begin(), hp.Sre[t].end());
-    Sv.insert(Sv.end(), hp.Sim[t].begin(), hp.Sim[t].end());
-  }
-  p->grid_cells = 1;
-  for (int a = 0; a < hp.ndim; ++a) p->grid_cells *= (size_t)hp.ext[a];
-  if ((e = upload(&p->dF, F.data(), F.size(), acc)) != cudaSuccess ||
-      (e = upload(&p->dS, Sv.data(), Sv.size(), acc)) != cudaSuccess ||
-      (e = upload(&p->dW, hp.w.data(), hp.w.size(), acc)) != cudaSuccess ||
-      (e = upload(&p->dBlocks, hp.band_blocks.data(), hp.band_blocks.size(), acc)) != cudaSuccess ||
-      (hp.ndim == 1 && (e = upload(&p->dCrt, hp.crt.data(), hp.crt.size(), acc)) != cudaSuccess)) {
-    cuda_fail(e, "device upload");
-    free_plan(p);
-    return nullptr;
-  }
-  e = cudaMalloc((void**)&p->dScratch, p->grid_cells * sizeof(double));
-  if (e != cudaSuccess) {
-    set_error(std::string("scratch grid allocation: ") + cudaGetErrorString(e));
-    free_plan(p);
-    return nullptr;
-  }
-  acc += p->grid_cells * sizeof(double);
-  p->device_bytes = acc;
-
-  int occ = 0;
-  if (hp.ndim == 2) {
-    // double-buffered prefetch pays only where it does not cost occupancy (profiles/r01_variants.txt)
-    p->variant = hp.L[0] >= 56 ? 1 : 0;
-    if (const char* v = std::getenv("FFTSTENCIL_VARIANT")) p->variant = std::atoi(v);
-    if (p->variant < 0 || p->variant > 2) { set_error("FFTSTENCIL_VARIANT must be 0, 1 or 2"); free_plan(p); return nullptr; }
-    e = fused2d_configure(hp.L[0], p->variant, &occ);
-    if (e != cudaSuccess) { cuda_fail(e, "fused 2D kernel configuration"); free_plan(p); return nullptr; }
-    if (occ < 1) { set_error("fused 2D kernel cannot be resident"); free_plan(p); return nullptr; }
-    const int64_t want = (int64_t)p->sm_count * occ;
-    p->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, hp.pairs));
-  } else if (hp.ndim == 3) {
-    e = fused3d_configure(&occ);
-    if (e != cudaSuccess) { cuda_fail(e, "fused 3D kernel configuration"); free_plan(p); return nullptr; }
-    if (occ < 1) { set_error("fused 3D kernel cannot be resident"); free_plan(p); return nullptr; }
-    const int64_t want = (int64_t)p->sm_count * occ;
-    p->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, hp.pairs));
-  } else {
-    e = fused1d_configure(&occ);
-    if (e != cudaSuccess || occ < 1) { cuda_fail(e, "fused 1D kernel configuration"); free_plan(p); return nullptr; }
-    const int64_t blocks = (hp.pairs + kFft1dWarpsPerBlock - 1) / kFft1dWarpsPerBlock;
-    p->fused_grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)p->sm_count * occ));
-  }
-  p->band_smem = (size_t)2 * hp.band_region_cells * sizeof(double);
-  if (p->band_smem > 0) {
-    e = band_configure(p->band_smem);
-    if (e != cudaSuccess) { cuda_fail(e, "band kernel configuration"); free_plan(p); return nullptr; }
+fftstencil_plan* fftstencil_plan_create_dist(int ndim, const int64_t* extents, const double* weights, int radius,
+                                             int T, int nranks, int rank, const void* nccl_unique_id) {
+  if (nranks == 1 && rank == 0) return fftstencil_plan_create(ndim, extents, weights, radius, T);
+  fftstencil_plan* p = new (std::nothrow) fftstencil_plan();
+  if (!p) { set_error("host allocation failed"); return nullptr; }
+  std::string err;
+  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err, nranks, rank);
+  if (rc != FFTSTENCIL_OK) { set_error(err); delete p; return nullptr; }
+  p->dist = true;
+  p->loopback = nccl_unique_id == nullptr;
+  if (setup_device(p) != FFTSTENCIL_OK) { free_plan(p); return nullptr; }
+  if (!p->loopback) {
+    ncclUniqueId id;
+    std::memcpy(&id, nccl_unique_id, sizeof id);
+    ncclResult_t r = ncclCommInitRank(&p->comm, nranks, id, rank);
+    if (r != ncclSuccess) { nccl_fail(r, "ncclCommInitRank"); p->comm = nullptr; free_plan(p); return nullptr; }
+    cudaError_t e = cudaStreamCreateWithFlags(&p->comm_stream, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->ev_ready, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->ev_xchg, cudaEventDisableTiming);
+    if (e != cudaSuccess) { cuda_fail(e, "comm stream/events"); free_plan(p); return nullptr; }
   }
   clear_error();
   return p;
+}
+
+int fftstencil_nccl_unique_id(void* out) {
+  if (!out) { set_error("out must be non-NULL"); return FFTSTENCIL_EINVAL; }
+  ncclUniqueId id;
+  ncclResult_t r = ncclGetUniqueId(&id);
+  if (r != ncclSuccess) return nccl_fail(r, "ncclGetUniqueId");
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId is 128 bytes");
+  std::memcpy(out, &id, sizeof id);
+  clear_error();
+  return FFTSTENCIL_OK;
 }
 
 int fftstencil_run(fftstencil_plan* p, const double* in, double* out, int64_t total_steps, void* stream) {
   if (!p || !in || !out) { set_error("plan, in and out must be non-NULL"); return FFTSTENCIL_EINVAL; }
   if (total_steps < 0) { set_error("total_steps must be >= 0"); return FFTSTENCIL_EINVAL; }
   cudaStream_t s = (cudaStream_t)stream;
-  const size_t bytes = p->grid_cells * sizeof(double);
   p->last_launches = 0;
   int cur = -1;
   cudaGetDevice(&cur);
   if (cur != p->device) cudaSetDevice(p->device);
-  int rc = FFTSTENCIL_OK;
-  do {
-    if (total_steps == 0) {
-      if (in != out) {
-        cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
-        if (e != cudaSuccess) { rc = cuda_fail(e, "copy"); break; }
-      }
-      break;
-    }
-    const int T = p->hp.T;
-    const int64_t nfull = total_steps / T;
-    const int rem = (int)(total_steps % T);
-    const int64_t passes = nfull + (rem ? 1 : 0);
-    // destination sequence: alternate out / scratch so the last pass writes `out`;
-    // with in == out the first destination must be scratch (a final copy if needed).
-    const bool alias = in == out;
-    double* dsts[2];
-    bool final_copy = false;
-    if (!alias) {
-      dsts[0] = (passes % 2) ? out : p->dScratch;
-      dsts[1] = (passes % 2) ? p->dScratch : out;
-    } else {
-      dsts[0] = p->dScratch;
-      dsts[1] = out;
-      final_copy = (passes % 2) == 1;
-    }
-    // fixed ring: copied once into every buffer that receives a pass
-    rc = copy_ring(p, in, alias ? nullptr : out, passes > 1 || alias ? p->dScratch : nullptr, s);
-    if (rc) break;
-    const double* src = in;
-    for (int64_t i = 0; i < passes; ++i) {
-      const int t = i < nfull ? T : rem;
-      double* dst = dsts[i % 2];
-      rc = enqueue_pass(p, src, dst, t, s);
-      if (rc) break;
-      src = dst;
-    }
-    if (rc) break;
-    if (final_copy) {
-      cudaError_t e = cudaMemcpyAsync(out, p->dScratch, bytes, cudaMemcpyDeviceToDevice, s);
-      if (e != cudaSuccess) { rc = cuda_fail(e, "final copy"); break; }
-    }
-  } while (0);
+  const int rc = p->dist ? run_dist(p, in, out, total_steps, s) : run_single(p, in, out, total_steps, s);
   if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
+  if (rc == FFTSTENCIL_OK) clear_error();
+  return rc;
+}
+
+int fftstencil_run_group(fftstencil_plan* const* plans, const double* const* in, double* const* out, int nranks,
+                         int64_t total_steps, void* stream) {
+  if (!plans || !in || !out || nranks < 1) { set_error("invalid group arguments"); return FFTSTENCIL_EINVAL; }
+  if (total_steps < 0) { set_error("total_steps must be >= 0"); return FFTSTENCIL_EINVAL; }
+  for (int k = 0; k < nranks; ++k) {
+    const fftstencil_plan* p = plans[k];
+    if (!p || !in[k] || !out[k] || !p->dist || !p->loopback || p->hp.nranks != nranks || p->hp.rank != k ||
+        p->hp.T != plans[0]->hp.T || p->device != plans[0]->device) {
+      set_error("plans must be loopback ranks 0..nranks-1 of one decomposition on one device");
+      return FFTSTENCIL_EINVAL;
+    }
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  int rc = FFTSTENCIL_OK;
+  for (int k = 0; k < nranks; ++k) plans[k]->last_launches = 0;
+  if (total_steps == 0) {
+    for (int k = 0; k < nranks && !rc; ++k)
+      if (in[k] != out[k]) {
+        cudaError_t e = cudaMemcpyAsync(out[k], in[k], plans[k]->grid_cells * sizeof(double),
+                                        cudaMemcpyDeviceToDevice, s);
+        if (e != cudaSuccess) rc = cuda_fail(e, "copy");
+      }
+    return rc;
+  }
+  for (int k = 0; k < nranks && !rc; ++k) rc = dist_begin(plans[k], in[k], s);
+  const int T = plans[0]->hp.T;
+  const int64_t nfull = total_steps / T;
+  const int rem = (int)(total_steps % T);
+  for (int64_t i = 0; i < nfull + (rem ? 1 : 0) && !rc; ++i) {
+    // loopback halo exchange: neighbours' owned boundary rows -> this rank's halo rows
+    for (int k = 0; k < nranks && !rc; ++k) {
+      fftstencil_plan* p = plans[k];
+      const HostPlan& hp = p->hp;
+      double* buf = p->dE[p->ecur];
+      const size_t rcs = p->row_cells * sizeof(double);
+      cudaError_t e = cudaSuccess;
+      if (k > 0) {
+        const fftstencil_plan* q = plans[k - 1];
+        const double* src = q->dE[q->ecur] + (size_t)(q->hp.row_hi - hp.h - q->hp.g0) * q->row_cells;
+        e = cudaMemcpyAsync(buf, src, (size_t)(hp.row_lo - hp.g0) * rcs, cudaMemcpyDeviceToDevice, s);
+      }
+      if (e == cudaSuccess && k < nranks - 1) {
+        const fftstencil_plan* q = plans[k + 1];
+        const double* src = q->dE[q->ecur] + (size_t)(q->hp.row_lo - q->hp.g0) * q->row_cells;
+        e = cudaMemcpyAsync(buf + (size_t)(hp.row_hi - hp.g0) * p->row_cells, src, (size_t)(hp.g1 - hp.row_hi) * rcs,
+                            cudaMemcpyDeviceToDevice, s);
+      }
+      if (e != cudaSuccess) rc = cuda_fail(e, "loopback halo copy");
+    }
+    for (int k = 0; k < nranks && !rc; ++k) rc = dist_pass(plans[k], i < nfull ? T : rem, false, s);
+  }
+  for (int k = 0; k < nranks && !rc; ++k) rc = dist_end(plans[k], out[k], s);
   if (rc == FFTSTENCIL_OK) clear_error();
   return rc;
 }
@@ -489,6 +746,16 @@ int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, i
 
 void fftstencil_destroy(fftstencil_plan* p) { free_plan(p); }
 
+int fftstencil_plan_info(const fftstencil_plan* p, fftstencil_info* info) {
+  if (!p || !info) { set_error("plan and info must be non-NULL"); return FFTSTENCIL_EINVAL; }
+  fill_info(p->hp, info);
+  info->device_bytes = p->device_bytes;
+  info->fused_grid = p->fused_grid;
+  info->last_run_launches = p->last_launches;
+  clear_error();
+  return FFTSTENCIL_OK;
+}
+
 int fftstencil_set_profiling(fftstencil_plan* p, int enable) {
   if (!p) { set_error("plan must be non-NULL"); return FFTSTENCIL_EINVAL; }
   p->profiling = enable != 0;
@@ -517,16 +784,6 @@ int fftstencil_profile_read(fftstencil_plan* p, double* fused_ms, int64_t* fused
   if (fused_launches) *fused_launches = cnt[0];
   if (band_ms) *band_ms = ms[1];
   if (band_launches) *band_launches = cnt[1];
-  clear_error();
-  return FFTSTENCIL_OK;
-}
-
-int fftstencil_plan_info(const fftstencil_plan* p, fftstencil_info* info) {
-  if (!p || !info) { set_error("plan and info must be non-NULL"); return FFTSTENCIL_EINVAL; }
-  fill_info(p->hp, info);
-  info->device_bytes = p->device_bytes;
-  info->fused_grid = p->fused_grid;
-  info->last_run_launches = p->last_launches;
   clear_error();
   return FFTSTENCIL_OK;
 }

@@ -18,21 +18,24 @@ namespace {
 __global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
   extern __shared__ double sb[];
   const int* blk = a.blocks + 8 * blockIdx.x;
-  int64_t lo[3], hi[3], rl[3], D[3];
+  int64_t lo[3], hi[3], rl[3], D[3], off[3] = {0, 0, 0};
+  off[a.oax] = a.g0;   // buffers start at global outer-axis row g0
 #pragma unroll
   for (int q = 0; q < 3; ++q) {
     lo[q] = blk[q];
     hi[q] = blk[3 + q];
     const int64_t gq = a.active[q] ? (int64_t)a.r * a.t : 0;
-    rl[q] = max((int64_t)0, lo[q] - gq);
-    D[q] = min(a.n[q], hi[q] + gq) - rl[q];
+    int64_t l = max((int64_t)0, lo[q] - gq), u = min(a.n[q], hi[q] + gq);
+    if (q == a.oax) { l = max(l, a.g0); u = min(u, a.g0 + a.gn); }
+    rl[q] = l;
+    D[q] = u - l;
   }
   const int64_t vol = D[0] * D[1] * D[2];
   double* b0 = sb;
   double* b1 = sb + vol;
   for (int64_t e = threadIdx.x; e < vol; e += blockDim.x) {
     const int64_t i2 = e % D[2], i1 = (e / D[2]) % D[1], i0 = e / (D[1] * D[2]);
-    b0[e] = a.src[((rl[0] + i0) * a.n[1] + (rl[1] + i1)) * a.n[2] + (rl[2] + i2)];
+    b0[e] = a.src[((rl[0] + i0 - off[0]) * a.n[1] + (rl[1] + i1 - off[1])) * a.n[2] + (rl[2] + i2 - off[2])];
   }
   __syncthreads();
   const int r = a.r, wd = 2 * r + 1;
@@ -74,7 +77,7 @@ __global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
   for (int64_t e = threadIdx.x; e < ovol; e += blockDim.x) {
     const int64_t j2 = e % O2, j1 = (e / O2) % O1, j0 = e / (O1 * O2);
     const int64_t c0 = lo[0] + j0, c1 = lo[1] + j1, c2 = lo[2] + j2;
-    a.dst[(c0 * a.n[1] + c1) * a.n[2] + c2] =
+    a.dst[((c0 - off[0]) * a.n[1] + (c1 - off[1])) * a.n[2] + (c2 - off[2])] =
         b0[((c0 - rl[0]) * D[1] + (c1 - rl[1])) * D[2] + (c2 - rl[2])];
   }
 }
@@ -84,10 +87,14 @@ __global__ void box_copy_kernel(const BoxCopyArgs a) {
   const int64_t vol = L0 * L1 * L2;
   for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < vol; e += (int64_t)gridDim.x * blockDim.x) {
     const int64_t j2 = e % L2, j1 = (e / L2) % L1, j0 = e / (L1 * L2);
-    const int64_t idx = ((a.lo[0] + j0) * a.n[1] + (a.lo[1] + j1)) * a.n[2] + (a.lo[2] + j2);
-    const double v = a.src[idx];
-    if (a.dst0) a.dst0[idx] = v;
-    if (a.dst1) a.dst1[idx] = v;
+    int64_t c[3] = {a.lo[0] + j0, a.lo[1] + j1, a.lo[2] + j2};
+    int64_t d[3] = {c[0], c[1], c[2]};
+    c[a.oax] -= a.src_off;
+    d[a.oax] -= a.dst_off;
+    const double v = a.src[(c[0] * a.n[1] + c[1]) * a.n[2] + c[2]];
+    const int64_t di = (d[0] * a.n[1] + d[1]) * a.n[2] + d[2];
+    if (a.dst0) a.dst0[di] = v;
+    if (a.dst1) a.dst1[di] = v;
   }
 }
 

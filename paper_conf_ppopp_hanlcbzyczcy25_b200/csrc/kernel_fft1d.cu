@@ -42,7 +42,7 @@ __device__ __forceinline__ void cgemm8(const double (&ar)[2], const double (&ai)
 
 __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const Fft1dArgs a) {
   const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
-  const int64_t warp = (int64_t)blockIdx.x * kFft1dWarpsPerBlock + (threadIdx.x >> 5);
+  const int64_t warp = a.win.p_begin + (int64_t)blockIdx.x * kFft1dWarpsPerBlock + (threadIdx.x >> 5);
   const int64_t nwarps = (int64_t)gridDim.x * kFft1dWarpsPerBlock;
 
   // A fragments: chunk j of row g is logical column 2q+j (device_common.cuh)
@@ -61,8 +61,9 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
   }
   const int L = a.L, S = a.S, h = a.h;
 
-  for (int64_t p = warp; p < a.npairs; p += nwarps) {
-    const int64_t oa = 2 * p * S, ob = (2 * p + 1) * S;
+  const int64_t g0 = a.win.g0, g1 = a.win.g0 + a.win.gn;
+  for (int64_t p = warp; p < a.win.p_end; p += nwarps) {
+    const int64_t oa = 2 * p * S, ob = (2 * p + 1) * S;   // global cell of tile position 0
     const bool has_b = 2 * p + 1 < a.ntiles;
     // B fragment of X^T:  X[l1 = g][l2 = 2q+j] = x[crt(g, 2q+j)]  (CRT gather, L1-resident)
     double xr[2], xi[2];
@@ -71,8 +72,9 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
       xr[j] = 0.0;
       xi[j] = 0.0;
       if (pos[j] >= 0) {
-        if (oa + pos[j] < a.n) xr[j] = __ldg(a.src + oa + pos[j]);
-        if (has_b && ob + pos[j] < a.n) xi[j] = __ldg(a.src + ob + pos[j]);
+        const int64_t xa = oa + pos[j], xb = ob + pos[j];
+        if (xa < a.n && xa >= g0 && xa < g1) xr[j] = __ldg(a.src + (xa - g0));
+        if (has_b && xb < a.n && xb >= g0 && xb < g1) xi[j] = __ldg(a.src + (xb - g0));
       }
     }
     double m1r[2], m1i[2], m2r[2], m2i[2];
@@ -92,8 +94,8 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
       const int l = pos[j];
       if (l >= h && l < L - h) {                   // valid window (Eq. 7, reading Q4)
         const int64_t xa = oa + l, xb = ob + l;
-        if (xa < a.n - h) a.dst[xa] = m2r[j];
-        if (has_b && xb < a.n - h) a.dst[xb] = m2i[j];
+        if (xa < a.n - h && xa >= a.win.w_lo && xa < a.win.w_hi) a.dst[xa - g0] = m2r[j];
+        if (has_b && xb < a.n - h && xb >= a.win.w_lo && xb < a.win.w_hi) a.dst[xb - g0] = m2i[j];
       }
     }
   }

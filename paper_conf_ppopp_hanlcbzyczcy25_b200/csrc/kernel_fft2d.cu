@@ -40,29 +40,27 @@ __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool v
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
+// Pair p = tiles (t0, 2j) and (t0, 2j+1) with t0 = p / npr, j = p % npr (kernels.cuh).
 template <int L, bool ASYNC>
 __device__ __forceinline__ void load_pair(double* sXa, double* sXb, const Fft2dArgs& a, int64_t p, int tid) {
   constexpr int LD = L + 4, NTHR = L * 4;
+  const int64_t t0 = p / a.npr, j = p - t0 * a.npr;
+  const int64_t o0 = t0 * a.S;            // global row of tile row 0
 #pragma unroll
   for (int t = 0; t < 2; ++t) {
-    const int64_t tile = 2 * p + t;
+    const int64_t t1 = 2 * j + t;
     double* sX = t ? sXb : sXa;
-    const bool have = tile < a.ntiles;
-    int64_t o0 = 0, o1 = 0;
-    if (have) {
-      const int64_t t0 = tile / a.nt1;
-      o0 = t0 * a.S;
-      o1 = (tile - t0 * a.nt1) * a.S;
-    }
+    const bool have = t1 < a.nt1;
+    const int64_t o1 = t1 * a.S;
     for (int e = tid; e < L * L; e += NTHR) {
       const int r = e / L, c = e - r * L;
-      const int64_t gr = o0 + r, gc = o1 + c;
-      const bool valid = have && gr < a.n0 && gc < a.n1;
+      const int64_t gr = o0 + r, gc = o1 + c, lr = gr - a.win.g0;
+      const bool valid = have && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc < a.n1;
       double* dst = sX + r * LD + perm8(c);
       if (ASYNC) {
-        cp_async8(dst, valid ? a.src + gr * a.n1 + gc : a.src, valid);
+        cp_async8(dst, valid ? a.src + lr * a.n1 + gc : a.src, valid);
       } else {
-        *dst = valid ? __ldg(a.src + gr * a.n1 + gc) : 0.0;
+        *dst = valid ? __ldg(a.src + lr * a.n1 + gc) : 0.0;
       }
     }
   }
@@ -106,12 +104,12 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
   const int MT = (S + 7) >> 3;   // output 8-tiles per axis (S padded to 8)
   int cur = 0;
 
-  if (DB && blockIdx.x < a.npairs) {
-    load_pair<L, true>(sbuf, sbuf + L * LD, a, blockIdx.x, tid);
+  if (DB && a.win.p_begin + blockIdx.x < a.win.p_end) {
+    load_pair<L, true>(sbuf, sbuf + L * LD, a, a.win.p_begin + blockIdx.x, tid);
     cp_async_commit();
     cp_async_wait_all();
   }
-  for (int64_t p = blockIdx.x; p < a.npairs; p += gridDim.x) {
+  for (int64_t p = a.win.p_begin + blockIdx.x; p < a.win.p_end; p += gridDim.x) {
     double* sXa = sbuf + cur * 2 * L * LD;   // tile 2p (real part) ... later Q' real part
     double* sXb = sXa + L * LD;              // tile 2p+1 (imag part) ... later Q' imag part
     if (!DB) {
@@ -188,7 +186,7 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
     // ---- prefetch the next pair into the other buffer while the inverse half runs ----
     if (DB) {
       const int64_t pn = p + gridDim.x;
-      if (pn < a.npairs) {
+      if (pn < a.win.p_end) {
         double* nb = sbuf + (cur ^ 1) * 2 * L * LD;
         load_pair<L, true>(nb, nb + L * LD, a, pn, tid);
       }
@@ -243,26 +241,25 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
           }
         }
       }
-      // ---- stitch: the S x S valid window of each tile, exact region only ----
-      const int64_t ta = 2 * p, tb = 2 * p + 1;
-      const int64_t a0 = ta / a.nt1, a1 = ta - a0 * a.nt1;
-      const int64_t b0 = tb / a.nt1, b1 = tb - b0 * a.nt1;
-      const bool has_b = tb < a.ntiles;
+      // ---- stitch: the S x S valid window of each tile, exact region and window only ----
+      const int64_t t0 = p / a.npr, pj = p - t0 * a.npr;
+      const int64_t a1 = 2 * pj, b1 = a1 + 1;
+      const bool has_b = b1 < a.nt1;
 #pragma unroll
       for (int mt = 0; mt < NT; ++mt) {
         if (mt < MT) {
           const int l0 = 8 * mt + g;
+          const int64_t c0 = t0 * S + h + l0;
+          const bool row_ok = l0 < S && c0 < a.n0 - h && c0 >= a.win.w_lo && c0 < a.win.w_hi;
+          double* drow = a.dst + (c0 - a.win.g0) * a.n1;
 #pragma unroll
           for (int j = 0; j < 2; ++j) {
             const int l1 = 8 * warp + 2 * q + j;
-            if (l0 < S && l1 < S) {
-              int64_t c0 = a0 * S + h + l0, c1 = a1 * S + h + l1;
-              if (c0 < a.n0 - h && c1 < a.n1 - h) a.dst[c0 * a.n1 + c1] = Yr[mt][j];
-              if (has_b) {
-                c0 = b0 * S + h + l0;
-                c1 = b1 * S + h + l1;
-                if (c0 < a.n0 - h && c1 < a.n1 - h) a.dst[c0 * a.n1 + c1] = Yi[mt][j];
-              }
+            if (row_ok && l1 < S) {
+              int64_t c1 = a1 * S + h + l1;
+              if (c1 < a.n1 - h) drow[c1] = Yr[mt][j];
+              c1 = b1 * S + h + l1;
+              if (has_b && c1 < a.n1 - h) drow[c1] = Yi[mt][j];
             }
           }
         }

@@ -57,29 +57,26 @@ __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
   }
   const int S = a.S, h = a.h;
   const int MT = (S + 7) >> 3;     // output 8-tiles per axis (1 or 2)
-  const int64_t ntt = a.nt1 * a.nt2;
-
-  for (int64_t p = blockIdx.x; p < a.npairs; p += gridDim.x) {
+  // pair p = tiles (t0, t1, 2j) and (t0, t1, 2j+1): line = p / npr = t0 * nt1 + t1 (kernels.cuh)
+  for (int64_t p = a.win.p_begin + blockIdx.x; p < a.win.p_end; p += gridDim.x) {
     __syncthreads();
+    const int64_t line = p / a.npr, pj = p - line * a.npr;
+    const int64_t t0 = line / a.nt1, t1 = line - t0 * a.nt1;
+    const int64_t o0 = t0 * S, o1 = t1 * S;
     // ---- load the halo'd pair: rows of 16 doubles (128 B), OOB = 0 ----
 #pragma unroll
     for (int t = 0; t < 2; ++t) {
-      const int64_t tile = 2 * p + t;
+      const int64_t t2 = 2 * pj + t;
       double* sX = t ? sXb : sXa;
-      const bool have = tile < a.ntiles;
-      int64_t o0 = 0, o1 = 0, o2 = 0;
-      if (have) {
-        const int64_t t0 = tile / ntt, rem = tile - t0 * ntt, t1 = rem / a.nt2, t2 = rem - t1 * a.nt2;
-        o0 = t0 * S;
-        o1 = t1 * S;
-        o2 = t2 * S;
-      }
+      const bool have = t2 < a.nt2;
+      const int64_t o2 = t2 * S;
       for (int e = tid; e < L * L * L; e += NW3 * 32) {
         const int l0 = e >> 8, l1 = (e >> 4) & 15, l2 = e & 15;
         double v = 0.0;
         if (have) {
-          const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = o2 + l2;
-          if (g0 < a.n0 && g1 < a.n1 && g2 < a.n2) v = __ldg(a.src + (g0 * a.n1 + g1) * a.n2 + g2);
+          const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = o2 + l2, lg0 = g0 - a.win.g0;
+          if (g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2)
+            v = __ldg(a.src + (lg0 * a.n1 + g1) * a.n2 + g2);
         }
         sX[l0 * SL + l1 * LD + perm8(l2)] = v;
       }
@@ -203,16 +200,12 @@ __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
     __syncthreads();
 
     // ---- phase 3: per output slice l0 < S: inverse along axes 2 then 1, crop, store ----
-    const int64_t ta = 2 * p, tb = 2 * p + 1;
-    const bool has_b = tb < a.ntiles;
-    int64_t oa[3], ob[3];
-    {
-      int64_t t0 = ta / ntt, rem = ta - t0 * ntt, t1 = rem / a.nt2;
-      oa[0] = t0 * S; oa[1] = t1 * S; oa[2] = (rem - t1 * a.nt2) * S;
-      t0 = tb / ntt; rem = tb - t0 * ntt; t1 = rem / a.nt2;
-      ob[0] = t0 * S; ob[1] = t1 * S; ob[2] = (rem - t1 * a.nt2) * S;
-    }
+    const bool has_b = 2 * pj + 1 < a.nt2;
+    const int64_t oa2 = 2 * pj * S, ob2 = oa2 + S;
     for (int l0 = warp; l0 < S; l0 += NW3) {
+      const int64_t c0 = o0 + h + l0;
+      if (c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
+      double* dplane = a.dst + (c0 - a.win.g0) * a.n1 * a.n2;
       const double* wa = sXa + l0 * SL;
       const double* wb = sXb + l0 * SL;
       // M5[l2][k1] = sum_k2 conj(F)[h + l2][k2] W[l0][k1][k2]
@@ -269,13 +262,12 @@ __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
 #pragma unroll
           for (int j = 0; j < 2; ++j) {
             const int l2 = 8 * n + 2 * q + j;
-            if (l1 < S && l2 < S) {
-              int64_t c0 = oa[0] + h + l0, c1 = oa[1] + h + l1, c2 = oa[2] + h + l2;
-              if (c0 < a.n0 - h && c1 < a.n1 - h && c2 < a.n2 - h) a.dst[(c0 * a.n1 + c1) * a.n2 + c2] = Yr[m][n][j];
-              if (has_b) {
-                c0 = ob[0] + h + l0; c1 = ob[1] + h + l1; c2 = ob[2] + h + l2;
-                if (c0 < a.n0 - h && c1 < a.n1 - h && c2 < a.n2 - h) a.dst[(c0 * a.n1 + c1) * a.n2 + c2] = Yi[m][n][j];
-              }
+            const int64_t c1 = o1 + h + l1;
+            if (l1 < S && l2 < S && c1 < a.n1 - h) {
+              int64_t c2 = oa2 + h + l2;
+              if (c2 < a.n2 - h) dplane[c1 * a.n2 + c2] = Yr[m][n][j];
+              c2 = ob2 + h + l2;
+              if (has_b && c2 < a.n2 - h) dplane[c1 * a.n2 + c2] = Yi[m][n][j];
             }
           }
         }

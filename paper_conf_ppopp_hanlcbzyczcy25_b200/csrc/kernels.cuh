@@ -7,6 +7,22 @@
 
 namespace fstencil {
 
+// Outer-axis window of one launch (multi-GPU decomposition).  The source
+// and destination buffers hold global axis-0 rows [g0, g0 + gn); the launch processes
+// tile pairs [p_begin, p_end) and writes only global axis-0 rows [w_lo, w_hi).  Input rows
+// outside the buffer read as zero (they only influence rows the launch does not write).
+// Single GPU: g0 = 0, gn = n0, [w_lo, w_hi) = [0, n0), all pairs.
+struct Window {
+  int64_t g0, gn;
+  int64_t w_lo, w_hi;
+  int64_t p_begin, p_end;
+};
+
+// Tile pairs (Double-layer Filling, Eq. 9): tiles are paired along the innermost tile axis
+// within one row of tiles -- (.., 2j) with (.., 2j+1); an odd row count pairs the last tile
+// with zeros.  Pairs never straddle an outer-axis tile row, so a decomposition into whole
+// tile rows computes exactly the single-GPU pairs (bitwise-equal results).
+
 // One fused pass of the 2D path over every tile pair (kernel_fft2d.cu).
 struct Fft2dArgs {
   const double* src;
@@ -14,7 +30,8 @@ struct Fft2dArgs {
   int64_t n0, n1;        // grid extents
   int h, S;              // halo r*T (tile geometry) and valid side L - 2h
   int64_t nt1;           // tiles along axis 1
-  int64_t ntiles, npairs;
+  int64_t npr;           // pairs per tile row = ceil(nt1 / 2)
+  Window win;
   const double* Fre;     // L x L forward DFT matrix, row-major, columns permuted (perm8)
   const double* Fim;
   const double* Sre;     // L x L powered spectrum of this pass, natural row-major
@@ -27,7 +44,8 @@ struct Fft1dArgs {
   double* dst;
   int64_t n;
   int h, S, L;           // L = N1*N2 = 56
-  int64_t ntiles, npairs;
+  int64_t ntiles;        // pair p holds tiles 2p and 2p+1
+  Window win;
   const double* Fre;     // 16 x 8: rows 0..7 F_N1, rows 8..15 F_N2 zero-padded
   const double* Fim;
   const double* Sre;     // 8 x 8 Ruritanian-ordered powered spectrum, zero-padded
@@ -42,7 +60,8 @@ struct Fft3dArgs {
   int64_t n0, n1, n2;
   int h, S;
   int64_t nt1, nt2;      // tiles along axes 1 and 2
-  int64_t ntiles, npairs;
+  int64_t npr;           // pairs per (t0, t1) tile line = ceil(nt2 / 2)
+  Window win;
   const double* Fre;     // 16 x 16 forward DFT matrix
   const double* Fim;
   const double* Sre;     // powered spectrum in [k1][k2][k0] order
@@ -57,8 +76,10 @@ struct BandArgs {
   int active[3];
   int r, t;              // radius, steps of this pass
   const double* w;       // (2r+1)^ndim weights, offset-cube row-major
-  const int* blocks;     // 8 ints per block: lo[3], hi[3], face, pad
+  const int* blocks;     // 8 ints per block: lo[3], hi[3], face, pad (global coordinates)
   int nblocks;
+  int oax;               // embedded index of the outer axis (3 - ndim)
+  int64_t g0, gn;        // buffers hold global outer-axis rows [g0, g0 + gn)
 };
 
 // Copy a box (embedded coordinates) from src to dst0 and dst1 (either may be null).
@@ -67,7 +88,9 @@ struct BoxCopyArgs {
   double* dst0;
   double* dst1;
   int64_t n[3];
-  int64_t lo[3], hi[3];
+  int64_t lo[3], hi[3];  // global embedded coordinates
+  int oax;               // embedded index of the outer axis
+  int64_t src_off, dst_off;   // global outer-axis row of buffer row 0 (src / dst0 and dst1)
 };
 
 // V: kernel variant (kernel_fft2d.cu header): 0 sync loads, 1 cp.async double buffer,

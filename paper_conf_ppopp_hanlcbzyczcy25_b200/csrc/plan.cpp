@@ -88,8 +88,9 @@ static double model_flops_1d(int S, int T) {  // one 8x8 complex tile, 4 GEMMs o
 }
 
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
-                    HostPlan& p, std::string& err) {
+                    HostPlan& p, std::string& err, int nranks, int rank) {
   p = HostPlan();
+  if (nranks < 1 || rank < 0 || rank >= nranks) { err = "need 0 <= rank < nranks"; return FFTSTENCIL_EINVAL; }
   if (ndim < 1 || ndim > 3) { err = "ndim must be 1, 2 or 3"; return FFTSTENCIL_EINVAL; }
   if (!extents || !weights) { err = "extents and weights must be non-NULL"; return FFTSTENCIL_EINVAL; }
   if (radius < 1 || radius > kMaxRadius) { err = "radius must be in 1..8"; return FFTSTENCIL_EINVAL; }
@@ -210,7 +211,57 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     p.nt[a] = ceil_div(p.ext[a] - 2 * p.h, p.S[a]);
     p.tiles *= p.nt[a];
   }
-  p.pairs = (p.tiles + 1) / 2;   // Double-layer Filling: tiles 2i (Re) and 2i+1 (Im)
+  // Double-layer Filling pairs (Eq. 9): along the innermost tile axis within one outer
+  // tile row/line (kernels.cuh), so a decomposition by whole tile rows keeps every pair.
+  const int inner = ndim - 1;
+  p.npr = (p.nt[inner] + 1) / 2;
+  p.pairs = p.tiles / p.nt[inner] * p.npr;
+
+  // ---- outer-axis decomposition: whole units per rank (DESIGN.md a10) ----
+  {
+    const int64_t n0 = p.ext[0];
+    int64_t US;                        // outer rows per unit
+    if (ndim == 1) {
+      p.units = p.pairs;
+      p.pairs_per_unit = 1;
+      US = 2 * (int64_t)p.S[0];
+    } else {
+      p.units = p.nt[0];
+      p.pairs_per_unit = p.pairs / p.nt[0];
+      US = p.S[0];
+    }
+    p.nranks = nranks;
+    p.rank = rank;
+    if (p.units < nranks) { err = "fewer outer tile rows than ranks"; return FFTSTENCIL_EINVAL; }
+    p.unit_lo = p.units * rank / nranks;
+    p.unit_hi = p.units * (rank + 1) / nranks;
+    p.row_lo = rank == 0 ? 0 : p.unit_lo * US + p.h;
+    p.row_hi = rank == nranks - 1 ? n0 : p.unit_hi * US + p.h;
+    if (nranks > 1) {
+      for (int k = 0; k < nranks; ++k) {   // every slab must cover one halo (ghosts = neighbours only)
+        const int64_t ul = p.units * k / nranks, uh = p.units * (k + 1) / nranks;
+        const int64_t s = k == 0 ? 0 : ul * US + p.h, e = k == nranks - 1 ? n0 : uh * US + p.h;
+        if (e - s < p.h) { err = "a rank's slab is thinner than the halo r*T"; return FFTSTENCIL_EINVAL; }
+      }
+    }
+    p.g0 = std::max<int64_t>(0, p.row_lo - p.h);
+    p.g1 = std::min<int64_t>(n0, p.row_hi + p.h);
+    p.pair_lo = p.unit_lo * p.pairs_per_unit;
+    p.pair_hi = p.unit_hi * p.pairs_per_unit;
+    // interior units: every input row of the unit's tiles lies in the owned rows
+    const int64_t span = ndim == 1 ? (int64_t)p.S[0] + p.L[0] : p.L[0];   // input rows of a unit
+    int64_t ilo = p.unit_hi, ihi = p.unit_hi;
+    for (int64_t u = p.unit_lo; u < p.unit_hi; ++u) {
+      const int64_t in_lo = u * US, in_hi = std::min<int64_t>(n0, u * US + span);
+      if (in_lo >= p.row_lo && in_hi <= p.row_hi) {
+        if (ilo == p.unit_hi) ilo = u;
+        ihi = u + 1;
+      }
+    }
+    if (ilo == p.unit_hi) ilo = ihi = p.unit_lo;
+    p.ipair_lo = ilo * p.pairs_per_unit;
+    p.ipair_hi = ihi * p.pairs_per_unit;
+  }
 
   // ---- DFT matrices (forward; the kernel conjugates for the inverse, L258/L278) ----
   if (ndim == 1) {
@@ -292,7 +343,9 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       b.lo[e] = side == 0 ? 0 : p.n[e] - r;
       b.hi[e] = side == 0 ? r : p.n[e];
       for (int c = 0; c < a; ++c) { b.lo[off + c] = r; b.hi[off + c] = p.n[off + c] - r; }
-      p.ring_boxes.push_back(b);
+      b.lo[off] = std::max<int64_t>(b.lo[off], p.row_lo);   // this rank's rows only
+      b.hi[off] = std::min<int64_t>(b.hi[off], p.row_hi);
+      if (b.hi[off] > b.lo[off]) p.ring_boxes.push_back(b);
     }
   }
   // ---- boundary band: interior cells outside the exact region [h, n-h) (reading Q5) ----
@@ -313,6 +366,8 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
           b.hi[ec] = c < a ? p.n[ec] - h : p.n[ec] - r;
         }
         b.face = e;
+        b.lo[off] = std::max<int64_t>(b.lo[off], p.row_lo);   // this rank's rows only
+        b.hi[off] = std::min<int64_t>(b.hi[off], p.row_hi);
         bool empty = false;
         for (int q = 0; q < 3; ++q) empty |= b.hi[q] <= b.lo[q];
         if (!empty) p.band_boxes.push_back(b);

@@ -39,6 +39,15 @@ struct HostPlan {
   int N1 = 0, N2 = 0;              // 1D prime-factor split
   int64_t nt[3] = {1, 1, 1};       // tiles per user axis
   int64_t tiles = 0, pairs = 0;
+  int64_t npr = 1;                 // pairs per outer tile row (2D) / tile line (3D)
+  // ---- outer-axis decomposition (a10; nranks = 1 on a single GPU) ----
+  // Unit of the partition: one outer tile row (2D/3D: S rows) or one pair (1D: 2S cells).
+  int nranks = 1, rank = 0;
+  int64_t units = 0, unit_lo = 0, unit_hi = 0, pairs_per_unit = 1;
+  int64_t row_lo = 0, row_hi = 0;    // owned global outer rows [row_lo, row_hi)
+  int64_t g0 = 0, g1 = 0;            // buffer window: owned rows + ghosts, [g0, g1)
+  int64_t pair_lo = 0, pair_hi = 0;  // this rank's tile pairs
+  int64_t ipair_lo = 0, ipair_hi = 0;  // pairs whose inputs lie in owned rows (no ghosts)
   // Device-format auxiliary tables (planar re / im, row-major):
   //   2D/3D: F is L x L;  1D: F holds F_N1 (8x8) then F_N2 zero-padded to 8x8.
   std::vector<double> Fre, Fim;
@@ -56,8 +65,9 @@ struct HostPlan {
 };
 
 // Builds the plan; returns 0 or a negative FFTSTENCIL_* code with `err` set.
+// nranks/rank select one slab of the outer-axis decomposition (1/0 = whole grid).
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
-                    HostPlan& p, std::string& err);
+                    HostPlan& p, std::string& err, int nranks = 1, int rank = 0);
 
 // Dense-DFT tile cost model (executed FP64 tensor flops per cell-step) used to pick L/T.
 double model_flops_2d(int L, int S, int T);
