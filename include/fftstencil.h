@@ -85,6 +85,8 @@ typedef struct {
   int64_t pair_begin, pair_end; /* tile pairs this rank computes                         */
   int64_t interior_begin, interior_end; /* pairs needing no halo rows (overlap the exchange) */
   int64_t ghost_lo, ghost_hi;   /* halo rows received from rank-1 / rank+1 per pass     */
+  int algo;                     /* 2D tile algorithm: 0 dense L x L DFT GEMMs, 1 factored
+                                   64 = 8 x 8 (Cooley-Tukey, DFT-8 GEMMs + twiddles)       */
 } fftstencil_info;
 
 /* Build a plan (host precompute + device upload).  Returns NULL on error. */
@@ -160,8 +162,9 @@ int fftstencil_describe(int ndim, const int64_t* extents, const double* weights,
                         int T, fftstencil_info* info);
 
 /* Export the host plan's auxiliary tables, for tests of the plan builder:
- *   which = 0: forward DFT matrix of axis `axis` (1D: axis 0 -> F_N1, axis 1 -> F_N2),
- *              row-major L x L complex as interleaved (re, im) pairs, 2*L*L doubles;
+ *   which = 0: forward DFT matrix of axis `axis` (1D: axis 0 -> F_N1, axis 1 -> F_N2;
+ *              factored 2D plans: axis 0 -> F_8, axis 1 -> the twiddles w64^(ka*lb)),
+ *              row-major complex as interleaved (re, im) pairs;
  *   which = 1: powered spectrum S_t (t = `t`, 1..T) in the kernel's order (2D:
  *              natural [k0][k1]; 3D: [k1][k2][k0]; 1D: N1 x N2 matrix in the Ruritanian
  *              order of Eq. 8),

@@ -31,6 +31,15 @@ namespace {
 
 thread_local std::string g_last_error;
 
+// FFTSTENCIL_ALGO=dense|factored pins the 2D tile algorithm (ablations); default: cost model.
+int env_algo() {
+  const char* v = std::getenv("FFTSTENCIL_ALGO");
+  if (!v) return -1;
+  if (!std::strcmp(v, "dense")) return 0;
+  if (!std::strcmp(v, "factored")) return 1;
+  return -1;
+}
+
 void set_error(const std::string& s) { g_last_error = s; }
 void clear_error() { g_last_error.clear(); }
 
@@ -53,7 +62,8 @@ struct fftstencil_plan {
   size_t row_cells = 0;       // cells per outer-axis row
   size_t device_bytes = 0;
   int fused_grid = 0;
-  int variant = 0;            // fused-kernel variant (2D)
+  int variant = 0;            // fused-kernel variant (2D dense)
+  int ct_warps = 8;           // warps per CTA of the factored 2D kernel
   size_t band_smem = 0;
   int64_t last_launches = 0;
   // ---- decomposition (dist) ----
@@ -146,6 +156,7 @@ void fill_info(const HostPlan& hp, fftstencil_info* info) {
   info->interior_end = hp.ipair_hi;
   info->ghost_lo = hp.row_lo - hp.g0;
   info->ghost_hi = hp.g1 - hp.row_hi;
+  info->algo = hp.algo;
 }
 
 // Profiling: a (start, end) event pair around one launch; returns the pair index or -1.
@@ -199,11 +210,16 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.nt1 = hp.nt[1];
     a.npr = hp.npr;
     a.win = win;
-    a.Fre = p->dF;
-    a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
     a.Sre = Sre;
     a.Sim = Sim;
-    e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(p->fused_grid, np), s);
+    a.Fre = p->dF;
+    if (hp.algo == 1) {
+      a.Fim = p->dF + 128;
+      e = launch_fused2d_ct(p->ct_warps, a, (int)std::min<int64_t>(p->fused_grid, np), s);
+    } else {
+      a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
+      e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(p->fused_grid, np), s);
+    }
   } else if (hp.ndim == 1) {
     Fft1dArgs a;
     a.src = src;
@@ -436,8 +452,8 @@ int setup_device(fftstencil_plan* p) {
   size_t acc = 0;
   std::vector<double> F(hp.Fre);
   F.insert(F.end(), hp.Fim.begin(), hp.Fim.end());
-  if (hp.ndim == 2) {
-    // the 2D kernel reads F with columns permuted within groups of 8 (device_common.cuh)
+  if (hp.ndim == 2 && hp.algo == 0) {
+    // the dense 2D kernel reads F with columns permuted within groups of 8 (device_common.cuh)
     const int L = hp.L[0];
     for (int plane = 0; plane < 2; ++plane)
       for (int r = 0; r < L; ++r)
@@ -476,7 +492,15 @@ int setup_device(fftstencil_plan* p) {
   p->device_bytes = acc;
 
   int occ = 0;
-  if (hp.ndim == 2) {
+  if (hp.ndim == 2 && hp.algo == 1) {
+    if (const char* v = std::getenv("FFTSTENCIL_CT_WARPS")) p->ct_warps = std::atoi(v);
+    if (p->ct_warps != 8 && p->ct_warps != 16) {
+      set_error("FFTSTENCIL_CT_WARPS must be 8 or 16");
+      return FFTSTENCIL_EINVAL;
+    }
+    e = fused2d_ct_configure(p->ct_warps, &occ);
+    if (e != cudaSuccess) return cuda_fail(e, "factored 2D kernel configuration");
+  } else if (hp.ndim == 2) {
     // double-buffered prefetch pays only where it does not cost occupancy (profiles/r01_variants.txt)
     p->variant = hp.L[0] >= 56 ? 1 : 0;
     if (const char* v = std::getenv("FFTSTENCIL_VARIANT")) p->variant = std::atoi(v);
@@ -522,7 +546,7 @@ int fftstencil_describe_dist(int ndim, const int64_t* extents, const double* wei
   if (!info) { set_error("info must be non-NULL"); return FFTSTENCIL_EINVAL; }
   HostPlan hp;
   std::string err;
-  const int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, nranks, rank);
+  const int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, nranks, rank, env_algo());
   if (rc != FFTSTENCIL_OK) { set_error(err); return rc; }
   fill_info(hp, info);
   clear_error();
@@ -533,7 +557,7 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
                               int which, int axis, int t, double* out, int64_t cap) {
   HostPlan hp;
   std::string err;
-  const int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err);
+  const int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, 1, 0, env_algo());
   if (rc != FFTSTENCIL_OK) { set_error(err); return rc; }
   std::vector<double> v;
   if (which == 0) {
@@ -542,6 +566,11 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
       if (axis < 0 || axis > 1) { set_error("axis must be 0 (N1) or 1 (N2) for 1D"); return FFTSTENCIL_EINVAL; }
       L = axis == 0 ? hp.N1 : hp.N2;
       row0 = axis == 0 ? 0 : 8;
+      ld = 8;
+    } else if (hp.ndim == 2 && hp.algo == 1) {
+      if (axis < 0 || axis > 1) { set_error("axis must be 0 (F_8) or 1 (twiddles)"); return FFTSTENCIL_EINVAL; }
+      L = 8;
+      row0 = 8 * axis;
       ld = 8;
     } else {
       if (axis < 0 || axis >= hp.ndim) { set_error("axis out of range"); return FFTSTENCIL_EINVAL; }
@@ -601,7 +630,7 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
   fftstencil_plan* p = new (std::nothrow) fftstencil_plan();
   if (!p) { set_error("host allocation failed"); return nullptr; }
   std::string err;
-  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err);
+  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err, 1, 0, env_algo());
   if (rc != FFTSTENCIL_OK) { set_error(err); delete p; return nullptr; }
   if (setup_device(p) != FFTSTENCIL_OK) { free_plan(p); return nullptr; }
   clear_error();
@@ -614,7 +643,7 @@ fftstencil_plan* fftstencil_plan_create_dist(int ndim, const int64_t* extents, c
   fftstencil_plan* p = new (std::nothrow) fftstencil_plan();
   if (!p) { set_error("host allocation failed"); return nullptr; }
   std::string err;
-  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err, nranks, rank);
+  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err, nranks, rank, env_algo());
   if (rc != FFTSTENCIL_OK) { set_error(err); delete p; return nullptr; }
   p->dist = true;
   p->loopback = nccl_unique_id == nullptr;

@@ -1,0 +1,235 @@
+// Fused 2D FFT-stencil tile kernel with FACTORED DFT GEMMs: 64 = 8 x 8 per axis (sm_100a).
+//
+// The same fused pass as kernel_fft2d.cu (Algorithm 1, Double-layer
+// Filling Eq. 9, temporal fusion Eq. 10, Stitching Eq. 7), but each length-64 axis DFT is
+// factored the way §3.2.1 factors the 1D transform (L208-L218: reshape a length-N DFT into
+// a 2D one so the tensor cores see dense 8x8 matrices), here by Cooley-Tukey:
+//     x[8 la + lb] --(DFT8 over la)--> * w64^(ka lb) --(DFT8 over lb)--> X[ka + 8 kb]
+// so every GEMM is a dense DFT-8 (8x8, K = 8 = two DMMA.8x8x4 k-steps) and the work per
+// element and axis drops from 8L = 512 to 2 x 64 (+ 6 for the twiddle) flops.  F8 and the
+// per-thread twiddles live in registers for the whole launch (Squeezing Registers, L274).
+//
+// Each 64-element line (row or column of the tile) is one 8x8 complex matrix held by one
+// warp in m8n8k4 fragments.  Chaining without shared memory (Swizzling Fragments L266-L272)
+// uses two register routes, both contracting the columns of the current C fragment:
+//   B-route  C' = F8 . C^T     (C's fragment is the B fragment of C^T)  -> rows from F8
+//   A-route  C' = C . F8^T     (C's fragment is the A fragment of C)    -> rows stay C's
+// Per tile pair (Re = tile 2j, Im = tile 2j+1 of one outer tile row):
+//   phase 1  rows l0 (64):     DFT8 over la1, twiddle, A-route DFT8 over lb1   -> row of Q
+//   phase 2  columns k1 (64):  DFT8 over la0, twiddle, A-route DFT8 over lb0,
+//                              * S_T (Eq. 10), B-route iDFT8 over kb0, twiddle*,
+//                              A-route iDFT8 over ka0                          -> column of W
+//   phase 3  output rows (S):  iDFT8 over kb1, twiddle*, B-route iDFT8 over ka1 -> store
+// Phases 1 and 2 overwrite exactly the shared-memory words each thread read (in place);
+// the two CTA barriers are the transpositions of ownership a 2D transform needs.
+// Shared layout: plane[r][c] at r*97 + c + 8*(c>>4) + 8*((r>>4)&1): both the row pattern
+// (c = 16q + 8j + g) and the column pattern (r = 16q + 8j + g) hit every bank pair twice.
+#include "device_common.cuh"
+#include "kernels.cuh"
+
+namespace fstencil {
+namespace {
+
+using dev::dmma;
+
+constexpr int L = 64;
+constexpr int LDR = 97;
+constexpr int PLANE = L * LDR;
+
+__device__ __forceinline__ int sw(int r, int c) { return r * LDR + c + 8 * (c >> 4) + 8 * ((r >> 4) & 1); }
+
+__device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
+}
+
+// B-route: C = F8 . B (F8 fragments f*, data fragments b*), CONJ -> conj(F8).
+template <bool CONJ>
+__device__ __forceinline__ void broute(double (&cr)[2], double (&ci)[2], const double (&fr)[2], const double (&fi)[2],
+                                       const double (&br)[2], const double (&bi)[2]) {
+  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    if (CONJ) {
+      dmma(cr, fr[j], br[j]);
+      dmma(ci, fr[j], bi[j]);
+      dmma(cr, fi[j], bi[j]);
+      dmma(ci, -fi[j], br[j]);
+    } else {
+      dmma(cr, fr[j], br[j]);
+      dmma(ci, fr[j], bi[j]);
+      dmma(cr, -fi[j], bi[j]);
+      dmma(ci, fi[j], br[j]);
+    }
+  }
+}
+
+// A-route: C = D . F8^T (data fragments d* as A, F8^T fragments = F8 fragments as B).
+template <bool CONJ>
+__device__ __forceinline__ void aroute(double (&cr)[2], double (&ci)[2], const double (&dr)[2], const double (&di)[2],
+                                       const double (&fr)[2], const double (&fi)[2]) {
+  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    if (CONJ) {
+      dmma(cr, dr[j], fr[j]);
+      dmma(ci, di[j], fr[j]);
+      dmma(cr, di[j], fi[j]);
+      dmma(ci, -dr[j], fi[j]);
+    } else {
+      dmma(cr, dr[j], fr[j]);
+      dmma(ci, di[j], fr[j]);
+      dmma(cr, -di[j], fi[j]);
+      dmma(ci, dr[j], fi[j]);
+    }
+  }
+}
+
+template <bool CONJ>
+__device__ __forceinline__ void twiddle(double (&cr)[2], double (&ci)[2], const double (&tr)[2], const double (&ti)[2]) {
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const double t_i = CONJ ? -ti[j] : ti[j];
+    const double r = cr[j] * tr[j] - ci[j] * t_i;
+    const double i = cr[j] * t_i + ci[j] * tr[j];
+    cr[j] = r;
+    ci[j] = i;
+  }
+}
+
+template <int NW>
+__global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a) {
+  extern __shared__ __align__(16) double smem[];
+  double* sR = smem;            // plane 0: tile 2j (Re), then Q/W real parts
+  double* sI = smem + PLANE;    // plane 1: tile 2j+1 (Im), then Q/W imaginary parts
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31, g = lane >> 2, q = lane & 3;
+
+  // register-resident F8 fragments (row g, logical column 2q+j) and twiddles w64^(g (2q+j))
+  double fr[2], fi[2], tr[2], ti[2];
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const int c = 2 * q + j;
+    fr[j] = a.Fre[g * 8 + c];
+    fi[j] = a.Fim[g * 8 + c];
+    tr[j] = a.Fre[64 + g * 8 + c];
+    ti[j] = a.Fim[64 + g * 8 + c];
+  }
+  const int S = a.S, h = a.h;
+  int cl[2];                     // the thread's line positions 16q + 8j + g
+#pragma unroll
+  for (int j = 0; j < 2; ++j) cl[j] = 16 * q + 8 * j + g;
+
+  for (int64_t p = a.win.p_begin + blockIdx.x; p < a.win.p_end; p += gridDim.x) {
+    const int64_t t0 = p / a.npr, pj = p - t0 * a.npr;
+    const int64_t o0 = t0 * S, oa1 = 2 * pj * S, ob1 = oa1 + S;
+    const bool has_b = 2 * pj + 1 < a.nt1;
+    __syncthreads();   // previous pair's phase 3 reads are done
+    // ---- load the halo'd pair (cp.async, OOB = 0) ----
+    for (int e = tid; e < 2 * L * L; e += NW * 32) {
+      const int t = e >> 12, r = (e >> 6) & 63, c = e & 63;
+      const int64_t gr = o0 + r, gc = (t ? ob1 : oa1) + c, lr = gr - a.win.g0;
+      const bool valid = (t == 0 || has_b) && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc < a.n1;
+      cp_async8((t ? sI : sR) + sw(r, c), valid ? a.src + lr * a.n1 + gc : a.src, valid);
+    }
+    asm volatile("cp.async.commit_group;\n" ::);
+    asm volatile("cp.async.wait_all;\n" ::: "memory");
+    __syncthreads();
+
+    // ---- phase 1: forward DFT along axis 1, every row ----
+    for (int l0 = warp; l0 < L; l0 += NW) {
+      double br[2], bi[2], c1r[2], c1i[2], c2r[2], c2i[2];
+#pragma unroll
+      for (int j = 0; j < 2; ++j) { br[j] = sR[sw(l0, cl[j])]; bi[j] = sI[sw(l0, cl[j])]; }
+      broute<false>(c1r, c1i, fr, fi, br, bi);     // [ka1][lb1]
+      twiddle<false>(c1r, c1i, tr, ti);
+      aroute<false>(c2r, c2i, c1r, c1i, fr, fi);   // [ka1][kb1]: k1 = g + 8(2q+j) = cl[j]
+#pragma unroll
+      for (int j = 0; j < 2; ++j) { sR[sw(l0, cl[j])] = c2r[j]; sI[sw(l0, cl[j])] = c2i[j]; }
+    }
+    __syncthreads();
+
+    // ---- phase 2: axis 0 forward, * S_T, axis 0 inverse, every column ----
+    for (int k1 = warp; k1 < L; k1 += NW) {
+      double br[2], bi[2], c1r[2], c1i[2], c2r[2], c2i[2];
+#pragma unroll
+      for (int j = 0; j < 2; ++j) { br[j] = sR[sw(cl[j], k1)]; bi[j] = sI[sw(cl[j], k1)]; }
+      broute<false>(c1r, c1i, fr, fi, br, bi);     // [ka0][lb0]
+      twiddle<false>(c1r, c1i, tr, ti);
+      aroute<false>(c2r, c2i, c1r, c1i, fr, fi);   // [ka0][kb0]: k0 = cl[j]
+      {
+        const double2 sr = __ldg(reinterpret_cast<const double2*>(a.Sre + k1 * 64 + g * 8 + 2 * q));
+        const double2 si = __ldg(reinterpret_cast<const double2*>(a.Sim + k1 * 64 + g * 8 + 2 * q));
+        const double s_r[2] = {sr.x, sr.y}, s_i[2] = {si.x, si.y};
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const double r = c2r[j] * s_r[j] - c2i[j] * s_i[j];
+          const double i = c2r[j] * s_i[j] + c2i[j] * s_r[j];
+          c2r[j] = r;
+          c2i[j] = i;
+        }
+      }
+      broute<true>(c1r, c1i, fr, fi, c2r, c2i);    // [lb0][ka0]
+      twiddle<true>(c1r, c1i, tr, ti);
+      aroute<true>(c2r, c2i, c1r, c1i, fr, fi);    // [lb0][la0]: l0 = cl[j]
+#pragma unroll
+      for (int j = 0; j < 2; ++j) { sR[sw(cl[j], k1)] = c2r[j]; sI[sw(cl[j], k1)] = c2i[j]; }
+    }
+    __syncthreads();
+
+    // ---- phase 3: inverse DFT along axis 1 on the S output rows, store the window ----
+    for (int i = warp; i < S; i += NW) {
+      const int l0 = h + i;
+      const int64_t c0 = o0 + l0;
+      if (c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
+      double br[2], bi[2], c1r[2], c1i[2], c2r[2], c2i[2];
+#pragma unroll
+      for (int j = 0; j < 2; ++j) { br[j] = sR[sw(l0, cl[j])]; bi[j] = sI[sw(l0, cl[j])]; }
+      broute<true>(c1r, c1i, fr, fi, br, bi);      // [lb1][ka1]
+      twiddle<true>(c1r, c1i, tr, ti);
+      broute<true>(c2r, c2i, fr, fi, c1r, c1i);    // [la1][lb1]: l1 = 8g + 2q + j
+      double* drow = a.dst + (c0 - a.win.g0) * a.n1;
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const int l1 = 8 * g + 2 * q + j;
+        if (l1 >= h && l1 < h + S) {
+          int64_t c1 = oa1 + l1;
+          if (c1 < a.n1 - h) drow[c1] = c2r[j];
+          c1 = ob1 + l1;
+          if (has_b && c1 < a.n1 - h) drow[c1] = c2i[j];
+        }
+      }
+    }
+  }
+}
+
+template <int NW>
+cudaError_t configure_nw(int* max_blocks) {
+  const size_t smem = fused2d_ct_smem();
+  cudaError_t e = cudaFuncSetAttribute(fft2d_ct_kernel<NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_ct_kernel<NW>, NW * 32, smem);
+}
+
+}  // namespace
+
+size_t fused2d_ct_smem() { return (size_t)2 * PLANE * sizeof(double); }
+
+cudaError_t fused2d_ct_configure(int nw, int* max_blocks) {
+  switch (nw) {
+    case 8: return configure_nw<8>(max_blocks);
+    case 16: return configure_nw<16>(max_blocks);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+cudaError_t launch_fused2d_ct(int nw, const Fft2dArgs& a, int grid, cudaStream_t s) {
+  switch (nw) {
+    case 8: fft2d_ct_kernel<8><<<grid, 8 * 32, fused2d_ct_smem(), s>>>(a); break;
+    case 16: fft2d_ct_kernel<16><<<grid, 16 * 32, fused2d_ct_smem(), s>>>(a); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace fstencil

@@ -100,6 +100,13 @@ size_t fused2d_smem(int L, int V);
 cudaError_t fused2d_configure(int L, int V, int* max_blocks_per_sm);
 cudaError_t launch_fused2d(int L, int V, const Fft2dArgs& a, int grid, cudaStream_t s);
 
+// Factored-DFT 2D kernel (kernel_fft2d_ct.cu): L = 64 = 8 x 8 Cooley-Tukey per axis.
+// Fre/Fim = [F8 (8x8) | twiddles w64^(ka lb) (8x8)]; Sre/Sim = S_T in [k1][8 g + c] order with
+// k0 = g + 8 c.  nw = warps per CTA (8 or 16).
+size_t fused2d_ct_smem();
+cudaError_t fused2d_ct_configure(int nw, int* max_blocks_per_sm);
+cudaError_t launch_fused2d_ct(int nw, const Fft2dArgs& a, int grid, cudaStream_t s);
+
 constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused1d(const Fft1dArgs& a, int grid, cudaStream_t s);

@@ -61,6 +61,16 @@ double model_flops_2d(int L, int S, int T) {
   return 8.0 * dm / (2.0 * S * (double)S * T);
 }
 
+// Factored tile (kernel_fft2d_ct.cu), per pair: DMMA.8x8x4 x 512 flops for 64 rows x 2
+// stages + 64 columns x 4 stages + S rows x 2 stages (8 DMMA per stage and line), twiddles
+// (6 flops per element, 192 + S lines of 64) and the S_T multiply (6 flops per element).
+double model_flops_2d_ct(int S, int T) {
+  const double f = 512.0 * (3072.0 + 16.0 * S) + 384.0 * (192.0 + S) + 6.0 * 4096.0;
+  return f / (2.0 * S * (double)S * T);
+}
+
+static constexpr double kEffCt = 0.70;   // assumed until measured (profiles/)
+
 // Measured DMMA issue efficiency of the fused 2D kernel per tile side (fraction of the
 // 37.18 TF/s peak, B200, profiles/r01_sweep.txt / r01_variants.txt): the plan minimises
 // executed flops / efficiency, i.e. predicted time per cell-step (the role of Eq. 5's
@@ -88,7 +98,7 @@ static double model_flops_1d(int S, int T) {  // one 8x8 complex tile, 4 GEMMs o
 }
 
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
-                    HostPlan& p, std::string& err, int nranks, int rank) {
+                    HostPlan& p, std::string& err, int nranks, int rank, int algo) {
   p = HostPlan();
   if (nranks < 1 || rank < 0 || rank >= nranks) { err = "need 0 <= rank < nranks"; return FFTSTENCIL_EINVAL; }
   if (ndim < 1 || ndim > 3) { err = "ndim must be 1, 2 or 3"; return FFTSTENCIL_EINVAL; }
@@ -138,43 +148,49 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     p.flops_per_cell_step = (16.0 * p.N1 * p.N2 * (p.N1 + p.N2) + 6.0 * p.N1 * p.N2) / (2.0 * p.S[0] * p.T);
     p.mma_flops_per_pair = 32.0 * 512.0;
   } else if (ndim == 2) {
+    // candidates: dense L x L DFT tiles and the factored 64 = 8 x 8 tile (NEXT-1)
     static const int cand[] = {16, 24, 32, 40, 48, 56, 64};
+    auto cost = [&](int al, int L, int S, int t) {
+      return al ? model_flops_2d_ct(S, t) / kEffCt : model_flops_2d(L, S, t) / eff_2d(L);
+    };
     double best = 1e300;
-    int bL = 0, bT = 0;
+    int bL = 0, bT = 0, bA = 0;
     const int tlo = T == 0 ? 1 : T, thi = T == 0 ? 16 : T;
-    for (int t = tlo; t <= thi; ++t) {
-      const int h = radius * t;
-      if (h > hmax_grid) break;
-      for (int L : cand) {
-        const int S = L - 2 * h;
-        if (S < 8) continue;
-        const double f = model_flops_2d(L, S, t) / eff_2d(L);
-        if (f < best * (1 - 1e-12)) { best = f; bL = L; bT = t; }
-      }
-    }
-    if (bL == 0) {
-      // requested T too deep for the largest tile or the grid: lower it.
-      for (int t = std::min(thi, 64); t >= 1 && bL == 0; --t) {
+    for (int pass = 0; pass < 2 && bL == 0; ++pass) {
+      // pass 0: the requested T (or the auto range); pass 1: lower a too-deep T
+      const int a0 = pass == 0 ? tlo : 1, a1 = pass == 0 ? thi : std::min(thi, 64);
+      for (int t = a0; t <= a1; ++t) {
         const int h = radius * t;
-        if (h > hmax_grid) continue;
-        for (int L : cand) {
-          const int S = L - 2 * h;
-          if (S < 8) continue;
-          const double f = model_flops_2d(L, S, t) / eff_2d(L);
-          if (f < best) { best = f; bL = L; bT = t; }
+        if (h > hmax_grid) break;
+        for (int al = 0; al < 2; ++al) {
+          if (algo >= 0 && al != algo) continue;
+          for (int L : cand) {
+            if (al == 1 && L != 64) continue;
+            const int S = L - 2 * h;
+            if (S < 8) continue;
+            const double f = cost(al, L, S, t);
+            if (f < best * (1 - 1e-12)) { best = f; bL = L; bT = t; bA = al; }
+          }
         }
       }
     }
     if (bL == 0) { err = "no 2D tile fits this radius/grid"; return FFTSTENCIL_EINVAL; }
+    p.algo = bA;
     p.T = bT;
     p.h = radius * bT;
     p.L[0] = p.L[1] = bL;
     p.S[0] = p.S[1] = bL - 2 * p.h;
     const double L = bL, S = p.S[0];
-    p.flops_per_cell_step = (16.0 * L * L * L + 6.0 * L * L + 8.0 * S * L * L + 8.0 * S * S * L) / (2.0 * S * S * bT);
-    const double Sp = round8(p.S[0]);
-    p.mma_flops_per_pair = 8.0 * (2.0 * L * L * L + Sp * L * L + Sp * Sp * L);
-    p.fused_smem = (size_t)(bL >= 56 ? 48 : 32) * bL * (bL + 4);   // F + pair buffer(s)
+    if (bA == 0) {
+      p.flops_per_cell_step = (16.0 * L * L * L + 6.0 * L * L + 8.0 * S * L * L + 8.0 * S * S * L) / (2.0 * S * S * bT);
+      const double Sp = round8(p.S[0]);
+      p.mma_flops_per_pair = 8.0 * (2.0 * L * L * L + Sp * L * L + Sp * Sp * L);
+      p.fused_smem = (size_t)(bL >= 56 ? 48 : 32) * bL * (bL + 4);   // F + pair buffer(s)
+    } else {
+      p.flops_per_cell_step = model_flops_2d_ct(p.S[0], bT);
+      p.mma_flops_per_pair = 512.0 * (3072.0 + 16.0 * S);
+      p.fused_smem = (size_t)2 * 64 * 97 * sizeof(double);
+    }
   } else {
     const int L = k3DTile;
     const int hmax = std::min(hmax_grid, (L - 2) / 2);
@@ -272,6 +288,17 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     p.crt.assign(64, -1);
     const int L = p.N1 * p.N2;
     for (int l = 0; l < L; ++l) p.crt[(l % p.N1) * 8 + (l % p.N2)] = l;   // diagonal / CRT map
+  } else if (ndim == 2 && p.algo == 1) {
+    // [F8 | twiddles w64^(ka lb)], 8 x 8 each (kernel_fft2d_ct.cu)
+    p.Fre.assign(128, 0.0);
+    p.Fim.assign(128, 0.0);
+    fill_dft(8, 8, 0, 0, p.Fre, p.Fim);
+    for (int ka = 0; ka < 8; ++ka)
+      for (int lb = 0; lb < 8; ++lb) {
+        const cplx v = root((int64_t)ka * lb, 64);
+        p.Fre[64 + ka * 8 + lb] = v.real();
+        p.Fim[64 + ka * 8 + lb] = v.imag();
+      }
   } else {
     const int L = p.L[0];
     p.Fre.assign((size_t)L * L, 0.0);
@@ -325,6 +352,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         if (ndim == 3) {
           const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
           dst = k12 * L + k0;
+        } else if (p.algo == 1) {
+          // factored 2D: [k1][8 g + c] holds k0 = g + 8 c (digit order of the CT output)
+          const int64_t k0 = i / 64, k1 = i % 64;
+          dst = k1 * 64 + 8 * (k0 % 8) + k0 / 8;
         }
         re[dst] = v.real();
         im[dst] = v.imag();

@@ -37,6 +37,7 @@ struct HostPlan {
   int L[3] = {1, 1, 1};            // tile extent per user axis
   int S[3] = {1, 1, 1};            // valid extent per user axis
   int N1 = 0, N2 = 0;              // 1D prime-factor split
+  int algo = 0;                    // 2D: 0 = dense L x L DFT GEMMs, 1 = factored 64 = 8 x 8 (CT)
   int64_t nt[3] = {1, 1, 1};       // tiles per user axis
   int64_t tiles = 0, pairs = 0;
   int64_t npr = 1;                 // pairs per outer tile row (2D) / tile line (3D)
@@ -66,10 +67,13 @@ struct HostPlan {
 
 // Builds the plan; returns 0 or a negative FFTSTENCIL_* code with `err` set.
 // nranks/rank select one slab of the outer-axis decomposition (1/0 = whole grid).
+// algo (2D only): -1 = choose by the cost model, 0 = dense, 1 = factored (CT 8 x 8).
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
-                    HostPlan& p, std::string& err, int nranks = 1, int rank = 0);
+                    HostPlan& p, std::string& err, int nranks = 1, int rank = 0, int algo = -1);
 
 // Dense-DFT tile cost model (executed FP64 tensor flops per cell-step) used to pick L/T.
 double model_flops_2d(int L, int S, int T);
+// Factored (CT 8 x 8, L = 64) tile: executed FP64 flops per cell-step (DMMA + twiddles + S_T).
+double model_flops_2d_ct(int S, int T);
 
 }  // namespace fstencil
