@@ -63,7 +63,8 @@ struct fftstencil_plan {
   size_t device_bytes = 0;
   int fused_grid = 0;
   int variant = 0;            // fused-kernel variant (2D dense)
-  int ct_warps = 8;           // warps per CTA of the factored 2D kernel
+  int ct_cfg = 82;            // factored 2D kernel: 10 * warps per CTA + lines per warp step
+  int band_reference = 0;     // FFTSTENCIL_BAND=reference selects the first band kernel
   size_t band_smem = 0;
   int64_t last_launches = 0;
   // ---- decomposition (dist) ----
@@ -215,7 +216,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Fre = p->dF;
     if (hp.algo == 1) {
       a.Fim = p->dF + 128;
-      e = launch_fused2d_ct(p->ct_warps, a, (int)std::min<int64_t>(p->fused_grid, np), s);
+      e = launch_fused2d_ct(p->ct_cfg, a, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
       e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(p->fused_grid, np), s);
@@ -278,6 +279,7 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
   b.oax = 3 - hp.ndim;
   b.g0 = hp.g0;
   b.gn = hp.g1 - hp.g0;
+  b.reference = p->band_reference;
   const long pb = prof_begin(p, 1, s);
   cudaError_t e = launch_band(b, p->band_smem, s);
   prof_end(p, pb, s);
@@ -493,12 +495,12 @@ int setup_device(fftstencil_plan* p) {
 
   int occ = 0;
   if (hp.ndim == 2 && hp.algo == 1) {
-    if (const char* v = std::getenv("FFTSTENCIL_CT_WARPS")) p->ct_warps = std::atoi(v);
-    if (p->ct_warps != 8 && p->ct_warps != 16) {
-      set_error("FFTSTENCIL_CT_WARPS must be 8 or 16");
+    if (const char* v = std::getenv("FFTSTENCIL_CT_CFG")) p->ct_cfg = std::atoi(v);
+    e = fused2d_ct_configure(p->ct_cfg, &occ);
+    if (e == cudaErrorInvalidValue) {
+      set_error("FFTSTENCIL_CT_CFG must be one of 81, 82, 84, 161, 162");
       return FFTSTENCIL_EINVAL;
     }
-    e = fused2d_ct_configure(p->ct_warps, &occ);
     if (e != cudaSuccess) return cuda_fail(e, "factored 2D kernel configuration");
   } else if (hp.ndim == 2) {
     // double-buffered prefetch pays only where it does not cost occupancy (profiles/r01_variants.txt)
@@ -522,6 +524,7 @@ int setup_device(fftstencil_plan* p) {
     return FFTSTENCIL_EUNSUPPORTED;
   }
   p->fused_grid = (int)std::max<int64_t>(1, (int64_t)p->sm_count * occ);
+  if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
   p->band_smem = (size_t)2 * hp.band_region_cells * sizeof(double);
   if (p->band_smem > 0) {
     e = band_configure(p->band_smem);

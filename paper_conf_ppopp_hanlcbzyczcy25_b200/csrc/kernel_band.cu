@@ -82,6 +82,102 @@ __global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
   }
 }
 
+// Faster band kernel: the block's nonzero taps are compacted into shared memory with their
+// flattened region offsets; at step s only the dependency cone of the output block is
+// updated (distance >= r*s from every region edge that is not the grid boundary -- the
+// cells outside it are never read again), and threads map to (row, column) of the region
+// without per-cell divisions.  Same definition and result as band_kernel.
+constexpr int kMaxTaps = 512;
+
+__global__ void __launch_bounds__(kBandThreads) band_cone_kernel(const BandArgs a) {
+  extern __shared__ double sb[];
+  __shared__ int s_off[kMaxTaps];
+  __shared__ double s_w[kMaxTaps];
+  __shared__ int s_ntaps;
+  const int* blk = a.blocks + 8 * blockIdx.x;
+  int64_t lo[3], hi[3], rl[3], off[3] = {0, 0, 0};
+  int D[3], clo[3], chi[3];
+  bool open_lo[3], open_hi[3];
+  off[a.oax] = a.g0;
+#pragma unroll
+  for (int q = 0; q < 3; ++q) {
+    lo[q] = blk[q];
+    hi[q] = blk[3 + q];
+    const int64_t gq = a.active[q] ? (int64_t)a.r * a.t : 0;
+    int64_t l = max((int64_t)0, lo[q] - gq), u = min(a.n[q], hi[q] + gq);
+    if (q == a.oax) { l = max(l, a.g0); u = min(u, a.g0 + a.gn); }
+    rl[q] = l;
+    D[q] = (int)(u - l);
+    open_lo[q] = a.active[q] && l > 0;               // cells below were not loaded
+    open_hi[q] = a.active[q] && u < a.n[q];
+  }
+  const int r = a.r, wd = 2 * r + 1;
+  if (threadIdx.x == 0) {
+    int n = 0;
+    const int nw = (a.active[0] ? wd : 1) * (a.active[1] ? wd : 1) * (a.active[2] ? wd : 1);
+    int k = 0;
+    for (int o0 = a.active[0] ? -r : 0; o0 <= (a.active[0] ? r : 0); ++o0)
+      for (int o1 = a.active[1] ? -r : 0; o1 <= (a.active[1] ? r : 0); ++o1)
+        for (int o2 = a.active[2] ? -r : 0; o2 <= (a.active[2] ? r : 0); ++o2, ++k) {
+          const double wv = a.w[k];
+          if (wv != 0.0 && n < kMaxTaps) {
+            s_off[n] = (o0 * D[1] + o1) * D[2] + o2;
+            s_w[n] = wv;
+            ++n;
+          }
+        }
+    s_ntaps = n;
+    (void)nw;
+  }
+  const int vol = D[0] * D[1] * D[2];
+  double* b0 = sb;
+  double* b1 = sb + vol;
+  const int rows = D[0] * D[1];
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5, ny = kBandThreads / 32;
+  for (int row = ty; row < rows; row += ny) {
+    const int i0 = row / D[1], i1 = row - i0 * D[1];
+    const double* src = a.src + ((rl[0] + i0 - off[0]) * a.n[1] + (rl[1] + i1 - off[1])) * a.n[2] + (rl[2] - off[2]);
+    for (int i2 = tx; i2 < D[2]; i2 += 32) b0[row * D[2] + i2] = src[i2];
+  }
+  __syncthreads();
+  const int ntaps = s_ntaps;
+  for (int s = 1; s <= a.t; ++s) {
+#pragma unroll
+    for (int q = 0; q < 3; ++q) {
+      clo[q] = open_lo[q] ? r * s : 0;
+      chi[q] = D[q] - (open_hi[q] ? r * s : 0);
+    }
+    // cone box of this step, flattened over all threads (no idle lanes on narrow faces)
+    const int W0 = chi[0] - clo[0], W1 = chi[1] - clo[1], W2 = chi[2] - clo[2];
+    const int ncone = W0 * W1 * W2;
+    for (int f = threadIdx.x; f < ncone; f += kBandThreads) {
+      const int k2 = f % W2, k01 = f / W2, k1 = k01 % W1, k0 = k01 / W1;
+      const int i0 = clo[0] + k0, i1 = clo[1] + k1, i2 = clo[2] + k2;
+      const int e = (i0 * D[1] + i1) * D[2] + i2;
+      const int64_t c0 = rl[0] + i0, c1 = rl[1] + i1, c2 = rl[2] + i2;
+      double v;
+      if ((a.active[0] && (c0 < r || c0 >= a.n[0] - r)) || (a.active[1] && (c1 < r || c1 >= a.n[1] - r)) ||
+          (a.active[2] && (c2 < r || c2 >= a.n[2] - r))) {
+        v = b0[e];                                          // fixed ring
+      } else {
+        v = 0.0;
+        for (int k = 0; k < ntaps; ++k) v = fma(s_w[k], b0[e + s_off[k]], v);
+      }
+      b1[e] = v;
+    }
+    __syncthreads();
+    double* t = b0; b0 = b1; b1 = t;
+  }
+  const int O0 = (int)(hi[0] - lo[0]), O1 = (int)(hi[1] - lo[1]), O2 = (int)(hi[2] - lo[2]);
+  for (int row = ty; row < O0 * O1; row += ny) {
+    const int j0 = row / O1, j1 = row - j0 * O1;
+    const int64_t c0 = lo[0] + j0, c1 = lo[1] + j1;
+    double* dst = a.dst + ((c0 - off[0]) * a.n[1] + (c1 - off[1])) * a.n[2] + (lo[2] - off[2]);
+    const double* srow = b0 + ((c0 - rl[0]) * D[1] + (c1 - rl[1])) * D[2] + (lo[2] - rl[2]);
+    for (int j2 = tx; j2 < O2; j2 += 32) dst[j2] = srow[j2];
+  }
+}
+
 __global__ void box_copy_kernel(const BoxCopyArgs a) {
   const int64_t L0 = a.hi[0] - a.lo[0], L1 = a.hi[1] - a.lo[1], L2 = a.hi[2] - a.lo[2];
   const int64_t vol = L0 * L1 * L2;
@@ -101,12 +197,19 @@ __global__ void box_copy_kernel(const BoxCopyArgs a) {
 }  // namespace
 
 cudaError_t band_configure(size_t smem) {
-  return cudaFuncSetAttribute(band_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(band_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(band_cone_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
 }
 
 cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s) {
   if (a.nblocks <= 0) return cudaSuccess;
-  band_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
+  int taps = 1;
+  for (int q = 0; q < 3; ++q) taps *= a.active[q] ? 2 * a.r + 1 : 1;
+  if (taps <= kMaxTaps && !a.reference)
+    band_cone_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
+  else
+    band_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
   return cudaGetLastError();
 }
 

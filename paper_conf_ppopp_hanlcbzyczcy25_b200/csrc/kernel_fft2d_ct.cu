@@ -97,7 +97,53 @@ __device__ __forceinline__ void twiddle(double (&cr)[2], double (&ci)[2], const 
   }
 }
 
-template <int NW>
+// NL independent lines per warp, their DMMA chains interleaved for latency hiding.
+template <bool CONJ, int NL>
+__device__ __forceinline__ void broute_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&fr)[2],
+                                         const double (&fi)[2], const double (&br)[NL][2], const double (&bi)[NL][2]) {
+#pragma unroll
+  for (int u = 0; u < NL; ++u) cr[u][0] = cr[u][1] = ci[u][0] = ci[u][1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const double nfi = CONJ ? fi[j] : -fi[j];   // coefficient of bi in cr
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(cr[u], fr[j], br[u][j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(ci[u], fr[j], bi[u][j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(cr[u], nfi, bi[u][j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(ci[u], -nfi, br[u][j]);
+  }
+}
+
+template <bool CONJ, int NL>
+__device__ __forceinline__ void aroute_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&dr)[NL][2],
+                                         const double (&di)[NL][2], const double (&fr)[2], const double (&fi)[2]) {
+#pragma unroll
+  for (int u = 0; u < NL; ++u) cr[u][0] = cr[u][1] = ci[u][0] = ci[u][1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const double nfi = CONJ ? fi[j] : -fi[j];
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(cr[u], dr[u][j], fr[j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(ci[u], di[u][j], fr[j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(cr[u], di[u][j], nfi);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(ci[u], dr[u][j], -nfi);
+  }
+}
+
+template <bool CONJ, int NL>
+__device__ __forceinline__ void twiddle_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&tr)[2],
+                                          const double (&ti)[2]) {
+#pragma unroll
+  for (int u = 0; u < NL; ++u) twiddle<CONJ>(cr[u], ci[u], tr, ti);
+}
+
+template <int NW, int NL>
 __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a) {
   extern __shared__ __align__(16) double smem[];
   double* sR = smem;            // plane 0: tile 2j (Re), then Q/W real parts
@@ -136,97 +182,138 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a) {
     asm volatile("cp.async.wait_all;\n" ::: "memory");
     __syncthreads();
 
-    // ---- phase 1: forward DFT along axis 1, every row ----
-    for (int l0 = warp; l0 < L; l0 += NW) {
-      double br[2], bi[2], c1r[2], c1i[2], c2r[2], c2i[2];
+    // ---- phase 1: forward DFT along axis 1, every row (NL rows per warp step) ----
+    for (int l0b = warp * NL; l0b < L; l0b += NW * NL) {
+      double br[NL][2], bi[NL][2], c1r[NL][2], c1i[NL][2], c2r[NL][2], c2i[NL][2];
 #pragma unroll
-      for (int j = 0; j < 2; ++j) { br[j] = sR[sw(l0, cl[j])]; bi[j] = sI[sw(l0, cl[j])]; }
-      broute<false>(c1r, c1i, fr, fi, br, bi);     // [ka1][lb1]
-      twiddle<false>(c1r, c1i, tr, ti);
-      aroute<false>(c2r, c2i, c1r, c1i, fr, fi);   // [ka1][kb1]: k1 = g + 8(2q+j) = cl[j]
+      for (int u = 0; u < NL; ++u)
 #pragma unroll
-      for (int j = 0; j < 2; ++j) { sR[sw(l0, cl[j])] = c2r[j]; sI[sw(l0, cl[j])] = c2i[j]; }
+        for (int j = 0; j < 2; ++j) {
+          br[u][j] = sR[sw(l0b + u, cl[j])];
+          bi[u][j] = sI[sw(l0b + u, cl[j])];
+        }
+      broute_n<false, NL>(c1r, c1i, fr, fi, br, bi);     // [ka1][lb1]
+      twiddle_n<false, NL>(c1r, c1i, tr, ti);
+      aroute_n<false, NL>(c2r, c2i, c1r, c1i, fr, fi);   // [ka1][kb1]: k1 = g + 8(2q+j) = cl[j]
+#pragma unroll
+      for (int u = 0; u < NL; ++u)
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          sR[sw(l0b + u, cl[j])] = c2r[u][j];
+          sI[sw(l0b + u, cl[j])] = c2i[u][j];
+        }
     }
     __syncthreads();
 
     // ---- phase 2: axis 0 forward, * S_T, axis 0 inverse, every column ----
-    for (int k1 = warp; k1 < L; k1 += NW) {
-      double br[2], bi[2], c1r[2], c1i[2], c2r[2], c2i[2];
+    for (int k1b = warp * NL; k1b < L; k1b += NW * NL) {
+      double br[NL][2], bi[NL][2], c1r[NL][2], c1i[NL][2], c2r[NL][2], c2i[NL][2];
+      double s_r[NL][2], s_i[NL][2];
 #pragma unroll
-      for (int j = 0; j < 2; ++j) { br[j] = sR[sw(cl[j], k1)]; bi[j] = sI[sw(cl[j], k1)]; }
-      broute<false>(c1r, c1i, fr, fi, br, bi);     // [ka0][lb0]
-      twiddle<false>(c1r, c1i, tr, ti);
-      aroute<false>(c2r, c2i, c1r, c1i, fr, fi);   // [ka0][kb0]: k0 = cl[j]
-      {
-        const double2 sr = __ldg(reinterpret_cast<const double2*>(a.Sre + k1 * 64 + g * 8 + 2 * q));
-        const double2 si = __ldg(reinterpret_cast<const double2*>(a.Sim + k1 * 64 + g * 8 + 2 * q));
-        const double s_r[2] = {sr.x, sr.y}, s_i[2] = {si.x, si.y};
+      for (int u = 0; u < NL; ++u) {
+        const double2 sr = __ldg(reinterpret_cast<const double2*>(a.Sre + (k1b + u) * 64 + g * 8 + 2 * q));
+        const double2 si = __ldg(reinterpret_cast<const double2*>(a.Sim + (k1b + u) * 64 + g * 8 + 2 * q));
+        s_r[u][0] = sr.x; s_r[u][1] = sr.y; s_i[u][0] = si.x; s_i[u][1] = si.y;
 #pragma unroll
         for (int j = 0; j < 2; ++j) {
-          const double r = c2r[j] * s_r[j] - c2i[j] * s_i[j];
-          const double i = c2r[j] * s_i[j] + c2i[j] * s_r[j];
-          c2r[j] = r;
-          c2i[j] = i;
+          br[u][j] = sR[sw(cl[j], k1b + u)];
+          bi[u][j] = sI[sw(cl[j], k1b + u)];
         }
       }
-      broute<true>(c1r, c1i, fr, fi, c2r, c2i);    // [lb0][ka0]
-      twiddle<true>(c1r, c1i, tr, ti);
-      aroute<true>(c2r, c2i, c1r, c1i, fr, fi);    // [lb0][la0]: l0 = cl[j]
+      broute_n<false, NL>(c1r, c1i, fr, fi, br, bi);     // [ka0][lb0]
+      twiddle_n<false, NL>(c1r, c1i, tr, ti);
+      aroute_n<false, NL>(c2r, c2i, c1r, c1i, fr, fi);   // [ka0][kb0]: k0 = cl[j]
 #pragma unroll
-      for (int j = 0; j < 2; ++j) { sR[sw(cl[j], k1)] = c2r[j]; sI[sw(cl[j], k1)] = c2i[j]; }
+      for (int u = 0; u < NL; ++u)
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const double r = c2r[u][j] * s_r[u][j] - c2i[u][j] * s_i[u][j];
+          const double i = c2r[u][j] * s_i[u][j] + c2i[u][j] * s_r[u][j];
+          c2r[u][j] = r;
+          c2i[u][j] = i;
+        }
+      broute_n<true, NL>(c1r, c1i, fr, fi, c2r, c2i);    // [lb0][ka0]
+      twiddle_n<true, NL>(c1r, c1i, tr, ti);
+      aroute_n<true, NL>(c2r, c2i, c1r, c1i, fr, fi);    // [lb0][la0]: l0 = cl[j]
+#pragma unroll
+      for (int u = 0; u < NL; ++u)
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          sR[sw(cl[j], k1b + u)] = c2r[u][j];
+          sI[sw(cl[j], k1b + u)] = c2i[u][j];
+        }
     }
     __syncthreads();
 
     // ---- phase 3: inverse DFT along axis 1 on the S output rows, store the window ----
-    for (int i = warp; i < S; i += NW) {
-      const int l0 = h + i;
-      const int64_t c0 = o0 + l0;
-      if (c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
-      double br[2], bi[2], c1r[2], c1i[2], c2r[2], c2i[2];
+    for (int ib = warp * NL; ib < S; ib += NW * NL) {
+      double br[NL][2], bi[NL][2], c1r[NL][2], c1i[NL][2], c2r[NL][2], c2i[NL][2];
 #pragma unroll
-      for (int j = 0; j < 2; ++j) { br[j] = sR[sw(l0, cl[j])]; bi[j] = sI[sw(l0, cl[j])]; }
-      broute<true>(c1r, c1i, fr, fi, br, bi);      // [lb1][ka1]
-      twiddle<true>(c1r, c1i, tr, ti);
-      broute<true>(c2r, c2i, fr, fi, c1r, c1i);    // [la1][lb1]: l1 = 8g + 2q + j
-      double* drow = a.dst + (c0 - a.win.g0) * a.n1;
+      for (int u = 0; u < NL; ++u) {
+        const int l0 = h + min(ib + u, S - 1);       // a clamped duplicate is computed, not stored
 #pragma unroll
-      for (int j = 0; j < 2; ++j) {
-        const int l1 = 8 * g + 2 * q + j;
-        if (l1 >= h && l1 < h + S) {
-          int64_t c1 = oa1 + l1;
-          if (c1 < a.n1 - h) drow[c1] = c2r[j];
-          c1 = ob1 + l1;
-          if (has_b && c1 < a.n1 - h) drow[c1] = c2i[j];
+        for (int j = 0; j < 2; ++j) {
+          br[u][j] = sR[sw(l0, cl[j])];
+          bi[u][j] = sI[sw(l0, cl[j])];
+        }
+      }
+      broute_n<true, NL>(c1r, c1i, fr, fi, br, bi);      // [lb1][ka1]
+      twiddle_n<true, NL>(c1r, c1i, tr, ti);
+      broute_n<true, NL>(c2r, c2i, fr, fi, c1r, c1i);    // [la1][lb1]: l1 = 8g + 2q + j
+#pragma unroll
+      for (int u = 0; u < NL; ++u) {
+        const int i = ib + u;
+        const int64_t c0 = o0 + h + i;
+        if (i >= S || c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
+        double* drow = a.dst + (c0 - a.win.g0) * a.n1;
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const int l1 = 8 * g + 2 * q + j;
+          if (l1 >= h && l1 < h + S) {
+            int64_t c1 = oa1 + l1;
+            if (c1 < a.n1 - h) drow[c1] = c2r[u][j];
+            c1 = ob1 + l1;
+            if (has_b && c1 < a.n1 - h) drow[c1] = c2i[u][j];
+          }
         }
       }
     }
   }
 }
 
-template <int NW>
+template <int NW, int NL>
 cudaError_t configure_nw(int* max_blocks) {
   const size_t smem = fused2d_ct_smem();
-  cudaError_t e = cudaFuncSetAttribute(fft2d_ct_kernel<NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e =
+      cudaFuncSetAttribute(fft2d_ct_kernel<NW, NL>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_ct_kernel<NW>, NW * 32, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_ct_kernel<NW, NL>, NW * 32, smem);
 }
 
 }  // namespace
 
 size_t fused2d_ct_smem() { return (size_t)2 * PLANE * sizeof(double); }
 
-cudaError_t fused2d_ct_configure(int nw, int* max_blocks) {
-  switch (nw) {
-    case 8: return configure_nw<8>(max_blocks);
-    case 16: return configure_nw<16>(max_blocks);
+// cfg = 10 * NW + NL: 81, 82, 84, 161, 162
+cudaError_t fused2d_ct_configure(int cfg, int* max_blocks) {
+  switch (cfg) {
+    case 81: return configure_nw<8, 1>(max_blocks);
+    case 82: return configure_nw<8, 2>(max_blocks);
+    case 84: return configure_nw<8, 4>(max_blocks);
+    case 161: return configure_nw<16, 1>(max_blocks);
+    case 162: return configure_nw<16, 2>(max_blocks);
     default: return cudaErrorInvalidValue;
   }
 }
 
-cudaError_t launch_fused2d_ct(int nw, const Fft2dArgs& a, int grid, cudaStream_t s) {
-  switch (nw) {
-    case 8: fft2d_ct_kernel<8><<<grid, 8 * 32, fused2d_ct_smem(), s>>>(a); break;
-    case 16: fft2d_ct_kernel<16><<<grid, 16 * 32, fused2d_ct_smem(), s>>>(a); break;
+cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, int grid, cudaStream_t s) {
+  const size_t smem = fused2d_ct_smem();
+  switch (cfg) {
+    case 81: fft2d_ct_kernel<8, 1><<<grid, 256, smem, s>>>(a); break;
+    case 82: fft2d_ct_kernel<8, 2><<<grid, 256, smem, s>>>(a); break;
+    case 84: fft2d_ct_kernel<8, 4><<<grid, 256, smem, s>>>(a); break;
+    case 161: fft2d_ct_kernel<16, 1><<<grid, 512, smem, s>>>(a); break;
+    case 162: fft2d_ct_kernel<16, 2><<<grid, 512, smem, s>>>(a); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();

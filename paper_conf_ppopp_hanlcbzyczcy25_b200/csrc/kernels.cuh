@@ -80,6 +80,7 @@ struct BandArgs {
   int nblocks;
   int oax;               // embedded index of the outer axis (3 - ndim)
   int64_t g0, gn;        // buffers hold global outer-axis rows [g0, g0 + gn)
+  int reference;         // 1: the first (unoptimised) band kernel, for ablation/tests
 };
 
 // Copy a box (embedded coordinates) from src to dst0 and dst1 (either may be null).
@@ -102,10 +103,10 @@ cudaError_t launch_fused2d(int L, int V, const Fft2dArgs& a, int grid, cudaStrea
 
 // Factored-DFT 2D kernel (kernel_fft2d_ct.cu): L = 64 = 8 x 8 Cooley-Tukey per axis.
 // Fre/Fim = [F8 (8x8) | twiddles w64^(ka lb) (8x8)]; Sre/Sim = S_T in [k1][8 g + c] order with
-// k0 = g + 8 c.  nw = warps per CTA (8 or 16).
+// k0 = g + 8 c.  cfg = 10 * (warps per CTA) + (lines per warp step): 81, 82, 84, 161, 162.
 size_t fused2d_ct_smem();
-cudaError_t fused2d_ct_configure(int nw, int* max_blocks_per_sm);
-cudaError_t launch_fused2d_ct(int nw, const Fft2dArgs& a, int grid, cudaStream_t s);
+cudaError_t fused2d_ct_configure(int cfg, int* max_blocks_per_sm);
+cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, int grid, cudaStream_t s);
 
 constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);

@@ -78,6 +78,31 @@ def test_parity_vs_oracle(fs, ext, shape, r, T, steps, kind):
     assert np.array_equal(got[ring], u0[ring])
 
 
+@pytest.mark.parametrize("ext,shape,r,T,steps,kind", [c for c in CASES if len(c[0]) == 2])
+@pytest.mark.parametrize("variant", ["0", "1", "2"])
+def test_parity_dense_kernel(fs, monkeypatch, ext, shape, r, T, steps, kind, variant):
+    """The dense L x L DFT-GEMM kernel (all variants) stays parity-green beside the factored default."""
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "dense")
+    monkeypatch.setenv("FFTSTENCIL_VARIANT", variant)
+    w = wl.stencil_weights(shape, 2, r, kind)
+    u0 = wl.grid(ext, 13)
+    got, p = run_gpu(fs, u0, w, r, T, steps)
+    assert p.info()["algo"] == "dense"
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(got, ref) <= TOL
+
+
+@pytest.mark.parametrize("ext,shape,r,T,steps,kind", CASES[::3])
+def test_band_kernels_agree(fs, monkeypatch, ext, shape, r, T, steps, kind):
+    """The cone-restricted band kernel equals the first (reference) band kernel bitwise."""
+    w = wl.stencil_weights(shape, len(ext), r, kind)
+    u0 = wl.grid(ext, 17)
+    fast, _ = run_gpu(fs, u0, w, r, T, steps)
+    monkeypatch.setenv("FFTSTENCIL_BAND", "reference")
+    ref, _ = run_gpu(fs, u0, w, r, T, steps)
+    assert np.array_equal(fast, ref)
+
+
 @pytest.mark.parametrize("ext,r,T,steps", [((96, 90), 1, 4, 8), ((96, 90), 1, 4, 12), ((500,), 1, 8, 16),
                                            ((500,), 1, 8, 24)])
 def test_in_place_aliasing(fs, ext, r, T, steps):

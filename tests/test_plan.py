@@ -45,8 +45,18 @@ def test_describe_rejects_invalid():
         fs.describe((100, 100), bad, 1)
 
 
+@pytest.fixture
+def dense(monkeypatch):
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "dense")
+
+
+@pytest.fixture
+def factored(monkeypatch):
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "factored")
+
+
 @pytest.mark.parametrize("r,T,L", [(1, 8, 48), (1, 1, 16), (1, 4, 24), (3, 4, 64)])
-def test_describe_2d_geometry(r, T, L):
+def test_describe_2d_geometry(dense, r, T, L):
     info = fs.describe((10240, 10240), wl.seeded_weights("box", 2, r), r, T)
     assert info["T"] == T and info["halo"] == r * T
     assert info["tile"] == [L, L] and info["valid"] == [L - 2 * r * T] * 2
@@ -66,7 +76,7 @@ def test_describe_auto_T_and_clamping():
 
 # ---------------------------------------------------------------- P1: DFT matrices
 @pytest.mark.parametrize("T", [1, 4, 8, 12, 16])
-def test_dft_matrix_vs_numpy(T):
+def test_dft_matrix_vs_numpy(dense, T):
     w = wl.seeded_weights("box", 2, 1)
     info = fs.describe((4000, 4000), w, 1, T)
     L = info["tile"][0]
@@ -85,7 +95,7 @@ def test_pfa_dft_matrices_vs_numpy():
 
 # ---------------------------------------------------------------- P2: powered spectra
 @pytest.mark.parametrize("shape,r,T", [("box", 1, 8), ("star", 3, 4), ("star", 1, 3)])
-def test_spectra_2d_vs_oracle_spectrum(shape, r, T):
+def test_spectra_2d_vs_oracle_spectrum(dense, shape, r, T):
     w = wl.seeded_weights(shape, 2, r)
     info = fs.describe((5000, 5000), w, r, T)
     L = info["tile"][0]
@@ -226,9 +236,73 @@ def _model_2d(u, w, r, T, steps):
 
 @pytest.mark.parametrize("ext,shape,r,T,steps", [((61, 70), "box", 1, 4, 11), ((58, 47), "star", 3, 2, 5),
                                                    ((40, 40), "box", 1, 8, 8)])
-def test_tile_algorithm_model_matches_oracle(ext, shape, r, T, steps):
+def test_tile_algorithm_model_matches_oracle(dense, ext, shape, r, T, steps):
     w = wl.seeded_weights(shape, 2, r)
     u = wl.grid(ext, 99)
     got = _model_2d(u, w, r, T, steps)
     ref = oracle.stencil_run(u, w, r, steps)
     assert np.abs(got - ref).max() <= 1e-12 * np.abs(ref).max()
+
+
+# ---------------------------------------------------------------- factored (CT 64 = 8 x 8) tables
+def test_factored_is_default_for_2d_and_geometry():
+    info = fs.describe((10240, 10240), wl.seeded_weights("star", 2, 1), 1, 0)
+    assert info["algo"] == "factored" and info["tile"] == [64, 64]
+    assert info["valid"][0] == 64 - 2 * info["halo"]
+
+
+def test_factored_dft8_and_twiddles_vs_numpy(factored):
+    w = wl.seeded_weights("box", 2, 1)
+    v = fs.export_aux((1000, 1000), w, 1, 8, which=0, axis=0)
+    F8 = (v[0::2] + 1j * v[1::2]).reshape(8, 8)
+    np.testing.assert_allclose(F8, np.fft.fft(np.eye(8), axis=0), atol=1e-15)
+    v = fs.export_aux((1000, 1000), w, 1, 8, which=0, axis=1)
+    tw = (v[0::2] + 1j * v[1::2]).reshape(8, 8)
+    ref = np.exp(-2j * np.pi * np.outer(np.arange(8), np.arange(8)) / 64)
+    np.testing.assert_allclose(tw, ref, atol=1e-15)
+
+
+@pytest.mark.parametrize("shape,r,T", [("box", 1, 8), ("star", 3, 4), ("box", 2, 5)])
+def test_factored_spectrum_digit_order(factored, shape, r, T):
+    """Kernel order [k1][8 g + c] holds k0 = g + 8 c (the CT output digit order)."""
+    w = wl.seeded_weights(shape, 2, r)
+    info = fs.describe((3000, 3000), w, r, T)
+    for t in (1, info["T"]):
+        v = fs.export_aux((3000, 3000), w, r, T, which=1, t=t)
+        G = (v[0::2] + 1j * v[1::2]).reshape(64, 64)
+        ref = spectrum.powered_spectrum(w, r, (64, 64), t)    # [k0][k1]
+        m = np.arange(64)
+        k0 = (m // 8) + 8 * (m % 8)
+        np.testing.assert_allclose(G, ref[k0, :].T, atol=1e-15)
+
+
+def _ct_axis(x, F8, tw, inverse=False):
+    """The kernel's per-axis factorisation, stage by stage (numpy, last axis)."""
+    sh = x.shape
+    x = x.reshape(-1, 64)
+    out = np.empty_like(x)
+    Fm, T = (np.conj(F8), np.conj(tw)) if inverse else (F8, tw)
+    for n, line in enumerate(x):
+        if not inverse:
+            B = line.reshape(8, 8)               # [la][lb]
+            C = (Fm @ B) * T                     # [ka][lb]
+            C = C @ Fm.T                         # [ka][kb]
+            out[n] = C.T.reshape(-1)             # k = ka + 8 kb
+        else:
+            B = line.reshape(8, 8)               # [kb][ka]  (k = ka + 8 kb)
+            Z = (Fm @ B) * T.T                   # [lb][ka]
+            out[n] = (Fm @ Z.T).reshape(-1)      # [la][lb]: l = 8 la + lb
+    return out.reshape(sh)
+
+
+def test_factored_chain_model_matches_numpy_fft(factored):
+    w = wl.seeded_weights("box", 2, 1)
+    v = fs.export_aux((1000, 1000), w, 1, 8, which=0, axis=0)
+    F8 = (v[0::2] + 1j * v[1::2]).reshape(8, 8)
+    v = fs.export_aux((1000, 1000), w, 1, 8, which=0, axis=1)
+    tw = (v[0::2] + 1j * v[1::2]).reshape(8, 8)
+    rng = np.random.default_rng(5)
+    X = rng.random((64, 64)) + 1j * rng.random((64, 64))
+    np.testing.assert_allclose(_ct_axis(X, F8, tw), np.fft.fft(X, axis=1), atol=1e-12)
+    Y = _ct_axis(np.fft.fft2(X), F8, tw, inverse=True) / 64
+    np.testing.assert_allclose(Y, np.fft.ifft(np.fft.fft2(X), axis=1), atol=1e-12)
