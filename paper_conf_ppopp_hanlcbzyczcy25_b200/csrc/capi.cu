@@ -252,10 +252,15 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.npr = hp.npr;
     a.win = win;
     a.Fre = p->dF;
-    a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
     a.Sre = Sre;
     a.Sim = Sim;
-    e = launch_fused3d(a, (int)std::min<int64_t>(p->fused_grid, np), s);
+    if (hp.algo == 1) {
+      a.Fim = p->dF + 128;
+      e = launch_fused3d_ct(a, (int)std::min<int64_t>(p->fused_grid, np), s);
+    } else {
+      a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
+      e = launch_fused3d(a, (int)std::min<int64_t>(p->fused_grid, np), s);
+    }
   }
   prof_end(p, pe_, s);
   if (e != cudaSuccess) return cuda_fail(e, "fused FFT-tile launch");
@@ -512,6 +517,9 @@ int setup_device(fftstencil_plan* p) {
     }
     e = fused2d_configure(hp.L[0], p->variant, &occ);
     if (e != cudaSuccess) return cuda_fail(e, "fused 2D kernel configuration");
+  } else if (hp.ndim == 3 && hp.algo == 1) {
+    e = fused3d_ct_configure(&occ);
+    if (e != cudaSuccess) return cuda_fail(e, "factored 3D kernel configuration");
   } else if (hp.ndim == 3) {
     e = fused3d_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "fused 3D kernel configuration");
@@ -574,6 +582,16 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
       if (axis < 0 || axis > 1) { set_error("axis must be 0 (F_8) or 1 (twiddles)"); return FFTSTENCIL_EINVAL; }
       L = 8;
       row0 = 8 * axis;
+      ld = 8;
+    } else if (hp.ndim == 3 && hp.algo == 1) {
+      if (axis < 0 || axis > 1) { set_error("axis must be 0 (F_8) or 1 (w16^k)"); return FFTSTENCIL_EINVAL; }
+      if (axis == 1) {
+        for (int k = 0; k < 16; ++k) { v.push_back(hp.Fre[64 + k]); v.push_back(hp.Fim[64 + k]); }
+        L = 0;
+      } else {
+        L = 8;
+      }
+      row0 = 0;
       ld = 8;
     } else {
       if (axis < 0 || axis >= hp.ndim) { set_error("axis out of range"); return FFTSTENCIL_EINVAL; }

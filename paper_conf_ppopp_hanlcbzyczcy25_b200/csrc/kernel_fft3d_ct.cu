@@ -1,0 +1,234 @@
+// Fused 3D FFT-stencil tile kernel with FACTORED DFTs: 16 = 8 x 2 per axis (sm_100a).
+//
+// Same fused pass as kernel_fft3d.cu (Algorithm 1 L252-L258 on 16^3 overlap-save
+// tiles, Double-layer Filling Eq. 9, temporal fusion Eq. 10, Stitching Eq. 7; 3D handled
+// axis by axis as in §3.2.1), but each length-16 axis DFT is factored (§3.2.1's
+// reshaping idea, L208-L218; Cooley-Tukey 16 = 8 x 2):
+//   forward  X[ka + 8 kb] = sum_lb (-1)^(lb kb) w16^(ka lb) sum_la w8^(la ka) x[2 la + lb]
+//   inverse  x[2 la + lb] = sum_ka w8^-(la ka) w16^-(ka lb) sum_kb (-1)^(lb kb) X[ka + 8 kb]
+// The DFT-8 runs on the FP64 tensor cores over a group of 4 lines at once: the B operand is
+// 8 x 8 with k = la and n = 2 m + lb (m = line of the group), so in the C fragment
+// (row g, columns 2q + j) a thread holds both lb of one line -- the twiddle and the DFT-2
+// are thread-local.  Per axis and element: 64 DMMA flops + 8 ALU flops instead of the
+// dense 128 (kernel_fft3d.cu).  F_8 and the twiddles live in registers.
+// Per tile pair, five shared-memory passes (each warp owns 4 lines; a group is read and
+// rewritten in place):
+//   P1 forward axis 2 | P2 forward axis 1 | P3 forward axis 0, * S_T, inverse axis 0 |
+//   P4 inverse axis 1 on the S output planes | P5 inverse axis 2 on the S x S output rows
+//   -> store the S^3 window.
+// Shared layout [l0][l1][l2] at l0*274 + l1*17 + l2: every fragment pattern of the five
+// passes costs at most 4 (mostly 2) wavefronts per 32 doubles; 68.5 KB -> 3 CTAs / SM.
+#include "device_common.cuh"
+#include "kernels.cuh"
+
+namespace fstencil {
+namespace {
+
+using dev::dmma;
+
+constexpr int L = 16;
+constexpr int R = 17;
+constexpr int SL = 274;
+constexpr int PLANE = L * SL;
+constexpr int NWC = 8;
+
+__device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
+}
+
+// Offsets of the 4 lines of a group along one axis: line m, position p.
+struct Lines {
+  int base, mstride, pstride;
+  __device__ __forceinline__ int at(int m, int p) const { return base + m * mstride + p * pstride; }
+};
+
+template <bool CONJ>
+__device__ __forceinline__ void cgemm(double (&cr)[2], double (&ci)[2], const double (&fr)[2], const double (&fi)[2],
+                                      const double (&br)[2], const double (&bi)[2]) {
+  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const double nfi = CONJ ? fi[j] : -fi[j];
+    dmma(cr, fr[j], br[j]);
+    dmma(ci, fr[j], bi[j]);
+    dmma(cr, nfi, bi[j]);
+    dmma(ci, -nfi, br[j]);
+  }
+}
+
+struct Regs {
+  double fr[2], fi[2];     // F8[g][2q + j]
+  double twr, twi;         // w16^g (forward, lb = 1)
+  double itr[2], iti[2];   // conj(w16^(2q + j)) (inverse, lb = 1)
+};
+
+// Forward DFT-16 of the 4 lines; result (natural k order) written back in place, optionally
+// multiplied by the spectrum (sp = S_T at [line q][g][j], k = g + 8 j).
+__device__ __forceinline__ void fwd_group(double* sR, double* sI, const Lines& ln, const Regs& rg, int g, int q,
+                                          const double* spr, const double* spi) {
+  double br[2], bi[2], cr[2], ci[2];
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const int o = ln.at(g >> 1, 4 * q + 2 * j + (g & 1));
+    br[j] = sR[o];
+    bi[j] = sI[o];
+  }
+  cgemm<false>(cr, ci, rg.fr, rg.fi, br, bi);       // C[ka = g][2q + lb]
+  const double tr = cr[1] * rg.twr - ci[1] * rg.twi, ti = cr[1] * rg.twi + ci[1] * rg.twr;
+  double xr[2] = {cr[0] + tr, cr[0] - tr}, xi[2] = {ci[0] + ti, ci[0] - ti};   // k = g, g + 8
+  if (spr) {
+    const double2 s_r = __ldg(reinterpret_cast<const double2*>(spr));
+    const double2 s_i = __ldg(reinterpret_cast<const double2*>(spi));
+    const double a0 = xr[0] * s_r.x - xi[0] * s_i.x, b0 = xr[0] * s_i.x + xi[0] * s_r.x;
+    const double a1 = xr[1] * s_r.y - xi[1] * s_i.y, b1 = xr[1] * s_i.y + xi[1] * s_r.y;
+    xr[0] = a0; xi[0] = b0; xr[1] = a1; xi[1] = b1;
+  }
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const int o = ln.at(q, g + 8 * j);
+    sR[o] = xr[j];
+    sI[o] = xi[j];
+  }
+}
+
+// Inverse DFT-16 (unnormalised; 1/16^3 is in S_T) of the 4 lines; returns the C fragment
+// (line q, positions 2g + j) in cr/ci; writes it back in place if `store`.
+__device__ __forceinline__ void inv_group(double* sR, double* sI, const Lines& ln, const Regs& rg, int g, int q,
+                                          bool store, double (&cr)[2], double (&ci)[2]) {
+  double br[2], bi[2];
+  const int lb = g & 1;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {          // B[ka = 2q + j][n = g]: line g >> 1, lb = g & 1
+    const int o0 = ln.at(g >> 1, 2 * q + j), o1 = ln.at(g >> 1, 2 * q + j + 8);
+    const double ar = sR[o0], ai = sI[o0], xr = sR[o1], xi = sI[o1];
+    double zr = lb ? ar - xr : ar + xr, zi = lb ? ai - xi : ai + xi;
+    if (lb) {
+      const double t = zr * rg.itr[j] - zi * rg.iti[j];
+      zi = zr * rg.iti[j] + zi * rg.itr[j];
+      zr = t;
+    }
+    br[j] = zr;
+    bi[j] = zi;
+  }
+  cgemm<true>(cr, ci, rg.fr, rg.fi, br, bi);         // C[la = g][2q + lb] -> position 2g + j of line q
+  if (store) {
+#pragma unroll
+    for (int j = 0; j < 2; ++j) {
+      const int o = ln.at(q, 2 * g + j);
+      sR[o] = cr[j];
+      sI[o] = ci[j];
+    }
+  }
+}
+
+__global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a) {
+  extern __shared__ __align__(16) double smem[];
+  double* sR = smem;
+  double* sI = smem + PLANE;
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31, g = lane >> 2, q = lane & 3;
+  Regs rg;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    rg.fr[j] = a.Fre[g * 8 + 2 * q + j];
+    rg.fi[j] = a.Fim[g * 8 + 2 * q + j];
+    rg.itr[j] = a.Fre[64 + 2 * q + j];
+    rg.iti[j] = -a.Fim[64 + 2 * q + j];
+  }
+  rg.twr = a.Fre[64 + g];
+  rg.twi = a.Fim[64 + g];
+  const int S = a.S, h = a.h;
+  const int G1 = (S + 3) >> 2;   // line groups of the last inverse pass
+
+  for (int64_t p = a.win.p_begin + blockIdx.x; p < a.win.p_end; p += gridDim.x) {
+    const int64_t line = p / a.npr, pj = p - line * a.npr;
+    const int64_t t0 = line / a.nt1, t1 = line - t0 * a.nt1;
+    const int64_t o0 = t0 * S, o1 = t1 * S, oa2 = 2 * pj * S, ob2 = oa2 + S;
+    const bool has_b = 2 * pj + 1 < a.nt2;
+    __syncthreads();
+    // ---- load the halo'd pair (cp.async, OOB = 0) ----
+    for (int e = tid; e < 2 * L * L * L; e += NWC * 32) {
+      const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
+      const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2, lg0 = g0 - a.win.g0;
+      const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2;
+      cp_async8((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src, valid);
+    }
+    asm volatile("cp.async.commit_group;\n" ::);
+    asm volatile("cp.async.wait_all;\n" ::: "memory");
+    __syncthreads();
+    // ---- P1: forward axis 2 (lines = l1, 4 per group) ----
+    for (int grp = warp; grp < 64; grp += NWC) {
+      const Lines ln{(grp >> 2) * SL + (grp & 3) * 4 * R, R, 1};
+      fwd_group(sR, sI, ln, rg, g, q, nullptr, nullptr);
+    }
+    __syncthreads();
+    // ---- P2: forward axis 1 (lines = l2) ----
+    for (int grp = warp; grp < 64; grp += NWC) {
+      const Lines ln{(grp >> 2) * SL + (grp & 3) * 4, 1, R};
+      fwd_group(sR, sI, ln, rg, g, q, nullptr, nullptr);
+    }
+    __syncthreads();
+    // ---- P3: forward axis 0, * S_T, inverse axis 0 (lines = l2 at fixed k1) ----
+    for (int grp = warp; grp < 64; grp += NWC) {
+      const int k1 = grp >> 2, k2b = (grp & 3) * 4;
+      const Lines ln{k1 * R + k2b, 1, SL};
+      const int64_t si = (((int64_t)k1 * 16 + k2b + q) * 8 + g) * 2;   // S_T at [k1][k2][g][j]
+      fwd_group(sR, sI, ln, rg, g, q, a.Sre + si, a.Sim + si);
+      __syncwarp();
+      double cr[2], ci[2];
+      inv_group(sR, sI, ln, rg, g, q, true, cr, ci);
+    }
+    __syncthreads();
+    // ---- P4: inverse axis 1 on the S output planes (lines = l2) ----
+    for (int grp = warp; grp < 4 * S; grp += NWC) {
+      const Lines ln{(h + (grp >> 2)) * SL + (grp & 3) * 4, 1, R};
+      double cr[2], ci[2];
+      inv_group(sR, sI, ln, rg, g, q, true, cr, ci);
+    }
+    __syncthreads();
+    // ---- P5: inverse axis 2 on the S x S output rows (lines = l1), store the window ----
+    for (int grp = warp; grp < S * G1; grp += NWC) {
+      const int i0 = grp / G1, gi = grp - i0 * G1;
+      const int l0 = h + i0;
+      // the last group of a ragged S shifts back inside the tile (its overlap is recomputed
+      // and stored twice with bitwise-identical values)
+      const int off1 = S >= 4 ? min(4 * gi, S - 4) : 0;
+      const int l1b = h + off1;
+      const Lines ln{l0 * SL + l1b * R, R, 1};
+      double cr[2], ci[2];
+      inv_group(sR, sI, ln, rg, g, q, false, cr, ci);
+      const int64_t c0 = o0 + l0, c1 = o1 + l1b + q;
+      if (off1 + q >= S || c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi || c1 >= a.n1 - h) continue;
+      double* drow = a.dst + ((c0 - a.win.g0) * a.n1 + c1) * a.n2;
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const int l2 = 2 * g + j;
+        if (l2 >= h && l2 < h + S) {
+          int64_t c2 = oa2 + l2;
+          if (c2 < a.n2 - h) drow[c2] = cr[j];
+          c2 = ob2 + l2;
+          if (has_b && c2 < a.n2 - h) drow[c2] = ci[j];
+        }
+      }
+    }
+  }
+}
+
+}  // namespace
+
+size_t fused3d_ct_smem() { return (size_t)2 * PLANE * sizeof(double); }
+
+cudaError_t fused3d_ct_configure(int* max_blocks) {
+  const size_t smem = fused3d_ct_smem();
+  cudaError_t e = cudaFuncSetAttribute(fft3d_ct_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_ct_kernel, NWC * 32, smem);
+}
+
+cudaError_t launch_fused3d_ct(const Fft3dArgs& a, int grid, cudaStream_t s) {
+  fft3d_ct_kernel<<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace fstencil

@@ -116,6 +116,12 @@ size_t fused3d_smem();
 cudaError_t fused3d_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused3d(const Fft3dArgs& a, int grid, cudaStream_t s);
 
+// Factored 3D kernel (kernel_fft3d_ct.cu): 16 = 8 x 2 per axis.  Fre/Fim = [F8 (8x8) | w16^k,
+// k = 0..15]; Sre/Sim = S_T in [k1][k2][k0 % 8][k0 / 8] order.
+size_t fused3d_ct_smem();
+cudaError_t fused3d_ct_configure(int* max_blocks_per_sm);
+cudaError_t launch_fused3d_ct(const Fft3dArgs& a, int grid, cudaStream_t s);
+
 constexpr int kBandThreads = 256;
 cudaError_t band_configure(size_t smem);
 cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s);

@@ -87,6 +87,16 @@ static double eff_2d(int L) {
   }
 }
 
+// Factored 3D tile (kernel_fft3d_ct.cu): line groups of 4 per pair (64 per forward axis,
+// 64 for the inverse axis 0, 4S for inverse axis 1, S ceil(S/4) for inverse axis 2), each
+// 8 DMMA.8x8x4 (4096 flops) + twiddle (32 x 6) + DFT-2 (64 x 2); + S_T (6 per element).
+static double groups_3d_ct(int S) { return 256.0 + 4.0 * S + S * (double)((S + 3) / 4); }
+static double model_flops_3d_ct(int S, int T) {
+  return (4416.0 * groups_3d_ct(S) + 6.0 * 4096.0) / (2.0 * S * (double)S * S * T);
+}
+static constexpr double kEff3d = 0.70;     // dense 3D: executed DMMA efficiency (profiles/r01_sweep.txt)
+static constexpr double kEff3dCt = 0.60;   // factored 3D: assumed until measured
+
 static double model_flops_3d(int L, int S, int T) {
   const double Sp = round8(S), l = L;
   const double f = 24.0 * l * l * l * l + 8.0 * Sp * l * l * l + 8.0 * Sp * Sp * l * l + 8.0 * Sp * Sp * Sp * l;
@@ -192,33 +202,42 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       p.fused_smem = (size_t)2 * 64 * 97 * sizeof(double);
     }
   } else {
+    // candidates: the dense 16^3 tile and the factored one (16 = 8 x 2 per axis)
     const int L = k3DTile;
     const int hmax = std::min(hmax_grid, (L - 2) / 2);
     const int tmax = hmax / radius;
     if (tmax < 1) { err = "radius too large for the 16^3 3D tile"; return FFTSTENCIL_EINVAL; }
-    int bestT = 1;
-    if (T == 0) {
-      double best = 1e300;
-      for (int t = 1; t <= tmax; ++t) {
-        const double f = model_flops_3d(L, L - 2 * radius * t, t);
-        if (f < best) { best = f; bestT = t; }
+    double best = 1e300;
+    int bestT = 1, bA = 0;
+    for (int t = 1; t <= tmax; ++t) {
+      if (T != 0 && t != std::min(T, tmax)) continue;
+      for (int al = 0; al < 2; ++al) {
+        if (algo >= 0 && al != algo) continue;
+        const int S = L - 2 * radius * t;
+        const double f = al ? model_flops_3d_ct(S, t) / kEff3dCt : model_flops_3d(L, S, t) / kEff3d;
+        if (f < best) { best = f; bestT = t; bA = al; }
       }
-    } else {
-      bestT = std::min(T, tmax);
     }
+    p.algo = bA;
     p.T = bestT;
     p.h = radius * bestT;
     for (int a = 0; a < 3; ++a) { p.L[a] = L; p.S[a] = L - 2 * p.h; }
     const double l = L, S = p.S[0];
-    p.flops_per_cell_step =
-        (24.0 * l * l * l * l + 6.0 * l * l * l + 8.0 * l * (S * l * l + S * S * l + S * S * S)) /
-        (2.0 * S * S * S * bestT);
-    const double Sp = round8(p.S[0]);
-    // executed DMMAs per pair (kernel_fft3d.cu): phase 1 16 slices x 128, phase 2 32 row
-    // blocks x (32 + 16 Sp/8), phase 3 S slices x (64 Sp/8 + 16 (Sp/8)^2)
-    const double mt = Sp / 8.0;
-    p.mma_flops_per_pair = 512.0 * (16 * 128 + 32 * (32 + 16 * mt) + S * (64 * mt + 16 * mt * mt));
-    p.fused_smem = (size_t)(2 * 16 * 20 + 2 * 16 * (16 * 20 + 4)) * sizeof(double);
+    if (bA == 0) {
+      p.flops_per_cell_step =
+          (24.0 * l * l * l * l + 6.0 * l * l * l + 8.0 * l * (S * l * l + S * S * l + S * S * S)) /
+          (2.0 * S * S * S * bestT);
+      const double Sp = round8(p.S[0]);
+      // executed DMMAs per pair (kernel_fft3d.cu): phase 1 16 slices x 128, phase 2 32 row
+      // blocks x (32 + 16 Sp/8), phase 3 S slices x (64 Sp/8 + 16 (Sp/8)^2)
+      const double mt = Sp / 8.0;
+      p.mma_flops_per_pair = 512.0 * (16 * 128 + 32 * (32 + 16 * mt) + S * (64 * mt + 16 * mt * mt));
+      p.fused_smem = (size_t)(2 * 16 * 20 + 2 * 16 * (16 * 20 + 4)) * sizeof(double);
+    } else {
+      p.flops_per_cell_step = model_flops_3d_ct(p.S[0], bestT);
+      p.mma_flops_per_pair = 4096.0 * groups_3d_ct(p.S[0]);
+      p.fused_smem = (size_t)2 * 16 * 274 * sizeof(double);
+    }
   }
 
   // ---- overlap-save schedule (Eq. 3 / Eq. 4 / Eq. 7; reading Q4: centred window) ----
@@ -288,6 +307,16 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     p.crt.assign(64, -1);
     const int L = p.N1 * p.N2;
     for (int l = 0; l < L; ++l) p.crt[(l % p.N1) * 8 + (l % p.N2)] = l;   // diagonal / CRT map
+  } else if (ndim == 3 && p.algo == 1) {
+    // [F8 | w16^k, k = 0..15] (kernel_fft3d_ct.cu)
+    p.Fre.assign(128, 0.0);
+    p.Fim.assign(128, 0.0);
+    fill_dft(8, 8, 0, 0, p.Fre, p.Fim);
+    for (int k = 0; k < 16; ++k) {
+      const cplx v = root(k, 16);
+      p.Fre[64 + k] = v.real();
+      p.Fim[64 + k] = v.imag();
+    }
   } else if (ndim == 2 && p.algo == 1) {
     // [F8 | twiddles w64^(ka lb)], 8 x 8 each (kernel_fft2d_ct.cu)
     p.Fre.assign(128, 0.0);
@@ -349,7 +378,11 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         // 2D: natural [k0][k1].  3D: [k1][k2][k0] -- the 3D kernel multiplies in C fragments
         // whose two adjacent columns are consecutive k0 (kernel_fft3d.cu phase 2).
         int64_t dst = i;
-        if (ndim == 3) {
+        if (ndim == 3 && p.algo == 1) {
+          // factored 3D: [k1][k2][k0 % 8][k0 / 8] (the thread-local DFT-2 output pair)
+          const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
+          dst = (k12 * 8 + k0 % 8) * 2 + k0 / 8;
+        } else if (ndim == 3) {
           const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
           dst = k12 * L + k0;
         } else if (p.algo == 1) {

@@ -26,7 +26,7 @@ def geometry(ext, w, r, T, n):
 
 @pytest.mark.parametrize("ext,shape,r,T,n", [((10240, 10240), "box", 1, 8, 8), ((300, 170), "star", 1, 4, 3),
                                              ((513,), "star", 2, 3, 4), ((60, 40, 50), "box", 1, 2, 2),
-                                             ((200, 97), "star", 3, 2, 5), ((40960, 640), "box", 1, 16, 8)])
+                                             ((400, 97), "star", 3, 2, 5), ((40960, 640), "box", 1, 16, 8)])
 def test_slabs_partition_rows_and_pairs(ext, shape, r, T, n):
     w = wl.seeded_weights(shape, len(ext), r)
     gs = geometry(ext, w, r, T, n)
