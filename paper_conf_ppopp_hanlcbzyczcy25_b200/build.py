@@ -44,7 +44,7 @@ CXXFLAGS = ["-O2", "-std=c++17", "-fPIC", "-I", INCLUDE, "-I", CSRC]
 
 CU = ["capi.cu", "kernel_fft2d.cu", "kernel_fft2d_ct.cu", "kernel_fft1d.cu", "kernel_fft3d.cu", "kernel_fft3d_ct.cu", "kernel_band.cu"]
 CPP = ["plan.cpp"]
-HEADERS = ["plan.h", "kernels.cuh", "device_common.cuh"]
+HEADERS = ["plan.h", "kernels.cuh", "device_common.cuh", "tma.cuh"]
 
 
 def _stale(obj: str, src: str) -> bool:

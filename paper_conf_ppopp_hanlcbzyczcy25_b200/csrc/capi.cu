@@ -24,6 +24,7 @@
 #include "fftstencil.h"
 #include "kernels.cuh"
 #include "plan.h"
+#include "tma.cuh"
 
 using namespace fstencil;
 
@@ -64,6 +65,7 @@ struct fftstencil_plan {
   int fused_grid = 0;
   int variant = 0;            // fused-kernel variant (2D dense)
   int ct_cfg = 82;            // factored 2D kernel: 10 * warps per CTA + lines per warp step
+  bool use_tma = true;        // TMA tile loads where the grid allows (FFTSTENCIL_TMA=0 disables)
   int band_reference = 0;     // FFTSTENCIL_BAND=reference selects the first band kernel
   size_t band_smem = 0;
   int64_t last_launches = 0;
@@ -83,6 +85,22 @@ struct fftstencil_plan {
 };
 
 namespace {
+
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return (EncodeTiledFn) nullptr;
+    return (EncodeTiledFn)f;
+  }();
+  return fn;
+}
 
 int cuda_fail(cudaError_t e, const char* what) {
   char buf[256];
@@ -216,7 +234,11 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Fre = p->dF;
     if (hp.algo == 1) {
       a.Fim = p->dF + 128;
-      e = launch_fused2d_ct(p->ct_cfg, a, (int)std::min<int64_t>(p->fused_grid, np), s);
+      CUtensorMap tm;
+      const uint64_t dims[2] = {(uint64_t)hp.ext[1], (uint64_t)(hp.g1 - hp.g0)};
+      const uint32_t box[2] = {64, 64};
+      const bool use_tma = p->use_tma && encode_tensor_map(&tm, src, 2, dims, box);
+      e = launch_fused2d_ct(p->ct_cfg, a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
       e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(p->fused_grid, np), s);
@@ -501,6 +523,7 @@ int setup_device(fftstencil_plan* p) {
   int occ = 0;
   if (hp.ndim == 2 && hp.algo == 1) {
     if (const char* v = std::getenv("FFTSTENCIL_CT_CFG")) p->ct_cfg = std::atoi(v);
+    if (const char* v = std::getenv("FFTSTENCIL_TMA")) p->use_tma = std::atoi(v) != 0;
     e = fused2d_ct_configure(p->ct_cfg, &occ);
     if (e == cudaErrorInvalidValue) {
       set_error("FFTSTENCIL_CT_CFG must be one of 81, 82, 84, 161, 162");
@@ -542,6 +565,28 @@ int setup_device(fftstencil_plan* p) {
 }
 
 }  // namespace
+
+namespace fstencil {
+bool encode_tensor_map(CUtensorMap* map, const void* base, int rank, const uint64_t* dims, const uint32_t* box) {
+  EncodeTiledFn fn = encode_fn();
+  if (!fn || rank < 1 || rank > 3 || (reinterpret_cast<uintptr_t>(base) & 15)) return false;
+  cuuint64_t gdim[3], gstride[2];
+  cuuint32_t bdim[3], es[3] = {1, 1, 1};
+  uint64_t stride = sizeof(double);
+  for (int i = 0; i < rank; ++i) {
+    gdim[i] = dims[i];
+    bdim[i] = box[i];
+    if (i > 0) {
+      gstride[i - 1] = stride;
+      if (stride % 16) return false;
+    }
+    stride *= dims[i];
+  }
+  return fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)rank, const_cast<void*>(base), gdim, gstride, bdim, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+}  // namespace fstencil
 
 extern "C" {
 

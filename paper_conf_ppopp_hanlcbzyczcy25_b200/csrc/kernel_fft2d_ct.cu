@@ -26,6 +26,7 @@
 // (c = 16q + 8j + g) and the column pattern (r = 16q + 8j + g) hit every bank pair twice.
 #include "device_common.cuh"
 #include "kernels.cuh"
+#include "tma.cuh"
 
 namespace fstencil {
 namespace {
@@ -143,13 +144,19 @@ __device__ __forceinline__ void twiddle_n(double (&cr)[NL][2], double (&ci)[NL][
   for (int u = 0; u < NL; ++u) twiddle<CONJ>(cr[u], ci[u], tr, ti);
 }
 
-template <int NW, int NL>
-__global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a) {
-  extern __shared__ __align__(16) double smem[];
+// TMA = true: each tile arrives by one 64 x 64 TMA box (OOB -> 0) in a dense staging
+// layout; phase 1 reads it (4-way bank conflicts on that pass only), keeps its results in
+// registers across a CTA barrier and writes Q into the padded layout over the same memory.
+template <int NW, int NL, bool TMA>
+__global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a, const __grid_constant__ CUtensorMap tm) {
+  extern __shared__ __align__(128) double smem[];
   double* sR = smem;            // plane 0: tile 2j (Re), then Q/W real parts
   double* sI = smem + PLANE;    // plane 1: tile 2j+1 (Im), then Q/W imaginary parts
+  __shared__ __align__(8) uint64_t bar;
   const int tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31, g = lane >> 2, q = lane & 3;
+  if (TMA && tid == 0) tma::mbar_init(&bar, 1);
+  uint32_t parity = 0;
 
   // register-resident F8 fragments (row g, logical column 2q+j) and twiddles w64^(g (2q+j))
   double fr[2], fi[2], tr[2], ti[2];
@@ -170,7 +177,52 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a) {
     const int64_t t0 = p / a.npr, pj = p - t0 * a.npr;
     const int64_t o0 = t0 * S, oa1 = 2 * pj * S, ob1 = oa1 + S;
     const bool has_b = 2 * pj + 1 < a.nt1;
+    if (TMA) tma::fence_proxy_async();
     __syncthreads();   // previous pair's phase 3 reads are done
+    if (TMA) {
+      // ---- load the halo'd pair: two 64 x 64 TMA boxes (OOB rows/columns -> 0) ----
+      if (tid == 0) {
+        tma::mbar_expect_tx(&bar, (has_b ? 2u : 1u) * L * L * 8u);
+        const int y = (int)(o0 - a.win.g0);
+        tma::load_2d(sR, &tm, (int)oa1, y, &bar);
+        if (has_b) tma::load_2d(sI, &tm, (int)ob1, y, &bar);
+      }
+      if (!has_b)
+        for (int e = tid; e < L * L; e += NW * 32) sI[e] = 0.0;
+      tma::mbar_wait(&bar, parity);
+      parity ^= 1;
+      __syncthreads();
+      // ---- phase 1 from the dense staging layout; results held until the barrier ----
+      constexpr int ITER = L / (NW * NL);
+      double qr[ITER][NL][2], qi[ITER][NL][2];
+#pragma unroll
+      for (int it = 0; it < ITER; ++it) {
+        const int l0b = warp * NL + it * NW * NL;
+        double br[NL][2], bi[NL][2], c1r[NL][2], c1i[NL][2];
+#pragma unroll
+        for (int u = 0; u < NL; ++u)
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            br[u][j] = sR[(l0b + u) * L + cl[j]];
+            bi[u][j] = sI[(l0b + u) * L + cl[j]];
+          }
+        broute_n<false, NL>(c1r, c1i, fr, fi, br, bi);
+        twiddle_n<false, NL>(c1r, c1i, tr, ti);
+        aroute_n<false, NL>(qr[it], qi[it], c1r, c1i, fr, fi);
+      }
+      __syncthreads();
+#pragma unroll
+      for (int it = 0; it < ITER; ++it) {
+        const int l0b = warp * NL + it * NW * NL;
+#pragma unroll
+        for (int u = 0; u < NL; ++u)
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            sR[sw(l0b + u, cl[j])] = qr[it][u][j];
+            sI[sw(l0b + u, cl[j])] = qi[it][u][j];
+          }
+      }
+    } else {
     // ---- load the halo'd pair (cp.async, OOB = 0) ----
     for (int e = tid; e < 2 * L * L; e += NW * 32) {
       const int t = e >> 12, r = (e >> 6) & 63, c = e & 63;
@@ -203,6 +255,7 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a) {
           sI[sw(l0b + u, cl[j])] = c2i[u][j];
         }
     }
+    }   // !TMA
     __syncthreads();
 
     // ---- phase 2: axis 0 forward, * S_T, axis 0 inverse, every column ----
@@ -281,40 +334,54 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a) {
   }
 }
 
-template <int NW, int NL>
+template <int NW, int NL, bool TMA>
 cudaError_t configure_nw(int* max_blocks) {
   const size_t smem = fused2d_ct_smem();
   cudaError_t e =
-      cudaFuncSetAttribute(fft2d_ct_kernel<NW, NL>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      cudaFuncSetAttribute(fft2d_ct_kernel<NW, NL, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_ct_kernel<NW, NL>, NW * 32, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_ct_kernel<NW, NL, TMA>, NW * 32, smem);
 }
 
 }  // namespace
 
 size_t fused2d_ct_smem() { return (size_t)2 * PLANE * sizeof(double); }
 
-// cfg = 10 * NW + NL: 81, 82, 84, 161, 162
+// cfg = 10 * NW + NL: 81, 82, 84, 161, 162 (the TMA instantiation exists for 82 and 84)
 cudaError_t fused2d_ct_configure(int cfg, int* max_blocks) {
   switch (cfg) {
-    case 81: return configure_nw<8, 1>(max_blocks);
-    case 82: return configure_nw<8, 2>(max_blocks);
-    case 84: return configure_nw<8, 4>(max_blocks);
-    case 161: return configure_nw<16, 1>(max_blocks);
-    case 162: return configure_nw<16, 2>(max_blocks);
+    case 81: return configure_nw<8, 1, false>(max_blocks);
+    case 82: {
+      cudaError_t e = configure_nw<8, 2, true>(max_blocks);
+      return e != cudaSuccess ? e : configure_nw<8, 2, false>(max_blocks);
+    }
+    case 84: {
+      cudaError_t e = configure_nw<8, 4, true>(max_blocks);
+      return e != cudaSuccess ? e : configure_nw<8, 4, false>(max_blocks);
+    }
+    case 161: return configure_nw<16, 1, false>(max_blocks);
+    case 162: return configure_nw<16, 2, false>(max_blocks);
     default: return cudaErrorInvalidValue;
   }
 }
 
-cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, int grid, cudaStream_t s) {
+cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s) {
   const size_t smem = fused2d_ct_smem();
-  switch (cfg) {
-    case 81: fft2d_ct_kernel<8, 1><<<grid, 256, smem, s>>>(a); break;
-    case 82: fft2d_ct_kernel<8, 2><<<grid, 256, smem, s>>>(a); break;
-    case 84: fft2d_ct_kernel<8, 4><<<grid, 256, smem, s>>>(a); break;
-    case 161: fft2d_ct_kernel<16, 1><<<grid, 512, smem, s>>>(a); break;
-    case 162: fft2d_ct_kernel<16, 2><<<grid, 512, smem, s>>>(a); break;
-    default: return cudaErrorInvalidValue;
+  static const CUtensorMap none = {};
+  const CUtensorMap& m = tm ? *tm : none;
+  if (tm && cfg == 82) {
+    fft2d_ct_kernel<8, 2, true><<<grid, 256, smem, s>>>(a, m);
+  } else if (tm && cfg == 84) {
+    fft2d_ct_kernel<8, 4, true><<<grid, 256, smem, s>>>(a, m);
+  } else {
+    switch (cfg) {
+      case 81: fft2d_ct_kernel<8, 1, false><<<grid, 256, smem, s>>>(a, m); break;
+      case 82: fft2d_ct_kernel<8, 2, false><<<grid, 256, smem, s>>>(a, m); break;
+      case 84: fft2d_ct_kernel<8, 4, false><<<grid, 256, smem, s>>>(a, m); break;
+      case 161: fft2d_ct_kernel<16, 1, false><<<grid, 512, smem, s>>>(a, m); break;
+      case 162: fft2d_ct_kernel<16, 2, false><<<grid, 512, smem, s>>>(a, m); break;
+      default: return cudaErrorInvalidValue;
+    }
   }
   return cudaGetLastError();
 }

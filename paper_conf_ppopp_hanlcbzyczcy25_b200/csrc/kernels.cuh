@@ -1,6 +1,7 @@
 // Kernel argument blocks and launchers of the fused FFT-stencil path (sm_100a).
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -106,7 +107,8 @@ cudaError_t launch_fused2d(int L, int V, const Fft2dArgs& a, int grid, cudaStrea
 // k0 = g + 8 c.  cfg = 10 * (warps per CTA) + (lines per warp step): 81, 82, 84, 161, 162.
 size_t fused2d_ct_smem();
 cudaError_t fused2d_ct_configure(int cfg, int* max_blocks_per_sm);
-cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, int grid, cudaStream_t s);
+// tm: tensor map of the source buffer (dims {n1, gn}, box {64, 64}) or null (cp.async path).
+cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
 
 constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);
