@@ -278,7 +278,8 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Sim = Sim;
     if (hp.algo == 1) {
       a.Fim = p->dF + 128;
-      e = launch_fused3d_ct(a, (int)std::min<int64_t>(p->fused_grid, np), s);
+      const bool v16 = p->use_tma && hp.ext[2] % 2 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0;
+      e = launch_fused3d_ct(a, v16, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
       e = launch_fused3d(a, (int)std::min<int64_t>(p->fused_grid, np), s);
@@ -541,6 +542,7 @@ int setup_device(fftstencil_plan* p) {
     e = fused2d_configure(hp.L[0], p->variant, &occ);
     if (e != cudaSuccess) return cuda_fail(e, "fused 2D kernel configuration");
   } else if (hp.ndim == 3 && hp.algo == 1) {
+    if (const char* v = std::getenv("FFTSTENCIL_TMA")) p->use_tma = std::atoi(v) != 0;
     e = fused3d_ct_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "factored 3D kernel configuration");
   } else if (hp.ndim == 3) {

@@ -16,8 +16,10 @@
 //   P1 forward axis 2 | P2 forward axis 1 | P3 forward axis 0, * S_T, inverse axis 0 |
 //   P4 inverse axis 1 on the S output planes | P5 inverse axis 2 on the S x S output rows
 //   -> store the S^3 window.
-// Shared layout [l0][l1][l2] at l0*274 + l1*17 + l2: every fragment pattern of the five
-// passes costs at most 4 (mostly 2) wavefronts per 32 doubles; 68.5 KB -> 3 CTAs / SM.
+// Shared layout [l0][l1][l2] at l0*290 + l1*18 + l2: every fragment pattern of the five
+// passes costs at most 4 (mostly 2) wavefronts per 32 doubles; 72.5 KB -> 3 CTAs / SM.
+// (R even keeps every tile row 16-byte aligned for 16-byte cp.async; TMA tensor copies
+// would need 128-byte-aligned destinations, which this conflict-free padding excludes.)
 #include "device_common.cuh"
 #include "kernels.cuh"
 
@@ -27,14 +29,18 @@ namespace {
 using dev::dmma;
 
 constexpr int L = 16;
-constexpr int R = 17;
-constexpr int SL = 274;
+constexpr int R = 18;               // 16-byte aligned rows (TMA destinations)
+constexpr int SL = 290;
 constexpr int PLANE = L * SL;
 constexpr int NWC = 8;
 
 __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
+}
+__device__ __forceinline__ void cp_async16(double* dst, const double* src, bool valid) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 16 : 0));
 }
 
 // Offsets of the 4 lines of a group along one axis: line m, position p.
@@ -122,6 +128,8 @@ __device__ __forceinline__ void inv_group(double* sR, double* sI, const Lines& l
   }
 }
 
+// V16: n2 even -> every tile row starts 16-byte aligned in HBM and in shared memory.
+template <bool V16>
 __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a) {
   extern __shared__ __align__(16) double smem[];
   double* sR = smem;
@@ -147,12 +155,24 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
     const int64_t o0 = t0 * S, o1 = t1 * S, oa2 = 2 * pj * S, ob2 = oa2 + S;
     const bool has_b = 2 * pj + 1 < a.nt2;
     __syncthreads();
-    // ---- load the halo'd pair (cp.async, OOB = 0) ----
-    for (int e = tid; e < 2 * L * L * L; e += NWC * 32) {
-      const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
-      const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2, lg0 = g0 - a.win.g0;
-      const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2;
-      cp_async8((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src, valid);
+    if (V16) {
+      // ---- load the halo'd pair: 16-byte cp.async (rows are even-length and 16 B aligned) ----
+      for (int e = tid; e < 2 * L * L * 8; e += NWC * 32) {
+        const int t = e >> 11, l0 = (e >> 7) & 15, l1 = (e >> 3) & 15, l2 = (e & 7) * 2;
+        const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2, lg0 = g0 - a.win.g0;
+        const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2;
+        cp_async16((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src,
+                   valid);
+      }
+    } else {
+      // ---- load the halo'd pair (8-byte cp.async, OOB = 0) ----
+      for (int e = tid; e < 2 * L * L * L; e += NWC * 32) {
+        const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
+        const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2, lg0 = g0 - a.win.g0;
+        const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2;
+        cp_async8((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src,
+                  valid);
+      }
     }
     asm volatile("cp.async.commit_group;\n" ::);
     asm volatile("cp.async.wait_all;\n" ::: "memory");
@@ -221,13 +241,18 @@ size_t fused3d_ct_smem() { return (size_t)2 * PLANE * sizeof(double); }
 
 cudaError_t fused3d_ct_configure(int* max_blocks) {
   const size_t smem = fused3d_ct_smem();
-  cudaError_t e = cudaFuncSetAttribute(fft3d_ct_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(fft3d_ct_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft3d_ct_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_ct_kernel, NWC * 32, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_ct_kernel<true>, NWC * 32, smem);
 }
 
-cudaError_t launch_fused3d_ct(const Fft3dArgs& a, int grid, cudaStream_t s) {
-  fft3d_ct_kernel<<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a);
+cudaError_t launch_fused3d_ct(const Fft3dArgs& a, bool v16, int grid, cudaStream_t s) {
+  if (v16)
+    fft3d_ct_kernel<true><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a);
+  else
+    fft3d_ct_kernel<false><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a);
   return cudaGetLastError();
 }
 

@@ -122,7 +122,8 @@ cudaError_t launch_fused3d(const Fft3dArgs& a, int grid, cudaStream_t s);
 // k = 0..15]; Sre/Sim = S_T in [k1][k2][k0 % 8][k0 / 8] order.
 size_t fused3d_ct_smem();
 cudaError_t fused3d_ct_configure(int* max_blocks_per_sm);
-cudaError_t launch_fused3d_ct(const Fft3dArgs& a, int grid, cudaStream_t s);
+// v16: 16-byte cp.async tile loads (n2 even and src 16-byte aligned), else 8-byte.
+cudaError_t launch_fused3d_ct(const Fft3dArgs& a, bool v16, int grid, cudaStream_t s);
 
 constexpr int kBandThreads = 256;
 cudaError_t band_configure(size_t smem);
