@@ -196,10 +196,25 @@ __global__ void box_copy_kernel(const BoxCopyArgs a) {
 
 }  // namespace
 
+// The max-dynamic-shared-memory attribute belongs to the function, not to a plan: set it to
+// the device limit once (minus each kernel's static shared memory) so plans of different
+// band sizes coexist, and refuse a plan whose band region does not fit.
 cudaError_t band_configure(size_t smem) {
-  cudaError_t e = cudaFuncSetAttribute(band_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  int dev = 0, optin = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(band_cone_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncAttributes fa;
+  if ((e = cudaFuncGetAttributes(&fa, band_kernel)) != cudaSuccess) return e;
+  const size_t lim0 = (size_t)optin - fa.sharedSizeBytes;
+  if ((e = cudaFuncSetAttribute(band_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim0)) != cudaSuccess)
+    return e;
+  if ((e = cudaFuncGetAttributes(&fa, band_cone_kernel)) != cudaSuccess) return e;
+  const size_t lim1 = (size_t)optin - fa.sharedSizeBytes;
+  if ((e = cudaFuncSetAttribute(band_cone_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
+      cudaSuccess)
+    return e;
+  return smem <= lim0 && smem <= lim1 ? cudaSuccess : cudaErrorInvalidValue;
 }
 
 cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s) {

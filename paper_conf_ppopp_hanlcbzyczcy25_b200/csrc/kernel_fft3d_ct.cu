@@ -90,6 +90,7 @@ __device__ __forceinline__ void fwd_group(double* sR, double* sI, const Lines& l
     const double a1 = xr[1] * s_r.y - xi[1] * s_i.y, b1 = xr[1] * s_i.y + xi[1] * s_r.y;
     xr[0] = a0; xi[0] = b0; xr[1] = a1; xi[1] = b1;
   }
+  __syncwarp();   // the group is rewritten in place with another thread-to-word map
 #pragma unroll
   for (int j = 0; j < 2; ++j) {
     const int o = ln.at(q, g + 8 * j);
@@ -119,6 +120,7 @@ __device__ __forceinline__ void inv_group(double* sR, double* sI, const Lines& l
   }
   cgemm<true>(cr, ci, rg.fr, rg.fi, br, bi);         // C[la = g][2q + lb] -> position 2g + j of line q
   if (store) {
+    __syncwarp();
 #pragma unroll
     for (int j = 0; j < 2; ++j) {
       const int o = ln.at(q, 2 * g + j);

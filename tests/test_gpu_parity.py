@@ -195,6 +195,22 @@ def test_3d_T_invariance_and_constant(fs):
     np.testing.assert_allclose(got, c, rtol=1e-12)
 
 
+def test_plans_with_different_band_sizes_coexist(fs):
+    """Regression (compute-sanitizer memcheck): the band kernel's shared-memory attribute is
+    per function; a later plan with a smaller band must not break an earlier one."""
+    w1 = wl.seeded_weights("box", 2, 3)
+    big = fs.Plan((300, 260), w1, 3, 4)
+    small = fs.Plan((120, 100), wl.seeded_weights("box", 2, 1), 1, 1)
+    u = wl.grid((300, 260), 9)
+    a = torch.from_numpy(u).cuda()
+    b = torch.empty_like(a)
+    big.run(a, b, 9)
+    torch.cuda.synchronize()
+    ref = oracle.stencil_run(u, w1, 3, 9)
+    assert rel_err(b.cpu().numpy(), ref) <= TOL
+    del small
+
+
 def test_invalid_arguments(fs):
     w = wl.seeded_weights("box", 2, 1)
     with pytest.raises(fs.FftStencilError):
