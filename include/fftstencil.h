@@ -85,13 +85,24 @@ typedef struct {
   int64_t pair_begin, pair_end; /* tile pairs this rank computes                         */
   int64_t interior_begin, interior_end; /* pairs needing no halo rows (overlap the exchange) */
   int64_t ghost_lo, ghost_hi;   /* halo rows received from rank-1 / rank+1 per pass     */
-  int algo;                     /* 2D tile algorithm: 0 dense L x L DFT GEMMs, 1 factored
-                                   64 = 8 x 8 (Cooley-Tukey, DFT-8 GEMMs + twiddles)       */
+  int algo;                     /* 2D/3D tile algorithm: 0 dense L^d DFT GEMMs, 1 factored
+                                   (2D 64 = 8 x 8, 3D 16 = 8 x 2 Cooley-Tukey)              */
+  int periodic;                 /* 1 for a FFTSTENCIL_PERIODIC plan                      */
 } fftstencil_info;
+
+/* Plan creation flags (fftstencil_plan_create_ex / fftstencil_describe_ex). */
+enum {
+  FFTSTENCIL_PERIODIC = 1   /* periodic boundary instead of the fixed ring: every cell is updated,
+                               neighbours wrap modulo the extents; single GPU */
+};
 
 /* Build a plan (host precompute + device upload).  Returns NULL on error. */
 fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const double* weights,
                                         int radius, int T);
+
+/* As fftstencil_plan_create with creation `flags` (FFTSTENCIL_PERIODIC or 0). */
+fftstencil_plan* fftstencil_plan_create_ex(int ndim, const int64_t* extents, const double* weights,
+                                           int radius, int T, int flags);
 
 /* Enqueue `total_steps` (>= 0) time steps on `stream` (a cudaStream_t; NULL = the
  * legacy default stream).  `in` and `out` are device pointers to prod(extents) FP64
@@ -100,6 +111,13 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
  * synchronisation.  Returns FFTSTENCIL_OK or a negative code. */
 int fftstencil_run(fftstencil_plan* plan, const double* in, double* out, int64_t total_steps,
                    void* stream);
+
+/* Flexible outputs (§4: results at chosen time steps): outs[k] receives
+ * the state after emit_steps[k] steps (non-decreasing, >= 0), k = 0..n_emit-1; each segment
+ * is fused independently (remainder pass per segment).  Device buffers; outs must not alias
+ * each other; `in` may alias outs[0].  Asynchronous on `stream`. */
+int fftstencil_run_emit(fftstencil_plan* plan, const double* in, const int64_t* emit_steps, int n_emit,
+                        double* const* outs, void* stream);
 
 /* End-to-end variant with HOST buffers: copies h_in (prod(extents) FP64, pageable or
  * pinned) to device, runs, copies the result to h_out, and synchronises `stream`
@@ -160,6 +178,10 @@ const char* fftstencil_last_error(void);
  * Run the plan builder alone and report the geometry it would choose. */
 int fftstencil_describe(int ndim, const int64_t* extents, const double* weights, int radius,
                         int T, fftstencil_info* info);
+
+/* As fftstencil_describe with creation `flags`. */
+int fftstencil_describe_ex(int ndim, const int64_t* extents, const double* weights, int radius, int T,
+                           int flags, fftstencil_info* info);
 
 /* Export the host plan's auxiliary tables, for tests of the plan builder:
  *   which = 0: forward DFT matrix of axis `axis` (1D: axis 0 -> F_N1, axis 1 -> F_N2;

@@ -37,12 +37,12 @@ def _dp(a):
     return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
 
 
-def describe(extents, weights, radius: int, T: int = 0) -> dict:
+def describe(extents, weights, radius: int, T: int = 0, periodic: bool = False) -> dict:
     """Run the host plan builder only (no GPU needed) and return its geometry."""
     ext, w = _arrays(extents, weights, radius)
     info = Info()
-    rc = _native.lib().fftstencil_describe(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
-                                           ctypes.byref(info))
+    rc = _native.lib().fftstencil_describe_ex(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
+                                              _native.PERIODIC if periodic else 0, ctypes.byref(info))
     if rc != 0:
         raise FftStencilError(rc, last_error())
     return info.as_dict()
@@ -105,7 +105,7 @@ class Plan:
     """A FlashFFTStencil plan bound to the current CUDA device."""
 
     def __init__(self, extents, weights, radius: int, T: int = 0, nranks: int = 1, rank: int = 0,
-                 nccl_id: bytes | None = None, loopback: bool = False):
+                 nccl_id: bytes | None = None, loopback: bool = False, periodic: bool = False):
         """extents are GLOBAL.  nranks > 1: this process's rank of the outer-axis decomposition;
         pass the group's nccl_id (bytes from nccl_unique_id()), or loopback=True for a rank
         run with run_group on one device.  in/out tensors then hold this rank's slab
@@ -115,7 +115,8 @@ class Plan:
         self.radius = int(radius)
         self._lib = _native.lib()
         if nranks == 1:
-            h = self._lib.fftstencil_plan_create(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T))
+            h = self._lib.fftstencil_plan_create_ex(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
+                                                    _native.PERIODIC if periodic else 0)
         else:
             if nccl_id is None and not loopback:
                 raise ValueError("nranks > 1 needs nccl_id (or loopback=True)")
@@ -184,6 +185,23 @@ class Plan:
         s = stream if stream is not None else torch.cuda.current_stream(inp.device)
         rc = self._lib.fftstencil_run(self._h, ctypes.c_void_p(inp.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                       int(total_steps), ctypes.c_void_p(s.cuda_stream))
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+
+    def run_emit(self, inp, outs, emit_steps, stream=None) -> None:
+        """outs[k] <- the state after emit_steps[k] time steps (flexible outputs, §4)."""
+        import torch
+        self._check_dev(inp, "inp")
+        for o in outs:
+            self._check_dev(o, "out")
+        n = len(outs)
+        steps = np.ascontiguousarray(np.asarray(emit_steps, dtype=np.int64))
+        if steps.size != n:
+            raise ValueError("one emit step per output")
+        O = (ctypes.c_void_p * n)(*[o.data_ptr() for o in outs])
+        s = stream if stream is not None else torch.cuda.current_stream(inp.device)
+        rc = self._lib.fftstencil_run_emit(self._h, ctypes.c_void_p(inp.data_ptr()), _i64p(steps), n, O,
+                                           ctypes.c_void_p(s.cuda_stream))
         if rc != 0:
             raise FftStencilError(rc, last_error())
 

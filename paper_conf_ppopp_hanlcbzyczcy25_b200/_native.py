@@ -12,6 +12,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 SO_PATH = os.path.join(HERE, "libfftstencil.so")
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = 0, -1, -2, -3, -4, -5
+PERIODIC = 1
 CODES = {OK: "OK", EINVAL: "EINVAL", ENOMEM: "ENOMEM", ECUDA: "ECUDA", ENCCL: "ENCCL",
          EUNSUPPORTED: "EUNSUPPORTED"}
 
@@ -19,7 +20,8 @@ CODES = {OK: "OK", EINVAL: "EINVAL", ENOMEM: "ENOMEM", ECUDA: "ECUDA", ENCCL: "E
 EXPORTS = ("fftstencil_plan_create", "fftstencil_run", "fftstencil_run_host", "fftstencil_destroy",
            "fftstencil_plan_info", "fftstencil_last_error", "fftstencil_describe", "fftstencil_export_aux",
            "fftstencil_set_profiling", "fftstencil_profile_read", "fftstencil_plan_create_dist",
-           "fftstencil_nccl_unique_id", "fftstencil_run_group", "fftstencil_describe_dist")
+           "fftstencil_nccl_unique_id", "fftstencil_run_group", "fftstencil_describe_dist",
+           "fftstencil_plan_create_ex", "fftstencil_describe_ex", "fftstencil_run_emit")
 
 
 class Info(ctypes.Structure):
@@ -52,6 +54,7 @@ class Info(ctypes.Structure):
         ("ghost_lo", ctypes.c_int64),
         ("ghost_hi", ctypes.c_int64),
         ("algo", ctypes.c_int),
+        ("periodic", ctypes.c_int),
     ]
 
     def as_dict(self) -> dict:
@@ -68,6 +71,7 @@ class Info(ctypes.Structure):
             "pair_begin": self.pair_begin, "pair_end": self.pair_end, "interior_begin": self.interior_begin,
             "interior_end": self.interior_end, "ghost_lo": self.ghost_lo, "ghost_hi": self.ghost_hi,
             "algo": ("dense", "factored")[self.algo] if nd >= 2 else "pfa",
+            "periodic": bool(self.periodic),
         }
 
 
@@ -118,6 +122,13 @@ def lib():
     L.fftstencil_describe_dist.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                            ctypes.c_int, ctypes.POINTER(Info)]
     L.fftstencil_describe_dist.restype = ctypes.c_int
+    L.fftstencil_plan_create_ex.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int]
+    L.fftstencil_plan_create_ex.restype = vp
+    L.fftstencil_describe_ex.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                         ctypes.POINTER(Info)]
+    L.fftstencil_describe_ex.restype = ctypes.c_int
+    L.fftstencil_run_emit.argtypes = [vp, vp, i64p, ctypes.c_int, ctypes.POINTER(vp), vp]
+    L.fftstencil_run_emit.restype = ctypes.c_int
     _lib = L
     return L
 

@@ -176,6 +176,7 @@ void fill_info(const HostPlan& hp, fftstencil_info* info) {
   info->ghost_lo = hp.row_lo - hp.g0;
   info->ghost_hi = hp.g1 - hp.row_hi;
   info->algo = hp.algo;
+  info->periodic = hp.periodic;
 }
 
 // Profiling: a (start, end) event pair around one launch; returns the pair index or -1.
@@ -216,6 +217,15 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
   win.p_begin = pb;
   win.p_end = pe;
   const int64_t np = pe - pb;
+  Bound bd;
+  bd.wrap = hp.periodic;
+  bd.shift = hp.periodic ? -hp.h : 0;
+  const int64_t lim[3] = {hp.periodic ? hp.ext[0] : hp.ext[0] - hp.h,
+                          hp.ndim > 1 ? (hp.periodic ? hp.ext[1] : hp.ext[1] - hp.h) : 0,
+                          hp.ndim > 2 ? (hp.periodic ? hp.ext[2] : hp.ext[2] - hp.h) : 0};
+  bd.lim0 = lim[0];
+  bd.lim1 = lim[1];
+  bd.lim2 = lim[2];
   cudaError_t e = cudaSuccess;
   const long pe_ = prof_begin(p, 0, s);
   if (hp.ndim == 2) {
@@ -229,6 +239,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.nt1 = hp.nt[1];
     a.npr = hp.npr;
     a.win = win;
+    a.bd = bd;
     a.Sre = Sre;
     a.Sim = Sim;
     a.Fre = p->dF;
@@ -237,7 +248,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
       CUtensorMap tm;
       const uint64_t dims[2] = {(uint64_t)hp.ext[1], (uint64_t)(hp.g1 - hp.g0)};
       const uint32_t box[2] = {64, 64};
-      const bool use_tma = p->use_tma && encode_tensor_map(&tm, src, 2, dims, box);
+      const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 2, dims, box);
       e = launch_fused2d_ct(p->ct_cfg, a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
@@ -253,6 +264,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.L = hp.L[0];
     a.ntiles = hp.tiles;
     a.win = win;
+    a.bd = bd;
     a.Fre = p->dF;
     a.Fim = p->dF + 128;
     a.Sre = Sre;
@@ -273,12 +285,13 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.nt2 = hp.nt[2];
     a.npr = hp.npr;
     a.win = win;
+    a.bd = bd;
     a.Fre = p->dF;
     a.Sre = Sre;
     a.Sim = Sim;
     if (hp.algo == 1) {
       a.Fim = p->dF + 128;
-      const bool v16 = p->use_tma && hp.ext[2] % 2 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0;
+      const bool v16 = p->use_tma && !hp.periodic && hp.ext[2] % 2 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0;
       e = launch_fused3d_ct(a, v16, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
@@ -599,6 +612,20 @@ int fftstencil_describe(int ndim, const int64_t* extents, const double* weights,
   return fftstencil_describe_dist(ndim, extents, weights, radius, T, 1, 0, info);
 }
 
+int fftstencil_describe_ex(int ndim, const int64_t* extents, const double* weights, int radius, int T, int flags,
+                           fftstencil_info* info) {
+  if (!info) { set_error("info must be non-NULL"); return FFTSTENCIL_EINVAL; }
+  if (flags & ~FFTSTENCIL_PERIODIC) { set_error("unknown flags"); return FFTSTENCIL_EINVAL; }
+  HostPlan hp;
+  std::string err;
+  const int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, 1, 0, env_algo(),
+                                 (flags & FFTSTENCIL_PERIODIC) ? 1 : 0);
+  if (rc != FFTSTENCIL_OK) { set_error(err); return rc; }
+  fill_info(hp, info);
+  clear_error();
+  return FFTSTENCIL_OK;
+}
+
 int fftstencil_describe_dist(int ndim, const int64_t* extents, const double* weights, int radius, int T,
                              int nranks, int rank, fftstencil_info* info) {
   if (!info) { set_error("info must be non-NULL"); return FFTSTENCIL_EINVAL; }
@@ -660,9 +687,9 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
       int64_t rem = ti, idx[3] = {0, 0, 0};
       for (int a = hp.ndim - 1; a >= 0; --a) { idx[a] = rem % hp.nt[a]; rem /= hp.nt[a]; }
       for (int a = 0; a < hp.ndim; ++a) {
-        const int64_t o = idx[a] * hp.S[a];
+        const int64_t o = idx[a] * hp.S[a] - (hp.periodic ? hp.h : 0);
         const int64_t first = o + hp.h;
-        const int64_t last = std::min<int64_t>(o + hp.h + hp.S[a], hp.ext[a] - hp.h);
+        const int64_t last = std::min<int64_t>(o + hp.h + hp.S[a], hp.periodic ? hp.ext[a] : hp.ext[a] - hp.h);
         v.push_back((double)o);
         v.push_back((double)first);
         v.push_back((double)(last - first));
@@ -695,10 +722,17 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
 
 fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const double* weights, int radius,
                                         int T) {
+  return fftstencil_plan_create_ex(ndim, extents, weights, radius, T, 0);
+}
+
+fftstencil_plan* fftstencil_plan_create_ex(int ndim, const int64_t* extents, const double* weights, int radius,
+                                           int T, int flags) {
+  if (flags & ~FFTSTENCIL_PERIODIC) { set_error("unknown flags"); return nullptr; }
   fftstencil_plan* p = new (std::nothrow) fftstencil_plan();
   if (!p) { set_error("host allocation failed"); return nullptr; }
   std::string err;
-  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err, 1, 0, env_algo());
+  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err, 1, 0, env_algo(),
+                           (flags & FFTSTENCIL_PERIODIC) ? 1 : 0);
   if (rc != FFTSTENCIL_OK) { set_error(err); delete p; return nullptr; }
   if (setup_device(p) != FFTSTENCIL_OK) { free_plan(p); return nullptr; }
   clear_error();
@@ -809,6 +843,28 @@ int fftstencil_run_group(fftstencil_plan* const* plans, const double* const* in,
   for (int k = 0; k < nranks && !rc; ++k) rc = dist_end(plans[k], out[k], s);
   if (rc == FFTSTENCIL_OK) clear_error();
   return rc;
+}
+
+int fftstencil_run_emit(fftstencil_plan* p, const double* in, const int64_t* emit_steps, int n_emit,
+                        double* const* outs, void* stream) {
+  if (!p || !in || !emit_steps || !outs || n_emit < 1) { set_error("invalid emit arguments"); return FFTSTENCIL_EINVAL; }
+  int64_t prev = 0;
+  for (int k = 0; k < n_emit; ++k) {
+    if (emit_steps[k] < prev || !outs[k]) { set_error("emit steps must be non-decreasing, outs non-NULL"); return FFTSTENCIL_EINVAL; }
+    prev = emit_steps[k];
+  }
+  // each segment is an ordinary run from the previous output (the semigroup property)
+  const double* src = in;
+  int64_t done = 0, launches = 0;
+  for (int k = 0; k < n_emit; ++k) {
+    const int rc = fftstencil_run(p, src, outs[k], emit_steps[k] - done, stream);
+    if (rc != FFTSTENCIL_OK) return rc;
+    launches += p->last_launches;
+    src = outs[k];
+    done = emit_steps[k];
+  }
+  p->last_launches = launches;
+  return FFTSTENCIL_OK;
 }
 
 int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, int64_t total_steps, void* stream) {

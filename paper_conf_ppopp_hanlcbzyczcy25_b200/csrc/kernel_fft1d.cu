@@ -63,7 +63,7 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
 
   const int64_t g0 = a.win.g0, g1 = a.win.g0 + a.win.gn;
   for (int64_t p = warp; p < a.win.p_end; p += nwarps) {
-    const int64_t oa = 2 * p * S, ob = (2 * p + 1) * S;   // global cell of tile position 0
+    const int64_t oa = 2 * p * S + a.bd.shift, ob = oa + S;   // global cell of tile position 0
     const bool has_b = 2 * p + 1 < a.ntiles;
     // B fragment of X^T:  X[l1 = g][l2 = 2q+j] = x[crt(g, 2q+j)]  (CRT gather, L1-resident)
     double xr[2], xi[2];
@@ -72,9 +72,10 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
       xr[j] = 0.0;
       xi[j] = 0.0;
       if (pos[j] >= 0) {
-        const int64_t xa = oa + pos[j], xb = ob + pos[j];
-        if (xa < a.n && xa >= g0 && xa < g1) xr[j] = __ldg(a.src + (xa - g0));
-        if (has_b && xb < a.n && xb >= g0 && xb < g1) xi[j] = __ldg(a.src + (xb - g0));
+        int64_t xa = oa + pos[j], xb = ob + pos[j];
+        if (a.bd.wrap) { xa = wrap_index(xa, a.n); xb = wrap_index(xb, a.n); }
+        if (xa >= 0 && xa < a.n && xa >= g0 && xa < g1) xr[j] = __ldg(a.src + (xa - g0));
+        if (has_b && xb >= 0 && xb < a.n && xb >= g0 && xb < g1) xi[j] = __ldg(a.src + (xb - g0));
       }
     }
     double m1r[2], m1i[2], m2r[2], m2i[2];
@@ -94,8 +95,8 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
       const int l = pos[j];
       if (l >= h && l < L - h) {                   // valid window (Eq. 7, reading Q4)
         const int64_t xa = oa + l, xb = ob + l;
-        if (xa < a.n - h && xa >= a.win.w_lo && xa < a.win.w_hi) a.dst[xa - g0] = m2r[j];
-        if (has_b && xb < a.n - h && xb >= a.win.w_lo && xb < a.win.w_hi) a.dst[xb - g0] = m2i[j];
+        if (xa < a.bd.lim0 && xa >= a.win.w_lo && xa < a.win.w_hi) a.dst[xa - g0] = m2r[j];
+        if (has_b && xb < a.bd.lim0 && xb >= a.win.w_lo && xb < a.win.w_hi) a.dst[xb - g0] = m2i[j];
       }
     }
   }

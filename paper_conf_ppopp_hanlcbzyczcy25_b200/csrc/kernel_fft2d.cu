@@ -45,17 +45,19 @@ template <int L, bool ASYNC>
 __device__ __forceinline__ void load_pair(double* sXa, double* sXb, const Fft2dArgs& a, int64_t p, int tid) {
   constexpr int LD = L + 4, NTHR = L * 4;
   const int64_t t0 = p / a.npr, j = p - t0 * a.npr;
-  const int64_t o0 = t0 * a.S;            // global row of tile row 0
+  const int64_t o0 = t0 * a.S + a.bd.shift;   // global row of tile row 0
 #pragma unroll
   for (int t = 0; t < 2; ++t) {
     const int64_t t1 = 2 * j + t;
     double* sX = t ? sXb : sXa;
     const bool have = t1 < a.nt1;
-    const int64_t o1 = t1 * a.S;
+    const int64_t o1 = t1 * a.S + a.bd.shift;
     for (int e = tid; e < L * L; e += NTHR) {
       const int r = e / L, c = e - r * L;
-      const int64_t gr = o0 + r, gc = o1 + c, lr = gr - a.win.g0;
-      const bool valid = have && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc < a.n1;
+      int64_t gr = o0 + r, gc = o1 + c;
+      if (a.bd.wrap) { gr = wrap_index(gr, a.n0); gc = wrap_index(gc, a.n1); }
+      const int64_t lr = gr - a.win.g0;
+      const bool valid = have && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc >= 0 && gc < a.n1;
       double* dst = sX + r * LD + perm8(c);
       if (ASYNC) {
         cp_async8(dst, valid ? a.src + lr * a.n1 + gc : a.src, valid);
@@ -249,17 +251,17 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
       for (int mt = 0; mt < NT; ++mt) {
         if (mt < MT) {
           const int l0 = 8 * mt + g;
-          const int64_t c0 = t0 * S + h + l0;
-          const bool row_ok = l0 < S && c0 < a.n0 - h && c0 >= a.win.w_lo && c0 < a.win.w_hi;
+          const int64_t c0 = t0 * S + a.bd.shift + h + l0;
+          const bool row_ok = l0 < S && c0 < a.bd.lim0 && c0 >= a.win.w_lo && c0 < a.win.w_hi;
           double* drow = a.dst + (c0 - a.win.g0) * a.n1;
 #pragma unroll
           for (int j = 0; j < 2; ++j) {
             const int l1 = 8 * warp + 2 * q + j;
             if (row_ok && l1 < S) {
-              int64_t c1 = a1 * S + h + l1;
-              if (c1 < a.n1 - h) drow[c1] = Yr[mt][j];
-              c1 = b1 * S + h + l1;
-              if (has_b && c1 < a.n1 - h) drow[c1] = Yi[mt][j];
+              int64_t c1 = a1 * S + a.bd.shift + h + l1;
+              if (c1 < a.bd.lim1) drow[c1] = Yr[mt][j];
+              c1 = b1 * S + a.bd.shift + h + l1;
+              if (has_b && c1 < a.bd.lim1) drow[c1] = Yi[mt][j];
             }
           }
         }

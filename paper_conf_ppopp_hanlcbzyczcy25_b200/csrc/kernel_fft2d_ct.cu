@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a, co
 
   for (int64_t p = a.win.p_begin + blockIdx.x; p < a.win.p_end; p += gridDim.x) {
     const int64_t t0 = p / a.npr, pj = p - t0 * a.npr;
-    const int64_t o0 = t0 * S, oa1 = 2 * pj * S, ob1 = oa1 + S;
+    const int64_t o0 = t0 * S + a.bd.shift, oa1 = 2 * pj * S + a.bd.shift, ob1 = oa1 + S;
     const bool has_b = 2 * pj + 1 < a.nt1;
     if (TMA) tma::fence_proxy_async();
     __syncthreads();   // previous pair's phase 3 reads are done
@@ -226,8 +226,10 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a, co
     // ---- load the halo'd pair (cp.async, OOB = 0) ----
     for (int e = tid; e < 2 * L * L; e += NW * 32) {
       const int t = e >> 12, r = (e >> 6) & 63, c = e & 63;
-      const int64_t gr = o0 + r, gc = (t ? ob1 : oa1) + c, lr = gr - a.win.g0;
-      const bool valid = (t == 0 || has_b) && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc < a.n1;
+      int64_t gr = o0 + r, gc = (t ? ob1 : oa1) + c;
+      if (a.bd.wrap) { gr = wrap_index(gr, a.n0); gc = wrap_index(gc, a.n1); }
+      const int64_t lr = gr - a.win.g0;
+      const bool valid = (t == 0 || has_b) && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc >= 0 && gc < a.n1;
       cp_async8((t ? sI : sR) + sw(r, c), valid ? a.src + lr * a.n1 + gc : a.src, valid);
     }
     asm volatile("cp.async.commit_group;\n" ::);
@@ -317,16 +319,16 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a, co
       for (int u = 0; u < NL; ++u) {
         const int i = ib + u;
         const int64_t c0 = o0 + h + i;
-        if (i >= S || c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
+        if (i >= S || c0 >= a.bd.lim0 || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
         double* drow = a.dst + (c0 - a.win.g0) * a.n1;
 #pragma unroll
         for (int j = 0; j < 2; ++j) {
           const int l1 = 8 * g + 2 * q + j;
           if (l1 >= h && l1 < h + S) {
             int64_t c1 = oa1 + l1;
-            if (c1 < a.n1 - h) drow[c1] = c2r[u][j];
+            if (c1 < a.bd.lim1) drow[c1] = c2r[u][j];
             c1 = ob1 + l1;
-            if (has_b && c1 < a.n1 - h) drow[c1] = c2i[u][j];
+            if (has_b && c1 < a.bd.lim1) drow[c1] = c2i[u][j];
           }
         }
       }

@@ -62,20 +62,22 @@ __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
     __syncthreads();
     const int64_t line = p / a.npr, pj = p - line * a.npr;
     const int64_t t0 = line / a.nt1, t1 = line - t0 * a.nt1;
-    const int64_t o0 = t0 * S, o1 = t1 * S;
+    const int64_t o0 = t0 * S + a.bd.shift, o1 = t1 * S + a.bd.shift;
     // ---- load the halo'd pair: rows of 16 doubles (128 B), OOB = 0 ----
 #pragma unroll
     for (int t = 0; t < 2; ++t) {
       const int64_t t2 = 2 * pj + t;
       double* sX = t ? sXb : sXa;
       const bool have = t2 < a.nt2;
-      const int64_t o2 = t2 * S;
+      const int64_t o2 = t2 * S + a.bd.shift;
       for (int e = tid; e < L * L * L; e += NW3 * 32) {
         const int l0 = e >> 8, l1 = (e >> 4) & 15, l2 = e & 15;
         double v = 0.0;
         if (have) {
-          const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = o2 + l2, lg0 = g0 - a.win.g0;
-          if (g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2)
+          int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = o2 + l2;
+          if (a.bd.wrap) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
+          const int64_t lg0 = g0 - a.win.g0;
+          if (g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 && g1 < a.n1 && g2 >= 0 && g2 < a.n2)
             v = __ldg(a.src + (lg0 * a.n1 + g1) * a.n2 + g2);
         }
         sX[l0 * SL + l1 * LD + perm8(l2)] = v;
@@ -201,10 +203,10 @@ __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
 
     // ---- phase 3: per output slice l0 < S: inverse along axes 2 then 1, crop, store ----
     const bool has_b = 2 * pj + 1 < a.nt2;
-    const int64_t oa2 = 2 * pj * S, ob2 = oa2 + S;
+    const int64_t oa2 = 2 * pj * S + a.bd.shift, ob2 = oa2 + S;
     for (int l0 = warp; l0 < S; l0 += NW3) {
       const int64_t c0 = o0 + h + l0;
-      if (c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
+      if (c0 >= a.bd.lim0 || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
       double* dplane = a.dst + (c0 - a.win.g0) * a.n1 * a.n2;
       const double* wa = sXa + l0 * SL;
       const double* wb = sXb + l0 * SL;
@@ -263,11 +265,11 @@ __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
           for (int j = 0; j < 2; ++j) {
             const int l2 = 8 * n + 2 * q + j;
             const int64_t c1 = o1 + h + l1;
-            if (l1 < S && l2 < S && c1 < a.n1 - h) {
+            if (l1 < S && l2 < S && c1 < a.bd.lim1) {
               int64_t c2 = oa2 + h + l2;
-              if (c2 < a.n2 - h) dplane[c1 * a.n2 + c2] = Yr[m][n][j];
+              if (c2 < a.bd.lim2) dplane[c1 * a.n2 + c2] = Yr[m][n][j];
               c2 = ob2 + h + l2;
-              if (has_b && c2 < a.n2 - h) dplane[c1 * a.n2 + c2] = Yi[m][n][j];
+              if (has_b && c2 < a.bd.lim2) dplane[c1 * a.n2 + c2] = Yi[m][n][j];
             }
           }
         }

@@ -154,7 +154,7 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
   for (int64_t p = a.win.p_begin + blockIdx.x; p < a.win.p_end; p += gridDim.x) {
     const int64_t line = p / a.npr, pj = p - line * a.npr;
     const int64_t t0 = line / a.nt1, t1 = line - t0 * a.nt1;
-    const int64_t o0 = t0 * S, o1 = t1 * S, oa2 = 2 * pj * S, ob2 = oa2 + S;
+    const int64_t o0 = t0 * S + a.bd.shift, o1 = t1 * S + a.bd.shift, oa2 = 2 * pj * S + a.bd.shift, ob2 = oa2 + S;
     const bool has_b = 2 * pj + 1 < a.nt2;
     __syncthreads();
     if (V16) {
@@ -162,7 +162,8 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
       for (int e = tid; e < 2 * L * L * 8; e += NWC * 32) {
         const int t = e >> 11, l0 = (e >> 7) & 15, l1 = (e >> 3) & 15, l2 = (e & 7) * 2;
         const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2, lg0 = g0 - a.win.g0;
-        const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2;
+        const bool valid = (t == 0 || has_b) && g0 >= 0 && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 &&
+                           g1 < a.n1 && g2 >= 0 && g2 < a.n2;
         cp_async16((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src,
                    valid);
       }
@@ -170,8 +171,11 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
       // ---- load the halo'd pair (8-byte cp.async, OOB = 0) ----
       for (int e = tid; e < 2 * L * L * L; e += NWC * 32) {
         const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
-        const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2, lg0 = g0 - a.win.g0;
-        const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 < a.n1 && g2 < a.n2;
+        int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2;
+        if (a.bd.wrap) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
+        const int64_t lg0 = g0 - a.win.g0;
+        const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 && g1 < a.n1 &&
+                           g2 >= 0 && g2 < a.n2;
         cp_async8((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src,
                   valid);
       }
@@ -221,16 +225,16 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
       double cr[2], ci[2];
       inv_group(sR, sI, ln, rg, g, q, false, cr, ci);
       const int64_t c0 = o0 + l0, c1 = o1 + l1b + q;
-      if (off1 + q >= S || c0 >= a.n0 - h || c0 < a.win.w_lo || c0 >= a.win.w_hi || c1 >= a.n1 - h) continue;
+      if (off1 + q >= S || c0 >= a.bd.lim0 || c0 < a.win.w_lo || c0 >= a.win.w_hi || c1 >= a.bd.lim1) continue;
       double* drow = a.dst + ((c0 - a.win.g0) * a.n1 + c1) * a.n2;
 #pragma unroll
       for (int j = 0; j < 2; ++j) {
         const int l2 = 2 * g + j;
         if (l2 >= h && l2 < h + S) {
           int64_t c2 = oa2 + l2;
-          if (c2 < a.n2 - h) drow[c2] = cr[j];
+          if (c2 < a.bd.lim2) drow[c2] = cr[j];
           c2 = ob2 + l2;
-          if (has_b && c2 < a.n2 - h) drow[c2] = ci[j];
+          if (has_b && c2 < a.bd.lim2) drow[c2] = ci[j];
         }
       }
     }

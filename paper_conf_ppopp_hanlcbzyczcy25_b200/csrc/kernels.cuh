@@ -19,6 +19,21 @@ struct Window {
   int64_t p_begin, p_end;
 };
 
+// Boundary handling of a launch (NEXT-2).  Fixed ring: wrap = 0, shift = 0, lim = n - h.
+// Periodic: wrap = 1, shift = -h, lim = n.  Tile t covers cells t*S + shift + [0, L) (taken
+// modulo n when wrapping, else zero outside the grid) and writes cells t*S + shift + h + l,
+// l in [0, S), below lim on every axis.
+struct Bound {
+  int wrap;
+  int shift;
+  int64_t lim0, lim1, lim2;
+};
+
+__host__ __device__ __forceinline__ int64_t wrap_index(int64_t x, int64_t n) {
+  x %= n;
+  return x < 0 ? x + n : x;
+}
+
 // Tile pairs (Double-layer Filling, Eq. 9): tiles are paired along the innermost tile axis
 // within one row of tiles -- (.., 2j) with (.., 2j+1); an odd row count pairs the last tile
 // with zeros.  Pairs never straddle an outer-axis tile row, so a decomposition into whole
@@ -33,6 +48,7 @@ struct Fft2dArgs {
   int64_t nt1;           // tiles along axis 1
   int64_t npr;           // pairs per tile row = ceil(nt1 / 2)
   Window win;
+  Bound bd;
   const double* Fre;     // L x L forward DFT matrix, row-major, columns permuted (perm8)
   const double* Fim;
   const double* Sre;     // L x L powered spectrum of this pass, natural row-major
@@ -47,6 +63,7 @@ struct Fft1dArgs {
   int h, S, L;           // L = N1*N2 = 56
   int64_t ntiles;        // pair p holds tiles 2p and 2p+1
   Window win;
+  Bound bd;
   const double* Fre;     // 16 x 8: rows 0..7 F_N1, rows 8..15 F_N2 zero-padded
   const double* Fim;
   const double* Sre;     // 8 x 8 Ruritanian-ordered powered spectrum, zero-padded
@@ -63,6 +80,7 @@ struct Fft3dArgs {
   int64_t nt1, nt2;      // tiles along axes 1 and 2
   int64_t npr;           // pairs per (t0, t1) tile line = ceil(nt2 / 2)
   Window win;
+  Bound bd;
   const double* Fre;     // 16 x 16 forward DFT matrix
   const double* Fim;
   const double* Sre;     // powered spectrum in [k1][k2][k0] order

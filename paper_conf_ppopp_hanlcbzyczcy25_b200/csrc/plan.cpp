@@ -108,8 +108,10 @@ static double model_flops_1d(int S, int T) {  // one 8x8 complex tile, 4 GEMMs o
 }
 
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
-                    HostPlan& p, std::string& err, int nranks, int rank, int algo) {
+                    HostPlan& p, std::string& err, int nranks, int rank, int algo, int periodic) {
   p = HostPlan();
+  p.periodic = periodic != 0;
+  if (p.periodic && nranks > 1) { err = "periodic boundaries are single-GPU in this build"; return FFTSTENCIL_EUNSUPPORTED; }
   if (nranks < 1 || rank < 0 || rank >= nranks) { err = "need 0 <= rank < nranks"; return FFTSTENCIL_EINVAL; }
   if (ndim < 1 || ndim > 3) { err = "ndim must be 1, 2 or 3"; return FFTSTENCIL_EINVAL; }
   if (!extents || !weights) { err = "extents and weights must be non-NULL"; return FFTSTENCIL_EINVAL; }
@@ -243,7 +245,8 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   // ---- overlap-save schedule (Eq. 3 / Eq. 4 / Eq. 7; reading Q4: centred window) ----
   p.tiles = 1;
   for (int a = 0; a < ndim; ++a) {
-    p.nt[a] = ceil_div(p.ext[a] - 2 * p.h, p.S[a]);
+    // fixed ring: the exact region [h, n-h) is tiled; periodic: every cell is (NEXT-2)
+    p.nt[a] = ceil_div(p.periodic ? p.ext[a] : p.ext[a] - 2 * p.h, p.S[a]);
     p.tiles *= p.nt[a];
   }
   // Double-layer Filling pairs (Eq. 9): along the innermost tile axis within one outer
@@ -399,7 +402,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   // ---- fixed ring: exact partition into boxes (axis a faces, lower axes interior) ----
   const int r = radius, h = p.h;
   const int off = 3 - ndim;
-  for (int a = 0; a < ndim; ++a) {
+  for (int a = 0; a < ndim && !p.periodic; ++a) {
     for (int side = 0; side < 2; ++side) {
       Box b;
       for (int e = 0; e < 3; ++e) { b.lo[e] = 0; b.hi[e] = p.n[e]; }
@@ -415,7 +418,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   // ---- boundary band: interior cells outside the exact region [h, n-h) (reading Q5) ----
   // Face of axis a: c_a in [r, h) or [n_a-h, n_a-r); axes before a exact ([h, n-h)),
   // axes after a interior ([r, n-r)).  The boxes partition the band exactly.
-  if (h > r) {
+  if (h > r && !p.periodic) {
     for (int a = 0; a < ndim; ++a)
       for (int side = 0; side < 2; ++side) {
         Box b;

@@ -38,6 +38,7 @@ struct HostPlan {
   int S[3] = {1, 1, 1};            // valid extent per user axis
   int N1 = 0, N2 = 0;              // 1D prime-factor split
   int algo = 0;                    // 2D: 0 = dense L x L DFT GEMMs, 1 = factored 64 = 8 x 8 (CT)
+  int periodic = 0;                // 1: periodic boundary (no ring/band, wrap-around tiles)
   int64_t nt[3] = {1, 1, 1};       // tiles per user axis
   int64_t tiles = 0, pairs = 0;
   int64_t npr = 1;                 // pairs per outer tile row (2D) / tile line (3D)
@@ -69,7 +70,8 @@ struct HostPlan {
 // nranks/rank select one slab of the outer-axis decomposition (1/0 = whole grid).
 // algo (2D only): -1 = choose by the cost model, 0 = dense, 1 = factored (CT 8 x 8).
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
-                    HostPlan& p, std::string& err, int nranks = 1, int rank = 0, int algo = -1);
+                    HostPlan& p, std::string& err, int nranks = 1, int rank = 0, int algo = -1,
+                    int periodic = 0);
 
 // Dense-DFT tile cost model (executed FP64 tensor flops per cell-step) used to pick L/T.
 double model_flops_2d(int L, int S, int T);

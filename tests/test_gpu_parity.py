@@ -211,6 +211,70 @@ def test_plans_with_different_band_sizes_coexist(fs):
     del small
 
 
+# ---------------------------------------------------------------- periodic mode + flexible outputs (NEXT-2)
+PERIODIC_CASES = [((300,), "star", 1, 8, 21), ((130, 141), "box", 1, 4, 11), ((96, 90), "star", 3, 2, 7),
+                  ((34, 30, 28), "box", 1, 2, 5), ((40, 33, 36), "star", 1, 3, 7)]
+
+
+@pytest.mark.parametrize("algo", ["factored", "dense"])
+@pytest.mark.parametrize("ext,shape,r,T,steps", PERIODIC_CASES)
+def test_periodic_parity_vs_oracle(fs, monkeypatch, algo, ext, shape, r, T, steps):
+    monkeypatch.setenv("FFTSTENCIL_ALGO", algo)
+    w = wl.seeded_weights(shape, len(ext), r)
+    u0 = wl.grid(ext, 19)
+    p = fs.Plan(ext, w, r, T, periodic=True)
+    assert p.info()["periodic"]
+    a = torch.from_numpy(u0).cuda()
+    b = torch.empty_like(a)
+    p.run(a, b, steps)
+    torch.cuda.synchronize()
+    ref = oracle.stencil_run(u0, w, r, steps, periodic=True)
+    assert rel_err(b.cpu().numpy(), ref) <= TOL
+
+
+@pytest.mark.parametrize("name,steps", [("heat2d", 1000), ("box2d49p", 200), ("box3d27p", 100)])
+def test_periodic_plane_wave_full_grid(fs, name, steps):
+    """Oracle-free full-grid pin at the BASELINE size: on a periodic grid a plane wave
+    cos(theta.c) becomes Re(sigma(theta)^s e^{i theta.c}) exactly."""
+    wk = wl.CONFIGS[name]
+    w = wk.weights()
+    nd, r = wk.ndim, wk.radius
+    n = wk.extents
+    ks = (3, 5, 2)[:nd]
+    th = [2 * np.pi * ks[a] / n[a] for a in range(nd)]
+    idx = np.meshgrid(*[np.arange(e, dtype=np.float64) for e in n], indexing="ij", sparse=True)
+    phase = sum(th[a] * idx[a] for a in range(nd))
+    sig = 0j
+    for off in np.ndindex(*w.shape):
+        sig += w[off] * np.exp(1j * sum((off[a] - r) * th[a] for a in range(nd)))
+    u0 = np.cos(phase)
+    p = fs.Plan(n, w, r, 0, periodic=True)
+    a = torch.from_numpy(np.ascontiguousarray(u0)).cuda()
+    del u0
+    b = torch.empty_like(a)
+    p.run(a, b, steps)
+    torch.cuda.synchronize()
+    del a
+    got = b.cpu().numpy()
+    ref = np.real(sig ** steps * np.exp(1j * phase))
+    assert np.abs(got - ref).max() <= 1e-9
+
+
+def test_run_emit_matches_separate_runs(fs):
+    ext = (150, 130)
+    w = wl.seeded_weights("box", 2, 1)
+    u0 = wl.grid(ext, 23)
+    p = fs.Plan(ext, w, 1, 8)
+    a = torch.from_numpy(u0).cuda()
+    steps = [0, 5, 13, 13, 40]
+    outs = [torch.empty_like(a) for _ in steps]
+    p.run_emit(a, outs, steps)
+    torch.cuda.synchronize()
+    for s, o in zip(steps, outs):
+        ref = oracle.stencil_run(u0, w, 1, s)
+        assert rel_err(o.cpu().numpy(), ref) <= TOL, s
+
+
 def test_invalid_arguments(fs):
     w = wl.seeded_weights("box", 2, 1)
     with pytest.raises(fs.FftStencilError):
