@@ -64,7 +64,7 @@ struct fftstencil_plan {
   size_t device_bytes = 0;
   int fused_grid = 0;
   int variant = 0;            // fused-kernel variant (2D dense)
-  int ct_cfg = 82;            // factored 2D kernel: 10 * warps per CTA + lines per warp step
+  int ct_cfg = 81;            // factored 2D kernel: 10 * warps per CTA + lines per warp step (TMA: 3 CTAs/SM)
   bool use_tma = true;        // TMA tile loads where the grid allows (FFTSTENCIL_TMA=0 disables)
   int band_reference = 0;     // FFTSTENCIL_BAND=reference selects the first band kernel
   size_t band_smem = 0;

@@ -22,8 +22,9 @@
 //   phase 3  output rows (S):  iDFT8 over kb1, twiddle*, B-route iDFT8 over ka1 -> store
 // Phases 1 and 2 overwrite exactly the shared-memory words each thread read (in place);
 // the two CTA barriers are the transpositions of ownership a 2D transform needs.
-// Shared layout: plane[r][c] at r*97 + c + 8*(c>>4) + 8*((r>>4)&1): both the row pattern
-// (c = 16q + 8j + g) and the column pattern (r = 16q + 8j + g) hit every bank pair twice.
+// Shared layout: plane[r][c] at r*64 + (c ^ 8((c>>4)&1) ^ (r&7) ^ 8((r>>4)&1)) (XOR swizzle):
+// both the row pattern (c = 16q + 8j + g) and the column pattern (r = 16q + 8j + g) hit every
+// bank pair exactly twice.
 #include "device_common.cuh"
 #include "kernels.cuh"
 #include "tma.cuh"
@@ -34,10 +35,14 @@ namespace {
 using dev::dmma;
 
 constexpr int L = 64;
-constexpr int LDR = 97;
-constexpr int PLANE = L * LDR;
+constexpr int PLANE = L * L;
 
-__device__ __forceinline__ int sw(int r, int c) { return r * LDR + c + 8 * (c >> 4) + 8 * ((r >> 4) & 1); }
+// XOR-swizzled dense layout: both fragment patterns (row r fixed, c = 16q + 8j + g; and
+// column c fixed, r = 16q + 8j + g) hit every bank pair exactly twice, the optimum for 32
+// doubles; 64 KB for the two planes (3 CTAs / SM on the cp.async path).
+__device__ __forceinline__ int sw(int r, int c) {
+  return r * L + (c ^ (8 * ((c >> 4) & 1)) ^ (r & 7) ^ (8 * ((r >> 4) & 1)));
+}
 
 __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
@@ -144,11 +149,12 @@ __device__ __forceinline__ void twiddle_n(double (&cr)[NL][2], double (&ci)[NL][
   for (int u = 0; u < NL; ++u) twiddle<CONJ>(cr[u], ci[u], tr, ti);
 }
 
-// TMA = true: each tile arrives by one 64 x 64 TMA box (OOB -> 0) in a dense staging
-// layout; phase 1 reads it (4-way bank conflicts on that pass only), keeps its results in
-// registers across a CTA barrier and writes Q into the padded layout over the same memory.
+// TMA = true: each tile arrives by one 64 x 64 TMA box (OOB -> 0) in a dense row-major
+// layout; phase 1 reads its rows there (4-way bank conflicts on that pass only) and, the
+// XOR swizzle being a permutation within a row, rewrites each row in place swizzled.
 template <int NW, int NL, bool TMA>
-__global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a, const __grid_constant__ CUtensorMap tm) {
+__global__ void __launch_bounds__(NW * 32, NL > 2 ? 2 : 3)
+    fft2d_ct_kernel(const Fft2dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ __align__(128) double smem[];
   double* sR = smem;            // plane 0: tile 2j (Re), then Q/W real parts
   double* sI = smem + PLANE;    // plane 1: tile 2j+1 (Im), then Q/W imaginary parts
@@ -192,13 +198,10 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a, co
       tma::mbar_wait(&bar, parity);
       parity ^= 1;
       __syncthreads();
-      // ---- phase 1 from the dense staging layout; results held until the barrier ----
-      constexpr int ITER = L / (NW * NL);
-      double qr[ITER][NL][2], qi[ITER][NL][2];
-#pragma unroll
-      for (int it = 0; it < ITER; ++it) {
-        const int l0b = warp * NL + it * NW * NL;
-        double br[NL][2], bi[NL][2], c1r[NL][2], c1i[NL][2];
+      // ---- phase 1 from the dense staging rows; the swizzled layout permutes words within a
+      // row only, so each warp rewrites its own rows in place ----
+      for (int l0b = warp * NL; l0b < L; l0b += NW * NL) {
+        double br[NL][2], bi[NL][2], c1r[NL][2], c1i[NL][2], c2r[NL][2], c2i[NL][2];
 #pragma unroll
         for (int u = 0; u < NL; ++u)
 #pragma unroll
@@ -208,18 +211,14 @@ __global__ void __launch_bounds__(NW * 32) fft2d_ct_kernel(const Fft2dArgs a, co
           }
         broute_n<false, NL>(c1r, c1i, fr, fi, br, bi);
         twiddle_n<false, NL>(c1r, c1i, tr, ti);
-        aroute_n<false, NL>(qr[it], qi[it], c1r, c1i, fr, fi);
-      }
-      __syncthreads();
-#pragma unroll
-      for (int it = 0; it < ITER; ++it) {
-        const int l0b = warp * NL + it * NW * NL;
+        aroute_n<false, NL>(c2r, c2i, c1r, c1i, fr, fi);
+        __syncwarp();
 #pragma unroll
         for (int u = 0; u < NL; ++u)
 #pragma unroll
           for (int j = 0; j < 2; ++j) {
-            sR[sw(l0b + u, cl[j])] = qr[it][u][j];
-            sI[sw(l0b + u, cl[j])] = qi[it][u][j];
+            sR[sw(l0b + u, cl[j])] = c2r[u][j];
+            sI[sw(l0b + u, cl[j])] = c2i[u][j];
           }
       }
     } else {
@@ -349,10 +348,13 @@ cudaError_t configure_nw(int* max_blocks) {
 
 size_t fused2d_ct_smem() { return (size_t)2 * PLANE * sizeof(double); }
 
-// cfg = 10 * NW + NL: 81, 82, 84, 161, 162 (the TMA instantiation exists for 82 and 84)
+// cfg = 10 * NW + NL: 81, 82, 84, 161, 162 (TMA instantiations for 81, 82 and 84)
 cudaError_t fused2d_ct_configure(int cfg, int* max_blocks) {
   switch (cfg) {
-    case 81: return configure_nw<8, 1, false>(max_blocks);
+    case 81: {
+      cudaError_t e = configure_nw<8, 1, true>(max_blocks);
+      return e != cudaSuccess ? e : configure_nw<8, 1, false>(max_blocks);
+    }
     case 82: {
       cudaError_t e = configure_nw<8, 2, true>(max_blocks);
       return e != cudaSuccess ? e : configure_nw<8, 2, false>(max_blocks);
@@ -371,7 +373,9 @@ cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, const CUtensorMap* tm
   const size_t smem = fused2d_ct_smem();
   static const CUtensorMap none = {};
   const CUtensorMap& m = tm ? *tm : none;
-  if (tm && cfg == 82) {
+  if (tm && cfg == 81) {
+    fft2d_ct_kernel<8, 1, true><<<grid, 256, smem, s>>>(a, m);
+  } else if (tm && cfg == 82) {
     fft2d_ct_kernel<8, 2, true><<<grid, 256, smem, s>>>(a, m);
   } else if (tm && cfg == 84) {
     fft2d_ct_kernel<8, 4, true><<<grid, 256, smem, s>>>(a, m);

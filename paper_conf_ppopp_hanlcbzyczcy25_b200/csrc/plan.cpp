@@ -201,7 +201,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     } else {
       p.flops_per_cell_step = model_flops_2d_ct(p.S[0], bT);
       p.mma_flops_per_pair = 512.0 * (3072.0 + 16.0 * S);
-      p.fused_smem = (size_t)2 * 64 * 97 * sizeof(double);
+      p.fused_smem = (size_t)2 * 64 * 64 * sizeof(double);
     }
   } else {
     // candidates: the dense 16^3 tile and the factored one (16 = 8 x 2 per axis)
