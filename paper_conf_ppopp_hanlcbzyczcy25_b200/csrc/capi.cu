@@ -291,8 +291,11 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Sim = Sim;
     if (hp.algo == 1) {
       a.Fim = p->dF + 128;
-      const bool v16 = p->use_tma && !hp.periodic && hp.ext[2] % 2 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0;
-      e = launch_fused3d_ct(a, v16, (int)std::min<int64_t>(p->fused_grid, np), s);
+      CUtensorMap tm;
+      const uint64_t dims[3] = {(uint64_t)hp.ext[2], (uint64_t)hp.ext[1], (uint64_t)(hp.g1 - hp.g0)};
+      const uint32_t box[3] = {16, 16, 16};
+      const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 3, dims, box);
+      e = launch_fused3d_ct(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
       e = launch_fused3d(a, (int)std::min<int64_t>(p->fused_grid, np), s);

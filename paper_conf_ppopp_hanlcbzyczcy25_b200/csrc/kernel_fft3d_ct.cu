@@ -16,12 +16,16 @@
 //   P1 forward axis 2 | P2 forward axis 1 | P3 forward axis 0, * S_T, inverse axis 0 |
 //   P4 inverse axis 1 on the S output planes | P5 inverse axis 2 on the S x S output rows
 //   -> store the S^3 window.
-// Shared layout [l0][l1][l2] at l0*290 + l1*18 + l2: every fragment pattern of the five
-// passes costs at most 4 (mostly 2) wavefronts per 32 doubles; 72.5 KB -> 3 CTAs / SM.
-// (R even keeps every tile row 16-byte aligned for 16-byte cp.async; TMA tensor copies
-// would need 128-byte-aligned destinations, which this conflict-free padding excludes.)
+// Shared layout: dense [l0][l1][l2] with l2 XOR-swizzled by a GF(2)-linear f(l0, l1) (parity
+// masks 0xB2, 0x21, 0xA5, 0xEE of l0 | l1 << 4, found by search and checked exhaustively;
+// evaluated as T0[l0] ^ T1[l1] from two packed 4-bit tables):
+// every fragment pattern of the five passes costs the optimal 2 wavefronts per 32 doubles,
+// 64 KB for both planes -> 3 CTAs / SM.  f permutes words within a 16-element row only, so
+// with TMA the tiles land as two dense 16^3 boxes and P1 (whose groups own whole rows)
+// reads them unswizzled and rewrites its rows swizzled in place.
 #include "device_common.cuh"
 #include "kernels.cuh"
+#include "tma.cuh"
 
 namespace fstencil {
 namespace {
@@ -29,24 +33,34 @@ namespace {
 using dev::dmma;
 
 constexpr int L = 16;
-constexpr int R = 18;               // 16-byte aligned rows (TMA destinations)
-constexpr int SL = 290;
-constexpr int PLANE = L * SL;
+constexpr int PLANE = L * L * L;
 constexpr int NWC = 8;
+
+// f(l0, l1) = T0[l0] ^ T1[l1] (f is GF(2)-linear); the 16 x 4-bit tables packed in 64 bits.
+__device__ __forceinline__ int swz(int l0, int l1) {
+  constexpr unsigned long long kT0 = 0xbd2471e835acf960ull, kT1 = 0xba4532cd6798ef10ull;
+  return (int)(((kT0 >> (4 * l0)) ^ (kT1 >> (4 * l1))) & 15ull);
+}
+__device__ __forceinline__ int off3(int l0, int l1, int l2) { return (l0 << 8) | (l1 << 4) | (l2 ^ swz(l0, l1)); }
 
 __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
 }
-__device__ __forceinline__ void cp_async16(double* dst, const double* src, bool valid) {
-  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 16 : 0));
-}
 
-// Offsets of the 4 lines of a group along one axis: line m, position p.
+// The 4 lines of a group: MODE 0 -> lines along l2 (l0 = a, l1 = b + m); MODE 1 -> along l1
+// (l0 = a, l2 = b + m); MODE 2 -> along l0 (l1 = a, l2 = b + m).  DENSE: unswizzled offsets
+// (the TMA staging layout, P1 reads only).
+template <int MODE, bool DENSE = false>
 struct Lines {
-  int base, mstride, pstride;
-  __device__ __forceinline__ int at(int m, int p) const { return base + m * mstride + p * pstride; }
+  int a, b;
+  __device__ __forceinline__ int at(int m, int p) const {
+    int l0, l1, l2;
+    if (MODE == 0) { l0 = a; l1 = b + m; l2 = p; }
+    else if (MODE == 1) { l0 = a; l1 = p; l2 = b + m; }
+    else { l0 = p; l1 = a; l2 = b + m; }
+    return DENSE ? (l0 << 8) | (l1 << 4) | l2 : off3(l0, l1, l2);
+  }
 };
 
 template <bool CONJ>
@@ -69,14 +83,15 @@ struct Regs {
   double itr[2], iti[2];   // conj(w16^(2q + j)) (inverse, lb = 1)
 };
 
-// Forward DFT-16 of the 4 lines; result (natural k order) written back in place, optionally
-// multiplied by the spectrum (sp = S_T at [line q][g][j], k = g + 8 j).
-__device__ __forceinline__ void fwd_group(double* sR, double* sI, const Lines& ln, const Regs& rg, int g, int q,
-                                          const double* spr, const double* spi) {
+// Forward DFT-16 of the 4 lines read through `rd`; result (natural k order) written back
+// through `wr` (same words), optionally multiplied by the spectrum (S_T at [q][g][j]).
+template <class RD, class WR>
+__device__ __forceinline__ void fwd_group(double* sR, double* sI, const RD& rd, const WR& wr, const Regs& rg, int g,
+                                          int q, const double* spr, const double* spi) {
   double br[2], bi[2], cr[2], ci[2];
 #pragma unroll
   for (int j = 0; j < 2; ++j) {
-    const int o = ln.at(g >> 1, 4 * q + 2 * j + (g & 1));
+    const int o = rd.at(g >> 1, 4 * q + 2 * j + (g & 1));
     br[j] = sR[o];
     bi[j] = sI[o];
   }
@@ -93,7 +108,7 @@ __device__ __forceinline__ void fwd_group(double* sR, double* sI, const Lines& l
   __syncwarp();   // the group is rewritten in place with another thread-to-word map
 #pragma unroll
   for (int j = 0; j < 2; ++j) {
-    const int o = ln.at(q, g + 8 * j);
+    const int o = wr.at(q, g + 8 * j);
     sR[o] = xr[j];
     sI[o] = xi[j];
   }
@@ -101,7 +116,8 @@ __device__ __forceinline__ void fwd_group(double* sR, double* sI, const Lines& l
 
 // Inverse DFT-16 (unnormalised; 1/16^3 is in S_T) of the 4 lines; returns the C fragment
 // (line q, positions 2g + j) in cr/ci; writes it back in place if `store`.
-__device__ __forceinline__ void inv_group(double* sR, double* sI, const Lines& ln, const Regs& rg, int g, int q,
+template <class LN>
+__device__ __forceinline__ void inv_group(double* sR, double* sI, const LN& ln, const Regs& rg, int g, int q,
                                           bool store, double (&cr)[2], double (&ci)[2]) {
   double br[2], bi[2];
   const int lb = g & 1;
@@ -130,14 +146,16 @@ __device__ __forceinline__ void inv_group(double* sR, double* sI, const Lines& l
   }
 }
 
-// V16: n2 even -> every tile row starts 16-byte aligned in HBM and in shared memory.
-template <bool V16>
-__global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a) {
-  extern __shared__ __align__(16) double smem[];
+template <bool TMA>
+__global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
+  extern __shared__ __align__(128) double smem[];
   double* sR = smem;
   double* sI = smem + PLANE;
+  __shared__ __align__(8) uint64_t bar;
   const int tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31, g = lane >> 2, q = lane & 3;
+  if (TMA && tid == 0) tma::mbar_init(&bar, 1);
+  uint32_t parity = 0;
   Regs rg;
 #pragma unroll
   for (int j = 0; j < 2; ++j) {
@@ -156,64 +174,66 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
     const int64_t t0 = line / a.nt1, t1 = line - t0 * a.nt1;
     const int64_t o0 = t0 * S + a.bd.shift, o1 = t1 * S + a.bd.shift, oa2 = 2 * pj * S + a.bd.shift, ob2 = oa2 + S;
     const bool has_b = 2 * pj + 1 < a.nt2;
+    if (TMA) tma::fence_proxy_async();
     __syncthreads();
-    if (V16) {
-      // ---- load the halo'd pair: 16-byte cp.async (rows are even-length and 16 B aligned) ----
-      for (int e = tid; e < 2 * L * L * 8; e += NWC * 32) {
-        const int t = e >> 11, l0 = (e >> 7) & 15, l1 = (e >> 3) & 15, l2 = (e & 7) * 2;
-        const int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2, lg0 = g0 - a.win.g0;
-        const bool valid = (t == 0 || has_b) && g0 >= 0 && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 &&
-                           g1 < a.n1 && g2 >= 0 && g2 < a.n2;
-        cp_async16((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src,
-                   valid);
+    if (TMA) {
+      // ---- load the halo'd pair: two dense 16^3 TMA boxes (OOB -> 0) ----
+      if (tid == 0) {
+        tma::mbar_expect_tx(&bar, (has_b ? 2u : 1u) * PLANE * 8u);
+        tma::load_3d(sR, &tm, (int)oa2, (int)o1, (int)(o0 - a.win.g0), &bar);
+        if (has_b) tma::load_3d(sI, &tm, (int)ob2, (int)o1, (int)(o0 - a.win.g0), &bar);
       }
+      if (!has_b)
+        for (int e = tid; e < PLANE; e += NWC * 32) sI[e] = 0.0;
+      tma::mbar_wait(&bar, parity);
+      parity ^= 1;
     } else {
-      // ---- load the halo'd pair (8-byte cp.async, OOB = 0) ----
-      for (int e = tid; e < 2 * L * L * L; e += NWC * 32) {
+      // ---- load the halo'd pair (8-byte cp.async into the swizzled layout, OOB = 0) ----
+      for (int e = tid; e < 2 * PLANE; e += NWC * 32) {
         const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
         int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2;
         if (a.bd.wrap) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
         const int64_t lg0 = g0 - a.win.g0;
         const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 && g1 < a.n1 &&
                            g2 >= 0 && g2 < a.n2;
-        cp_async8((t ? sI : sR) + l0 * SL + l1 * R + l2, valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src,
-                  valid);
+        cp_async8((t ? sI : sR) + off3(l0, l1, l2), valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src, valid);
       }
+      asm volatile("cp.async.commit_group;\n" ::);
+      asm volatile("cp.async.wait_all;\n" ::: "memory");
     }
-    asm volatile("cp.async.commit_group;\n" ::);
-    asm volatile("cp.async.wait_all;\n" ::: "memory");
     __syncthreads();
-    // ---- P1: forward axis 2 (lines = l1, 4 per group) ----
+    // ---- P1: forward axis 2 (lines along l2; TMA: read the dense rows, write swizzled) ----
     for (int grp = warp; grp < 64; grp += NWC) {
-      const Lines ln{(grp >> 2) * SL + (grp & 3) * 4 * R, R, 1};
-      fwd_group(sR, sI, ln, rg, g, q, nullptr, nullptr);
+      const Lines<0, TMA> rd{grp >> 2, (grp & 3) * 4};
+      const Lines<0> wr{grp >> 2, (grp & 3) * 4};
+      fwd_group(sR, sI, rd, wr, rg, g, q, nullptr, nullptr);
     }
     __syncthreads();
-    // ---- P2: forward axis 1 (lines = l2) ----
+    // ---- P2: forward axis 1 (lines along l1) ----
     for (int grp = warp; grp < 64; grp += NWC) {
-      const Lines ln{(grp >> 2) * SL + (grp & 3) * 4, 1, R};
-      fwd_group(sR, sI, ln, rg, g, q, nullptr, nullptr);
+      const Lines<1> ln{grp >> 2, (grp & 3) * 4};
+      fwd_group(sR, sI, ln, ln, rg, g, q, nullptr, nullptr);
     }
     __syncthreads();
-    // ---- P3: forward axis 0, * S_T, inverse axis 0 (lines = l2 at fixed k1) ----
+    // ---- P3: forward axis 0, * S_T, inverse axis 0 (lines along l0 at fixed k1) ----
     for (int grp = warp; grp < 64; grp += NWC) {
       const int k1 = grp >> 2, k2b = (grp & 3) * 4;
-      const Lines ln{k1 * R + k2b, 1, SL};
+      const Lines<2> ln{k1, k2b};
       const int64_t si = (((int64_t)k1 * 16 + k2b + q) * 8 + g) * 2;   // S_T at [k1][k2][g][j]
-      fwd_group(sR, sI, ln, rg, g, q, a.Sre + si, a.Sim + si);
+      fwd_group(sR, sI, ln, ln, rg, g, q, a.Sre + si, a.Sim + si);
       __syncwarp();
       double cr[2], ci[2];
       inv_group(sR, sI, ln, rg, g, q, true, cr, ci);
     }
     __syncthreads();
-    // ---- P4: inverse axis 1 on the S output planes (lines = l2) ----
+    // ---- P4: inverse axis 1 on the S output planes (lines along l1) ----
     for (int grp = warp; grp < 4 * S; grp += NWC) {
-      const Lines ln{(h + (grp >> 2)) * SL + (grp & 3) * 4, 1, R};
+      const Lines<1> ln{h + (grp >> 2), (grp & 3) * 4};
       double cr[2], ci[2];
       inv_group(sR, sI, ln, rg, g, q, true, cr, ci);
     }
     __syncthreads();
-    // ---- P5: inverse axis 2 on the S x S output rows (lines = l1), store the window ----
+    // ---- P5: inverse axis 2 on the S x S output rows (lines along l2), store the window ----
     for (int grp = warp; grp < S * G1; grp += NWC) {
       const int i0 = grp / G1, gi = grp - i0 * G1;
       const int l0 = h + i0;
@@ -221,7 +241,7 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
       // and stored twice with bitwise-identical values)
       const int off1 = S >= 4 ? min(4 * gi, S - 4) : 0;
       const int l1b = h + off1;
-      const Lines ln{l0 * SL + l1b * R, R, 1};
+      const Lines<0> ln{l0, l1b};
       double cr[2], ci[2];
       inv_group(sR, sI, ln, rg, g, q, false, cr, ci);
       const int64_t c0 = o0 + l0, c1 = o1 + l1b + q;
@@ -254,11 +274,12 @@ cudaError_t fused3d_ct_configure(int* max_blocks) {
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_ct_kernel<true>, NWC * 32, smem);
 }
 
-cudaError_t launch_fused3d_ct(const Fft3dArgs& a, bool v16, int grid, cudaStream_t s) {
-  if (v16)
-    fft3d_ct_kernel<true><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a);
+cudaError_t launch_fused3d_ct(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s) {
+  static const CUtensorMap none = {};
+  if (tm)
+    fft3d_ct_kernel<true><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a, *tm);
   else
-    fft3d_ct_kernel<false><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a);
+    fft3d_ct_kernel<false><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a, none);
   return cudaGetLastError();
 }
 

@@ -140,8 +140,8 @@ cudaError_t launch_fused3d(const Fft3dArgs& a, int grid, cudaStream_t s);
 // k = 0..15]; Sre/Sim = S_T in [k1][k2][k0 % 8][k0 / 8] order.
 size_t fused3d_ct_smem();
 cudaError_t fused3d_ct_configure(int* max_blocks_per_sm);
-// v16: 16-byte cp.async tile loads (n2 even and src 16-byte aligned), else 8-byte.
-cudaError_t launch_fused3d_ct(const Fft3dArgs& a, bool v16, int grid, cudaStream_t s);
+// tm: tensor map of the source buffer (dims {n2, n1, gn}, box {16, 16, 16}) or null (cp.async).
+cudaError_t launch_fused3d_ct(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
 
 constexpr int kBandThreads = 256;
 cudaError_t band_configure(size_t smem);

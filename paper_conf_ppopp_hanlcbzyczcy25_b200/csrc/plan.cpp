@@ -238,7 +238,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     } else {
       p.flops_per_cell_step = model_flops_3d_ct(p.S[0], bestT);
       p.mma_flops_per_pair = 4096.0 * groups_3d_ct(p.S[0]);
-      p.fused_smem = (size_t)2 * 16 * 290 * sizeof(double);
+      p.fused_smem = (size_t)2 * 16 * 16 * 16 * sizeof(double);
     }
   }
 
