@@ -22,9 +22,9 @@
 //   phase 3  output rows (S):  iDFT8 over kb1, twiddle*, B-route iDFT8 over ka1 -> store
 // Phases 1 and 2 overwrite exactly the shared-memory words each thread read (in place);
 // the two CTA barriers are the transpositions of ownership a 2D transform needs.
-// Shared layout: plane[r][c] at r*64 + (c ^ 8((c>>4)&1) ^ (r&7) ^ 8((r>>4)&1)) (XOR swizzle):
-// both the row pattern (c = 16q + 8j + g) and the column pattern (r = 16q + 8j + g) hit every
-// bank pair exactly twice.
+// Shared layout: plane[r][c] at r*64 + (c ^ 4(((c>>4) ^ (r>>4)) & 3) ^ (r & 3)) (XOR swizzle):
+// both the row pattern (c = 16q + 8j + g) and the column pattern (r = 16q + 8j + g) are
+// bank-conflict free per half-warp.
 #include "device_common.cuh"
 #include "kernels.cuh"
 #include "tma.cuh"
@@ -38,10 +38,11 @@ constexpr int L = 64;
 constexpr int PLANE = L * L;
 
 // XOR-swizzled dense layout: both fragment patterns (row r fixed, c = 16q + 8j + g; and
-// column c fixed, r = 16q + 8j + g) hit every bank pair exactly twice, the optimum for 32
-// doubles; 64 KB for the two planes (3 CTAs / SM on the cp.async path).
+// column c fixed, r = 16q + 8j + g) are conflict-free per half-warp (8-byte accesses are
+// served 16 lanes at a time: lanes 4g + q, g in one half), the optimal 2 wavefronts per 32
+// doubles; a permutation within each row; 64 KB for the two planes (3 CTAs / SM).
 __device__ __forceinline__ int sw(int r, int c) {
-  return r * L + (c ^ (8 * ((c >> 4) & 1)) ^ (r & 7) ^ (8 * ((r >> 4) & 1)));
+  return r * L + (c ^ (((((c >> 4) & 3) ^ ((r >> 4) & 3))) << 2) ^ (r & 3));
 }
 
 __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {

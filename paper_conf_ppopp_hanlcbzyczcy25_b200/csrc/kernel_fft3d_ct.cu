@@ -17,9 +17,10 @@
 //   P4 inverse axis 1 on the S output planes | P5 inverse axis 2 on the S x S output rows
 //   -> store the S^3 window.
 // Shared layout: dense [l0][l1][l2] with l2 XOR-swizzled by a GF(2)-linear f(l0, l1) (parity
-// masks 0xB2, 0x21, 0xA5, 0xEE of l0 | l1 << 4, found by search and checked exhaustively;
-// evaluated as T0[l0] ^ T1[l1] from two packed 4-bit tables):
-// every fragment pattern of the five passes costs the optimal 2 wavefronts per 32 doubles,
+// masks 0x45, 0x86, 0xbd, 0xd7 of l0 | l1 << 4, found by search and checked exhaustively;
+// evaluated as T0[l0] ^ T1[l1] from two packed 4-bit tables): every fragment pattern of the
+// five passes is conflict-free per half-warp (8-byte accesses are served 16 lanes at a
+// time), i.e. the optimal 2 wavefronts per 32 doubles,
 // 64 KB for both planes -> 3 CTAs / SM.  f permutes words within a 16-element row only, so
 // with TMA the tiles land as two dense 16^3 boxes and P1 (whose groups own whole rows)
 // reads them unswizzled and rewrites its rows swizzled in place.
@@ -38,7 +39,7 @@ constexpr int NWC = 8;
 
 // f(l0, l1) = T0[l0] ^ T1[l1] (f is GF(2)-linear); the 16 x 4-bit tables packed in 64 bits.
 __device__ __forceinline__ int swz(int l0, int l1) {
-  constexpr unsigned long long kT0 = 0xbd2471e835acf960ull, kT1 = 0xba4532cd6798ef10ull;
+  constexpr unsigned long long kT0 = 0xc16b3e94852f7ad0ull, kT1 = 0xf3b76a2e1d5984c0ull;
   return (int)(((kT0 >> (4 * l0)) ^ (kT1 >> (4 * l1))) & 15ull);
 }
 __device__ __forceinline__ int off3(int l0, int l1, int l2) { return (l0 << 8) | (l1 << 4) | (l2 ^ swz(l0, l1)); }
