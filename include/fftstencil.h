@@ -85,8 +85,10 @@ typedef struct {
   int64_t pair_begin, pair_end; /* tile pairs this rank computes                         */
   int64_t interior_begin, interior_end; /* pairs needing no halo rows (overlap the exchange) */
   int64_t ghost_lo, ghost_hi;   /* halo rows received from rank-1 / rank+1 per pass     */
-  int algo;                     /* 2D/3D tile algorithm: 0 dense L^d DFT GEMMs, 1 factored
-                                   (2D 64 = 8 x 8, 3D 16 = 8 x 2 Cooley-Tukey)              */
+  int algo;                     /* tile algorithm: 0 dense L^d DFT GEMMs, 1 factored (2D 64 =
+                                   8 x 8, 3D 16 = 8 x 2 Cooley-Tukey), 2 unfused 2D ablation
+                                   (FFTSTENCIL_ALGO=unfused: forward / multiply / inverse as
+                                   three kernels with the spectrum in HBM)                  */
   int periodic;                 /* 1 for a FFTSTENCIL_PERIODIC plan                      */
 } fftstencil_info;
 

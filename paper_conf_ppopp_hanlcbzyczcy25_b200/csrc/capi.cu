@@ -32,12 +32,13 @@ namespace {
 
 thread_local std::string g_last_error;
 
-// FFTSTENCIL_ALGO=dense|factored pins the 2D tile algorithm (ablations); default: cost model.
+// FFTSTENCIL_ALGO=dense|factored|unfused pins the tile algorithm (ablations); default: cost model.
 int env_algo() {
   const char* v = std::getenv("FFTSTENCIL_ALGO");
   if (!v) return -1;
   if (!std::strcmp(v, "dense")) return 0;
   if (!std::strcmp(v, "factored")) return 1;
+  if (!std::strcmp(v, "unfused")) return 2;   // NEXT-3 ablation (2D): three kernels per pass
   return -1;
 }
 
@@ -56,6 +57,7 @@ struct fftstencil_plan {
   double* dW = nullptr;
   int* dBlocks = nullptr;
   double* dScratch = nullptr; // single GPU: ping-pong partner of `out`
+  double* dSpec = nullptr;    // unfused ablation: per-pair spectra in HBM
   double* dHostIn = nullptr;  // run_host staging grids (lazy)
   double* dHostOut = nullptr;
   size_t spec_vol = 0;
@@ -141,6 +143,7 @@ void free_plan(fftstencil_plan* p) {
   cudaFree(p->dW);
   cudaFree(p->dBlocks);
   cudaFree(p->dScratch);
+  cudaFree(p->dSpec);
   cudaFree(p->dHostIn);
   cudaFree(p->dHostOut);
   cudaFree(p->dE[0]);
@@ -243,7 +246,16 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Sre = Sre;
     a.Sim = Sim;
     a.Fre = p->dF;
-    if (hp.algo == 1) {
+    a.spec = p->dSpec;
+    if (hp.algo == 2) {
+      // unfused ablation: forward -> HBM spectrum, multiply in HBM, inverse (3 launches)
+      a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
+      const int grid = (int)std::min<int64_t>(p->fused_grid, np);
+      e = launch_unfused2d(hp.L[0], 1, a, grid, s);
+      if (e == cudaSuccess) e = launch_spec_mul(p->dSpec, hp.pairs, hp.L[0], Sre, Sim, s);
+      if (e == cudaSuccess) e = launch_unfused2d(hp.L[0], 2, a, grid, s);
+      p->last_launches += 2;
+    } else if (hp.algo == 1) {
       a.Fim = p->dF + 128;
       CUtensorMap tm;
       const uint64_t dims[2] = {(uint64_t)hp.ext[1], (uint64_t)(hp.g1 - hp.g0)};
@@ -498,7 +510,7 @@ int setup_device(fftstencil_plan* p) {
   size_t acc = 0;
   std::vector<double> F(hp.Fre);
   F.insert(F.end(), hp.Fim.begin(), hp.Fim.end());
-  if (hp.ndim == 2 && hp.algo == 0) {
+  if (hp.ndim == 2 && (hp.algo == 0 || hp.algo == 2)) {
     // the dense 2D kernel reads F with columns permuted within groups of 8 (device_common.cuh)
     const int L = hp.L[0];
     for (int plane = 0; plane < 2; ++plane)
@@ -550,11 +562,18 @@ int setup_device(fftstencil_plan* p) {
   } else if (hp.ndim == 2) {
     // double-buffered prefetch pays only where it does not cost occupancy (profiles/r01_variants.txt)
     p->variant = hp.L[0] >= 56 ? 1 : 0;
+    if (hp.algo == 2) {
+      const size_t sb = (size_t)hp.pairs * 2 * hp.L[0] * hp.L[0] * sizeof(double);
+      e = cudaMalloc((void**)&p->dSpec, sb);
+      if (e != cudaSuccess) return cuda_fail(e, "unfused spectrum buffer");
+      p->device_bytes += sb;
+    }
     if (const char* v = std::getenv("FFTSTENCIL_VARIANT")) p->variant = std::atoi(v);
     if (p->variant < 0 || p->variant > 2) {
       set_error("FFTSTENCIL_VARIANT must be 0, 1 or 2");
       return FFTSTENCIL_EINVAL;
     }
+    if (hp.algo == 2) p->variant = 0;   // the unfused stages use the V = 0 layout
     e = fused2d_configure(hp.L[0], p->variant, &occ);
     if (e != cudaSuccess) return cuda_fail(e, "fused 2D kernel configuration");
   } else if (hp.ndim == 3 && hp.algo == 1) {

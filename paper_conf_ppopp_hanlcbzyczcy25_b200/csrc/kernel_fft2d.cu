@@ -24,7 +24,17 @@
 //          while the inverse half (M3/M4) of the current pair runs; F in shared memory
 //   V = 2  as V = 1 but F is read through L1 (column-permuted copy in HBM), so a CTA's
 //          shared memory is just the two pair buffers (more CTAs per SM)
+// Stages (template ST, the UNFUSED ablation of NEXT-3 / PAPER.md Fig. 2 left and Fig. 7):
+//   ST = 0  the fused pass above
+//   ST = 1  load + forward DFT only; the spectrum goes to HBM (a.spec, [pair][re|im][k0][k1])
+//   ST = 2  reads the spectrum back from HBM, inverse DFT + crop + store only
+// with spec_mul_kernel in between: three kernels and two spectrum round trips per pass,
+// the "standard FFT stencil" structure Kernel Tailoring removes.
+#include <algorithm>
+
 #include "device_common.cuh"
+
+#pragma nv_diag_suppress 128   // ST = 1 leaves the inverse half unreachable by design
 #include "kernels.cuh"
 
 namespace fstencil {
@@ -74,7 +84,7 @@ __device__ __forceinline__ double ldF(const double* p) {
   return *p;
 }
 
-template <int L, int V>
+template <int L, int V, int ST = 0>
 __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
   constexpr int NT = L / 8;      // 8x8 tiles per side == warps
   constexpr int LD = L + 4;      // padded row stride (doubles): 8-bank shift per row
@@ -114,6 +124,17 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
   for (int64_t p = a.win.p_begin + blockIdx.x; p < a.win.p_end; p += gridDim.x) {
     double* sXa = sbuf + cur * 2 * L * LD;   // tile 2p (real part) ... later Q' real part
     double* sXb = sXa + L * LD;              // tile 2p+1 (imag part) ... later Q' imag part
+    if (ST == 2) {
+      // ---- unfused inverse stage: the multiplied spectrum comes back from HBM ----
+      __syncthreads();
+      const double* sp = a.spec + (size_t)p * 2 * L * L;
+      for (int e = tid; e < L * L; e += NTHR) {
+        const int k0 = e / L, k1 = e - k0 * L;
+        sXa[k0 * LD + perm8(k1)] = sp[e];
+        sXb[k0 * LD + perm8(k1)] = sp[L * L + e];
+      }
+      __syncthreads();
+    } else {
     if (!DB) {
       __syncthreads();
       load_pair<L, false>(sXa, sXb, a, p, tid);
@@ -163,6 +184,17 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
         }
       }
     }
+    if (ST == 1) {
+      // ---- unfused forward stage: the spectrum goes to HBM ----
+      double* sp = a.spec + (size_t)p * 2 * L * L;
+#pragma unroll
+      for (int mt = 0; mt < NT; ++mt) {
+        const int k0 = 8 * mt + g, k1 = 8 * warp + 2 * q;
+        *reinterpret_cast<double2*>(sp + k0 * L + k1) = make_double2(Qr[mt][0], Qr[mt][1]);
+        *reinterpret_cast<double2*>(sp + L * L + k0 * L + k1) = make_double2(Qi[mt][0], Qi[mt][1]);
+      }
+      continue;
+    }
     // ---- pointwise multiply by the powered spectrum (Eq. 10) in the C fragments ----
 #pragma unroll
     for (int mt = 0; mt < NT; ++mt) {
@@ -185,6 +217,7 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
         sXb[idx] = Qi[mt][j];
       }
     __syncthreads();
+    }   // ST != 2
     // ---- prefetch the next pair into the other buffer while the inverse half runs ----
     if (DB) {
       const int64_t pn = p + gridDim.x;
@@ -275,6 +308,20 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
   }
 }
 
+__global__ void spec_mul_kernel(double* spec, int64_t npairs, int vol, const double* __restrict__ Sre,
+                                const double* __restrict__ Sim) {
+  const int64_t total = npairs * vol;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t pr = i / vol;
+    const int k = (int)(i - pr * vol);
+    double* re = spec + pr * 2 * vol + k;
+    double* im = re + vol;
+    const double a = *re, b = *im, sr = __ldg(Sre + k), si = __ldg(Sim + k);
+    *re = a * sr - b * si;
+    *im = a * si + b * sr;
+  }
+}
+
 template <int L, int V>
 cudaError_t configure_LV(int* max_blocks) {
   const size_t smem = fused2d_smem(L, V);
@@ -285,6 +332,13 @@ cudaError_t configure_LV(int* max_blocks) {
 
 template <int L>
 cudaError_t configure_L(int V, int* max_blocks) {
+  if (V == 0) {   // the unfused stages share the V = 0 footprint
+    const size_t smem = fused2d_smem(L, 0);
+    cudaError_t e = cudaFuncSetAttribute(fft2d_kernel<L, 0, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(fft2d_kernel<L, 0, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+  }
   switch (V) {
     case 0: return configure_LV<L, 0>(max_blocks);
     case 1: return configure_LV<L, 1>(max_blocks);
@@ -325,6 +379,27 @@ cudaError_t fused2d_configure(int L, int V, int* max_blocks) {
     case 64: return configure_L<64>(V, max_blocks);
     default: return cudaErrorInvalidValue;
   }
+}
+
+cudaError_t launch_unfused2d(int L, int stage, const Fft2dArgs& a, int grid, cudaStream_t s) {
+  const size_t smem = fused2d_smem(L, 0);
+  switch (L * 10 + stage) {
+#define FS_CASE(LL)                                                                  \
+  case LL * 10 + 1: fft2d_kernel<LL, 0, 1><<<grid, LL * 4, smem, s>>>(a); break; \
+  case LL * 10 + 2: fft2d_kernel<LL, 0, 2><<<grid, LL * 4, smem, s>>>(a); break;
+    FS_CASE(16) FS_CASE(24) FS_CASE(32) FS_CASE(40) FS_CASE(48) FS_CASE(56) FS_CASE(64)
+#undef FS_CASE
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_spec_mul(double* spec, int64_t npairs, int L, const double* Sre, const double* Sim,
+                            cudaStream_t s) {
+  const int64_t total = npairs * L * L;
+  const int grid = (int)std::min<int64_t>((total + 255) / 256, 148 * 16);
+  spec_mul_kernel<<<grid, 256, 0, s>>>(spec, npairs, L * L, Sre, Sim);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_fused2d(int L, int V, const Fft2dArgs& a, int grid, cudaStream_t s) {

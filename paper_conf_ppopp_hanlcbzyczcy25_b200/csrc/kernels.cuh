@@ -53,6 +53,7 @@ struct Fft2dArgs {
   const double* Fim;
   const double* Sre;     // L x L powered spectrum of this pass, natural row-major
   const double* Sim;
+  double* spec;          // unfused ablation only: [pair][re|im][k0][k1] spectrum in HBM
 };
 
 // One fused pass of the 1D prime-factor path (kernel_fft1d.cu).
@@ -119,6 +120,10 @@ int fused2d_threads(int L);
 size_t fused2d_smem(int L, int V);
 cudaError_t fused2d_configure(int L, int V, int* max_blocks_per_sm);
 cudaError_t launch_fused2d(int L, int V, const Fft2dArgs& a, int grid, cudaStream_t s);
+// Unfused ablation (NEXT-3): stage 1 = forward DFT -> a.spec, stage 2 = a.spec -> inverse + store,
+// launch_spec_mul in between (spectrum *= S_t in HBM).
+cudaError_t launch_unfused2d(int L, int stage, const Fft2dArgs& a, int grid, cudaStream_t s);
+cudaError_t launch_spec_mul(double* spec, int64_t npairs, int L, const double* Sre, const double* Sim, cudaStream_t s);
 
 // Factored-DFT 2D kernel (kernel_fft2d_ct.cu): L = 64 = 8 x 8 Cooley-Tukey per axis.
 // Fre/Fim = [F8 (8x8) | twiddles w64^(ka lb) (8x8)]; Sre/Sim = S_T in [k1][8 g + c] order with

@@ -175,7 +175,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         const int h = radius * t;
         if (h > hmax_grid) break;
         for (int al = 0; al < 2; ++al) {
-          if (algo >= 0 && al != algo) continue;
+          if (algo >= 0 && al != (algo == 2 ? 0 : algo)) continue;   // 2 = unfused: dense geometry
           for (int L : cand) {
             if (al == 1 && L != 64) continue;
             const int S = L - 2 * h;
@@ -187,13 +187,14 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       }
     }
     if (bL == 0) { err = "no 2D tile fits this radius/grid"; return FFTSTENCIL_EINVAL; }
-    p.algo = bA;
+    p.algo = algo == 2 ? 2 : bA;
+    if (p.algo == 2 && nranks > 1) { err = "the unfused ablation is single-GPU"; return FFTSTENCIL_EUNSUPPORTED; }
     p.T = bT;
     p.h = radius * bT;
     p.L[0] = p.L[1] = bL;
     p.S[0] = p.S[1] = bL - 2 * p.h;
     const double L = bL, S = p.S[0];
-    if (bA == 0) {
+    if (bA == 0) {   // dense (and the unfused ablation, same GEMMs)
       p.flops_per_cell_step = (16.0 * L * L * L + 6.0 * L * L + 8.0 * S * L * L + 8.0 * S * S * L) / (2.0 * S * S * bT);
       const double Sp = round8(p.S[0]);
       p.mma_flops_per_pair = 8.0 * (2.0 * L * L * L + Sp * L * L + Sp * Sp * L);

@@ -37,7 +37,7 @@ struct HostPlan {
   int L[3] = {1, 1, 1};            // tile extent per user axis
   int S[3] = {1, 1, 1};            // valid extent per user axis
   int N1 = 0, N2 = 0;              // 1D prime-factor split
-  int algo = 0;                    // 2D: 0 = dense L x L DFT GEMMs, 1 = factored 64 = 8 x 8 (CT)
+  int algo = 0;                    // 0 dense DFT GEMMs, 1 factored (2D CT 8x8, 3D 8x2), 2 unfused 2D ablation
   int periodic = 0;                // 1: periodic boundary (no ring/band, wrap-around tiles)
   int64_t nt[3] = {1, 1, 1};       // tiles per user axis
   int64_t tiles = 0, pairs = 0;

@@ -103,6 +103,18 @@ def test_band_kernels_agree(fs, monkeypatch, ext, shape, r, T, steps, kind):
     assert np.array_equal(fast, ref)
 
 
+@pytest.mark.parametrize("ext,shape,r,T,steps,kind", [c for c in CASES if len(c[0]) == 2][::2])
+def test_parity_unfused_ablation(fs, monkeypatch, ext, shape, r, T, steps, kind):
+    """NEXT-3: the unfused three-kernel pass (spectrum through HBM) computes the same result."""
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "unfused")
+    w = wl.stencil_weights(shape, 2, r, kind)
+    u0 = wl.grid(ext, 29)
+    got, p = run_gpu(fs, u0, w, r, T, steps)
+    assert p.info()["algo"] == "unfused"
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(got, ref) <= TOL
+
+
 @pytest.mark.parametrize("ext,r,T,steps", [((96, 90), 1, 4, 8), ((96, 90), 1, 4, 12), ((500,), 1, 8, 16),
                                            ((500,), 1, 8, 24)])
 def test_in_place_aliasing(fs, ext, r, T, steps):
