@@ -40,6 +40,7 @@ __device__ __forceinline__ void cgemm8(const double (&ar)[2], const double (&ai)
   }
 }
 
+template <bool WRAP>   // periodic boundary: a separate instantiation (no wrap arithmetic otherwise)
 __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const Fft1dArgs a) {
   const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
   const int64_t warp = a.win.p_begin + (int64_t)blockIdx.x * kFft1dWarpsPerBlock + (threadIdx.x >> 5);
@@ -73,7 +74,7 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
       xi[j] = 0.0;
       if (pos[j] >= 0) {
         int64_t xa = oa + pos[j], xb = ob + pos[j];
-        if (a.bd.wrap) { xa = wrap_index(xa, a.n); xb = wrap_index(xb, a.n); }
+        if (WRAP) { xa = wrap_index(xa, a.n); xb = wrap_index(xb, a.n); }
         if (xa >= 0 && xa < a.n && xa >= g0 && xa < g1) xr[j] = __ldg(a.src + (xa - g0));
         if (has_b && xb >= 0 && xb < a.n && xb >= g0 && xb < g1) xi[j] = __ldg(a.src + (xb - g0));
       }
@@ -106,11 +107,14 @@ __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const F
 }  // namespace
 
 cudaError_t fused1d_configure(int* max_blocks) {
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft1d_kernel, kFft1dWarpsPerBlock * 32, 0);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft1d_kernel<false>, kFft1dWarpsPerBlock * 32, 0);
 }
 
 cudaError_t launch_fused1d(const Fft1dArgs& a, int grid, cudaStream_t s) {
-  fft1d_kernel<<<grid, kFft1dWarpsPerBlock * 32, 0, s>>>(a);
+  if (a.bd.wrap)
+    fft1d_kernel<true><<<grid, kFft1dWarpsPerBlock * 32, 0, s>>>(a);
+  else
+    fft1d_kernel<false><<<grid, kFft1dWarpsPerBlock * 32, 0, s>>>(a);
   return cudaGetLastError();
 }
 

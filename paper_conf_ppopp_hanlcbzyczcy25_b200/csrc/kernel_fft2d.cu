@@ -51,7 +51,7 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
 // Pair p = tiles (t0, 2j) and (t0, 2j+1) with t0 = p / npr, j = p % npr (kernels.cuh).
-template <int L, bool ASYNC>
+template <int L, bool ASYNC, bool WRAP>
 __device__ __forceinline__ void load_pair(double* sXa, double* sXb, const Fft2dArgs& a, int64_t p, int tid) {
   constexpr int LD = L + 4, NTHR = L * 4;
   const int64_t t0 = p / a.npr, j = p - t0 * a.npr;
@@ -65,9 +65,9 @@ __device__ __forceinline__ void load_pair(double* sXa, double* sXb, const Fft2dA
     for (int e = tid; e < L * L; e += NTHR) {
       const int r = e / L, c = e - r * L;
       int64_t gr = o0 + r, gc = o1 + c;
-      if (a.bd.wrap) { gr = wrap_index(gr, a.n0); gc = wrap_index(gc, a.n1); }
+      if (WRAP) { gr = wrap_index(gr, a.n0); gc = wrap_index(gc, a.n1); }
       const int64_t lr = gr - a.win.g0;
-      const bool valid = have && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc >= 0 && gc < a.n1;
+      const bool valid = have && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc < a.n1;   // gc >= 0 always
       double* dst = sX + r * LD + perm8(c);
       if (ASYNC) {
         cp_async8(dst, valid ? a.src + lr * a.n1 + gc : a.src, valid);
@@ -84,7 +84,9 @@ __device__ __forceinline__ double ldF(const double* p) {
   return *p;
 }
 
-template <int L, int V, int ST = 0>
+// WRAP: periodic boundary (NEXT-2), a separate instantiation so the fixed-ring kernel carries
+// no wrap-around arithmetic in its load loop.
+template <int L, int V, int ST = 0, bool WRAP = false>
 __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
   constexpr int NT = L / 8;      // 8x8 tiles per side == warps
   constexpr int LD = L + 4;      // padded row stride (doubles): 8-bank shift per row
@@ -117,7 +119,7 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
   int cur = 0;
 
   if (DB && a.win.p_begin + blockIdx.x < a.win.p_end) {
-    load_pair<L, true>(sbuf, sbuf + L * LD, a, a.win.p_begin + blockIdx.x, tid);
+    load_pair<L, true, WRAP>(sbuf, sbuf + L * LD, a, a.win.p_begin + blockIdx.x, tid);
     cp_async_commit();
     cp_async_wait_all();
   }
@@ -137,7 +139,7 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
     } else {
     if (!DB) {
       __syncthreads();
-      load_pair<L, false>(sXa, sXb, a, p, tid);
+      load_pair<L, false, WRAP>(sXa, sXb, a, p, tid);
     }
     __syncthreads();
 
@@ -223,7 +225,7 @@ __global__ void __launch_bounds__(L * 4) fft2d_kernel(const Fft2dArgs a) {
       const int64_t pn = p + gridDim.x;
       if (pn < a.win.p_end) {
         double* nb = sbuf + (cur ^ 1) * 2 * L * LD;
-        load_pair<L, true>(nb, nb + L * LD, a, pn, tid);
+        load_pair<L, true, WRAP>(nb, nb + L * LD, a, pn, tid);
       }
       cp_async_commit();
     }
@@ -332,9 +334,11 @@ cudaError_t configure_LV(int* max_blocks) {
 
 template <int L>
 cudaError_t configure_L(int V, int* max_blocks) {
-  if (V == 0) {   // the unfused stages share the V = 0 footprint
+  {   // the unfused stages and the periodic instantiation share the V = 0 footprint
     const size_t smem = fused2d_smem(L, 0);
     cudaError_t e = cudaFuncSetAttribute(fft2d_kernel<L, 0, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(fft2d_kernel<L, 0, 0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(fft2d_kernel<L, 0, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -350,6 +354,10 @@ cudaError_t configure_L(int V, int* max_blocks) {
 template <int L>
 void launch_L(int V, const Fft2dArgs& a, int grid, cudaStream_t s) {
   const size_t smem = fused2d_smem(L, V);
+  if (a.bd.wrap) {   // periodic plans run the V = 0 structure
+    fft2d_kernel<L, 0, 0, true><<<grid, L * 4, fused2d_smem(L, 0), s>>>(a);
+    return;
+  }
   switch (V) {
     case 0: fft2d_kernel<L, 0><<<grid, L * 4, smem, s>>>(a); break;
     case 1: fft2d_kernel<L, 1><<<grid, L * 4, smem, s>>>(a); break;

@@ -153,7 +153,7 @@ __device__ __forceinline__ void twiddle_n(double (&cr)[NL][2], double (&ci)[NL][
 // TMA = true: each tile arrives by one 64 x 64 TMA box (OOB -> 0) in a dense row-major
 // layout; phase 1 reads its rows there (4-way bank conflicts on that pass only) and, the
 // XOR swizzle being a permutation within a row, rewrites each row in place swizzled.
-template <int NW, int NL, bool TMA>
+template <int NW, int NL, bool TMA, bool WRAP = false>   // WRAP: periodic (cp.async path only)
 __global__ void __launch_bounds__(NW * 32, NL > 2 ? 2 : 3)
     fft2d_ct_kernel(const Fft2dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ __align__(128) double smem[];
@@ -227,7 +227,7 @@ __global__ void __launch_bounds__(NW * 32, NL > 2 ? 2 : 3)
     for (int e = tid; e < 2 * L * L; e += NW * 32) {
       const int t = e >> 12, r = (e >> 6) & 63, c = e & 63;
       int64_t gr = o0 + r, gc = (t ? ob1 : oa1) + c;
-      if (a.bd.wrap) { gr = wrap_index(gr, a.n0); gc = wrap_index(gc, a.n1); }
+      if (WRAP) { gr = wrap_index(gr, a.n0); gc = wrap_index(gc, a.n1); }
       const int64_t lr = gr - a.win.g0;
       const bool valid = (t == 0 || has_b) && gr < a.n0 && lr >= 0 && lr < a.win.gn && gc >= 0 && gc < a.n1;
       cp_async8((t ? sI : sR) + sw(r, c), valid ? a.src + lr * a.n1 + gc : a.src, valid);
@@ -353,7 +353,9 @@ size_t fused2d_ct_smem() { return (size_t)2 * PLANE * sizeof(double); }
 cudaError_t fused2d_ct_configure(int cfg, int* max_blocks) {
   switch (cfg) {
     case 81: {
-      cudaError_t e = configure_nw<8, 1, true>(max_blocks);
+      cudaError_t e = cudaFuncSetAttribute(fft2d_ct_kernel<8, 1, false, true>,
+                                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fused2d_ct_smem());
+      if (e == cudaSuccess) e = configure_nw<8, 1, true>(max_blocks);
       return e != cudaSuccess ? e : configure_nw<8, 1, false>(max_blocks);
     }
     case 82: {
@@ -374,7 +376,9 @@ cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, const CUtensorMap* tm
   const size_t smem = fused2d_ct_smem();
   static const CUtensorMap none = {};
   const CUtensorMap& m = tm ? *tm : none;
-  if (tm && cfg == 81) {
+  if (a.bd.wrap) {   // periodic: cp.async loads with wrap-around (single instantiation)
+    fft2d_ct_kernel<8, 1, false, true><<<grid, 256, smem, s>>>(a, m);
+  } else if (tm && cfg == 81) {
     fft2d_ct_kernel<8, 1, true><<<grid, 256, smem, s>>>(a, m);
   } else if (tm && cfg == 82) {
     fft2d_ct_kernel<8, 2, true><<<grid, 256, smem, s>>>(a, m);

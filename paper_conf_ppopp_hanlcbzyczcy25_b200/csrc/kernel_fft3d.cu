@@ -41,6 +41,7 @@ __device__ __forceinline__ void cmma(double (&cr)[2], double (&ci)[2], double ar
   }
 }
 
+template <bool WRAP>   // periodic boundary: a separate instantiation
 __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
   extern __shared__ __align__(16) double smem[];
   double* sFr = smem;
@@ -75,7 +76,7 @@ __global__ void __launch_bounds__(NW3 * 32) fft3d_kernel(const Fft3dArgs a) {
         double v = 0.0;
         if (have) {
           int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = o2 + l2;
-          if (a.bd.wrap) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
+          if (WRAP) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
           const int64_t lg0 = g0 - a.win.g0;
           if (g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 && g1 < a.n1 && g2 >= 0 && g2 < a.n2)
             v = __ldg(a.src + (lg0 * a.n1 + g1) * a.n2 + g2);
@@ -284,13 +285,17 @@ size_t fused3d_smem() { return (size_t)(2 * L * LD + 2 * L * SL) * sizeof(double
 
 cudaError_t fused3d_configure(int* max_blocks) {
   const size_t smem = fused3d_smem();
-  cudaError_t e = cudaFuncSetAttribute(fft3d_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(fft3d_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(fft3d_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_kernel, NW3 * 32, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_kernel<false>, NW3 * 32, smem);
 }
 
 cudaError_t launch_fused3d(const Fft3dArgs& a, int grid, cudaStream_t s) {
-  fft3d_kernel<<<grid, NW3 * 32, fused3d_smem(), s>>>(a);
+  if (a.bd.wrap)
+    fft3d_kernel<true><<<grid, NW3 * 32, fused3d_smem(), s>>>(a);
+  else
+    fft3d_kernel<false><<<grid, NW3 * 32, fused3d_smem(), s>>>(a);
   return cudaGetLastError();
 }
 

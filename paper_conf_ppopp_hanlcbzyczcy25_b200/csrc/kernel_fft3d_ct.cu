@@ -147,7 +147,7 @@ __device__ __forceinline__ void inv_group(double* sR, double* sI, const LN& ln, 
   }
 }
 
-template <bool TMA>
+template <bool TMA, bool WRAP = false>   // WRAP: periodic boundary (cp.async path only)
 __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ __align__(128) double smem[];
   double* sR = smem;
@@ -193,7 +193,7 @@ __global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a
       for (int e = tid; e < 2 * PLANE; e += NWC * 32) {
         const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
         int64_t g0 = o0 + l0, g1 = o1 + l1, g2 = (t ? ob2 : oa2) + l2;
-        if (a.bd.wrap) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
+        if (WRAP) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
         const int64_t lg0 = g0 - a.win.g0;
         const bool valid = (t == 0 || has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 && g1 < a.n1 &&
                            g2 >= 0 && g2 < a.n2;
@@ -271,6 +271,8 @@ cudaError_t fused3d_ct_configure(int* max_blocks) {
   cudaError_t e = cudaFuncSetAttribute(fft3d_ct_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(fft3d_ct_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft3d_ct_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_ct_kernel<true>, NWC * 32, smem);
 }
@@ -279,6 +281,8 @@ cudaError_t launch_fused3d_ct(const Fft3dArgs& a, const CUtensorMap* tm, int gri
   static const CUtensorMap none = {};
   if (tm)
     fft3d_ct_kernel<true><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a, *tm);
+  else if (a.bd.wrap)
+    fft3d_ct_kernel<false, true><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a, none);
   else
     fft3d_ct_kernel<false><<<grid, NWC * 32, fused3d_ct_smem(), s>>>(a, none);
   return cudaGetLastError();

@@ -114,6 +114,10 @@ CONFIGS = {
                        notes="configs[3]"),
     "box3d27p": Workload(6, "Box-3D27P", "box", 3, 1, (1024, 1024, 1024), 0, 100,
                          notes="configs[3]"),
+    # PAPER.md Table 3's 1D sizes (512M = 2^29 cells, reading Q16) for a meaningful 1D roofline
+    "heat1d_512m": Workload(9, "Heat-1D 512M", "star", 1, 1, (1 << 29,), 0, 1000, notes="Table 3 L332"),
+    "1d5p_512m": Workload(10, "1D5P 512M", "star", 1, 2, (1 << 29,), 0, 1000, notes="Table 3 L333"),
+    "1d7p_512m": Workload(11, "1D7P 512M", "star", 1, 3, (1 << 29,), 0, 1000, notes="Table 3 L334"),
     "box2d9p_weak": Workload(7, "Box-2D9P weak", "box", 2, 1, (5120, 40960), 0, 1000,
                              notes="configs[4]: per-GPU slab; global (5120 g) x 40960"),
     "heat3d_weak": Workload(8, "Heat-3D weak", "star", 3, 1, (256, 1024, 1024), 0, 100,
