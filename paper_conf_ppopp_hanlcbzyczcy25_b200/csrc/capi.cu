@@ -77,6 +77,12 @@ struct fftstencil_plan {
   ncclComm_t comm = nullptr;
   cudaStream_t comm_stream = nullptr;
   cudaEvent_t ev_ready = nullptr, ev_xchg = nullptr;
+  // ---- the band kernel runs on a side stream, concurrent with the fused kernel (it reads
+  // the same source and writes disjoint cells); FFTSTENCIL_BAND_STREAM=0 serialises it ----
+  bool band_concurrent = true;
+  cudaStream_t band_stream = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_band = nullptr;
+  bool band_pending = false;
   double* dE[2] = {nullptr, nullptr};   // slab + halo buffers, rows [g0, g1)
   int ecur = 0;               // index of the buffer holding the current state
   // ---- profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run() ----
@@ -136,6 +142,9 @@ void free_plan(fftstencil_plan* p) {
   if (p->comm_stream) cudaStreamDestroy(p->comm_stream);
   if (p->ev_ready) cudaEventDestroy(p->ev_ready);
   if (p->ev_xchg) cudaEventDestroy(p->ev_xchg);
+  if (p->band_stream) cudaStreamDestroy(p->band_stream);
+  if (p->ev_fork) cudaEventDestroy(p->ev_fork);
+  if (p->ev_band) cudaEventDestroy(p->ev_band);
   for (cudaEvent_t ev : p->ev_pool) cudaEventDestroy(ev);
   cudaFree(p->dF);
   cudaFree(p->dS);
@@ -319,6 +328,9 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
   return FFTSTENCIL_OK;
 }
 
+// The band pass of one fused pass.  Concurrent mode: forked from `s` (after everything
+// already enqueued there, i.e. after the pass that produced `src`) onto the band stream;
+// band_join() makes `s` wait for it before the next pass touches either buffer.
 int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s) {
   const HostPlan& hp = p->hp;
   const int nb = (int)(hp.band_blocks.size() / 8);
@@ -336,12 +348,30 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
   b.g0 = hp.g0;
   b.gn = hp.g1 - hp.g0;
   b.reference = p->band_reference;
-  const long pb = prof_begin(p, 1, s);
-  cudaError_t e = launch_band(b, p->band_smem, s);
-  prof_end(p, pb, s);
+  cudaStream_t bs = s;
+  if (p->band_concurrent) {
+    cudaError_t e = cudaEventRecord(p->ev_fork, s);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(p->band_stream, p->ev_fork, 0);
+    if (e != cudaSuccess) return cuda_fail(e, "band fork");
+    bs = p->band_stream;
+  }
+  const long pb = prof_begin(p, 1, bs);
+  cudaError_t e = launch_band(b, p->band_smem, bs);
+  prof_end(p, pb, bs);
   if (e != cudaSuccess) return cuda_fail(e, "band launch");
+  if (p->band_concurrent) {
+    if ((e = cudaEventRecord(p->ev_band, bs)) != cudaSuccess) return cuda_fail(e, "band event");
+    p->band_pending = true;
+  }
   ++p->last_launches;
   return FFTSTENCIL_OK;
+}
+
+int band_join(fftstencil_plan* p, cudaStream_t s) {
+  if (!p->band_pending) return FFTSTENCIL_OK;
+  p->band_pending = false;
+  cudaError_t e = cudaStreamWaitEvent(s, p->ev_band, 0);
+  return e == cudaSuccess ? FFTSTENCIL_OK : cuda_fail(e, "band join");
 }
 
 // Copy the (rank's) fixed ring from src (buffer rows start at global row src_off) into
@@ -397,8 +427,9 @@ int run_single(fftstencil_plan* p, const double* in, double* out, int64_t total_
   for (int64_t i = 0; i < passes; ++i) {
     const int t = i < nfull ? T : rem;
     double* dst = dsts[i % 2];
+    if ((rc = launch_band_pass(p, src, dst, t, s))) return rc;   // forked: overlaps the fused kernel
     if ((rc = launch_fused(p, src, dst, t, p->hp.pair_lo, p->hp.pair_hi, s))) return rc;
-    if ((rc = launch_band_pass(p, src, dst, t, s))) return rc;
+    if ((rc = band_join(p, s))) return rc;
     src = dst;
   }
   if (final_copy) {
@@ -473,6 +504,7 @@ int dist_pass(fftstencil_plan* p, int t, bool xchg, cudaStream_t s) {
   if ((rc = launch_fused(p, src, dst, t, hp.pair_lo, hp.ipair_lo, s))) return rc;
   if ((rc = launch_fused(p, src, dst, t, hp.ipair_hi, hp.pair_hi, s))) return rc;
   if ((rc = launch_band_pass(p, src, dst, t, s))) return rc;
+  if ((rc = band_join(p, s))) return rc;
   p->ecur ^= 1;
   return FFTSTENCIL_OK;
 }
@@ -593,6 +625,14 @@ int setup_device(fftstencil_plan* p) {
   }
   p->fused_grid = (int)std::max<int64_t>(1, (int64_t)p->sm_count * occ);
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
+  if (const char* v = std::getenv("FFTSTENCIL_BAND_STREAM")) p->band_concurrent = std::atoi(v) != 0;
+  if (hp.band_blocks.empty()) p->band_concurrent = false;
+  if (p->band_concurrent) {
+    e = cudaStreamCreateWithFlags(&p->band_stream, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->ev_band, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_fail(e, "band stream/events");
+  }
   p->band_smem = (size_t)2 * hp.band_region_cells * sizeof(double);
   if (p->band_smem > 0) {
     e = band_configure(p->band_smem);

@@ -89,7 +89,8 @@ __global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
 // without per-cell divisions.  Same definition and result as band_kernel.
 constexpr int kMaxTaps = 512;
 
-__global__ void __launch_bounds__(kBandThreads) band_cone_kernel(const BandArgs a) {
+// (256, 6): at most 40 registers, so one band CTA fits beside three fused CTAs on an SM
+__global__ void __launch_bounds__(kBandThreads, 6) band_cone_kernel(const BandArgs a) {
   extern __shared__ double sb[];
   __shared__ int s_off[kMaxTaps];
   __shared__ double s_w[kMaxTaps];
@@ -141,29 +142,44 @@ __global__ void __launch_bounds__(kBandThreads) band_cone_kernel(const BandArgs 
   }
   __syncthreads();
   const int ntaps = s_ntaps;
+  // fixed-ring bounds in region-local coordinates (inactive axes never hit)
+  int rlo[3], rhi[3];
+#pragma unroll
+  for (int q = 0; q < 3; ++q) {
+    rlo[q] = a.active[q] ? (int)(r - rl[q]) : -(1 << 30);
+    rhi[q] = a.active[q] ? (int)(a.n[q] - r - rl[q]) : (1 << 30);
+  }
   for (int s = 1; s <= a.t; ++s) {
 #pragma unroll
     for (int q = 0; q < 3; ++q) {
       clo[q] = open_lo[q] ? r * s : 0;
       chi[q] = D[q] - (open_hi[q] ? r * s : 0);
     }
-    // cone box of this step, flattened over all threads (no idle lanes on narrow faces)
+    // cone box of this step, flattened over all threads (no idle lanes on narrow faces);
+    // the (k0, k1, k2) decomposition is advanced by carries, not recomputed by divisions
     const int W0 = chi[0] - clo[0], W1 = chi[1] - clo[1], W2 = chi[2] - clo[2];
-    const int ncone = W0 * W1 * W2;
+    const int W12 = W1 * W2, ncone = W0 * W12;
+    int k0 = threadIdx.x / W12, k1 = (threadIdx.x - k0 * W12) / W2;
+    int k2 = threadIdx.x - k0 * W12 - k1 * W2;
+    const int d0 = kBandThreads / W12, d1 = (kBandThreads - d0 * W12) / W2;
+    const int d2 = kBandThreads - d0 * W12 - d1 * W2;
     for (int f = threadIdx.x; f < ncone; f += kBandThreads) {
-      const int k2 = f % W2, k01 = f / W2, k1 = k01 % W1, k0 = k01 / W1;
       const int i0 = clo[0] + k0, i1 = clo[1] + k1, i2 = clo[2] + k2;
       const int e = (i0 * D[1] + i1) * D[2] + i2;
-      const int64_t c0 = rl[0] + i0, c1 = rl[1] + i1, c2 = rl[2] + i2;
       double v;
-      if ((a.active[0] && (c0 < r || c0 >= a.n[0] - r)) || (a.active[1] && (c1 < r || c1 >= a.n[1] - r)) ||
-          (a.active[2] && (c2 < r || c2 >= a.n[2] - r))) {
+      if (i0 < rlo[0] || i0 >= rhi[0] || i1 < rlo[1] || i1 >= rhi[1] || i2 < rlo[2] || i2 >= rhi[2]) {
         v = b0[e];                                          // fixed ring
       } else {
         v = 0.0;
+#pragma unroll 4
         for (int k = 0; k < ntaps; ++k) v = fma(s_w[k], b0[e + s_off[k]], v);
       }
       b1[e] = v;
+      k2 += d2;
+      k1 += d1;
+      k0 += d0;
+      if (k2 >= W2) { k2 -= W2; ++k1; }
+      if (k1 >= W1) { k1 -= W1; ++k0; }
     }
     __syncthreads();
     double* t = b0; b0 = b1; b1 = t;

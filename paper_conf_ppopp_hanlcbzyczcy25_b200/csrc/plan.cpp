@@ -443,7 +443,9 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   }
   // Split each band box into CTA blocks whose input region (block + r*T on every
   // active side) fits the band kernel's shared-memory budget (2 buffers of FP64).
-  const int budget_cells = (96 * 1024) / 16;
+  // 24 KB of FP64 pairs: small enough to co-reside with three 64 KB fused CTAs per SM (the
+  // band runs concurrently on its own stream, capi.cu)
+  const int budget_cells = 1536;
   const int grow = 2 * r * p.T;
   for (const Box& b : p.band_boxes) {
     int64_t len[3], blk[3];
