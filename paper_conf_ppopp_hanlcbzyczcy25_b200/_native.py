@@ -70,7 +70,7 @@ class Info(ctypes.Structure):
             "nranks": self.nranks, "rank": self.rank, "row_begin": self.row_begin, "row_end": self.row_end,
             "pair_begin": self.pair_begin, "pair_end": self.pair_end, "interior_begin": self.interior_begin,
             "interior_end": self.interior_end, "ghost_lo": self.ghost_lo, "ghost_hi": self.ghost_hi,
-            "algo": ("dense", "factored", "unfused")[self.algo] if nd >= 2 else "pfa",
+            "algo": ("dense", "factored", "unfused")[self.algo] if nd >= 2 else ("pfa", "factored")[self.algo],
             "periodic": bool(self.periodic),
         }
 

@@ -291,8 +291,13 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Sre = Sre;
     a.Sim = Sim;
     a.crt = p->dCrt;
-    const int64_t blocks = (np + kFft1dWarpsPerBlock - 1) / kFft1dWarpsPerBlock;
-    e = launch_fused1d(a, (int)std::max<int64_t>(1, std::min<int64_t>(p->fused_grid, blocks)), s);
+    a.tw = p->dF + 256;
+    if (hp.algo == 1) {
+      e = launch_fused1d_ct(a, (int)std::min<int64_t>(p->fused_grid, np), s);
+    } else {
+      const int64_t blocks = (np + kFft1dWarpsPerBlock - 1) / kFft1dWarpsPerBlock;
+      e = launch_fused1d(a, (int)std::max<int64_t>(1, std::min<int64_t>(p->fused_grid, blocks)), s);
+    }
   } else {
     Fft3dArgs a;
     a.src = src;
@@ -542,6 +547,7 @@ int setup_device(fftstencil_plan* p) {
   size_t acc = 0;
   std::vector<double> F(hp.Fre);
   F.insert(F.end(), hp.Fim.begin(), hp.Fim.end());
+  F.insert(F.end(), hp.tw.begin(), hp.tw.end());   // factored 1D: [Fre 128 | Fim 128 | w4096]
   if (hp.ndim == 2 && (hp.algo == 0 || hp.algo == 2)) {
     // the dense 2D kernel reads F with columns permuted within groups of 8 (device_common.cuh)
     const int L = hp.L[0];
@@ -615,6 +621,9 @@ int setup_device(fftstencil_plan* p) {
   } else if (hp.ndim == 3) {
     e = fused3d_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "fused 3D kernel configuration");
+  } else if (hp.algo == 1) {
+    e = fused1d_ct_configure(&occ);
+    if (e != cudaSuccess) return cuda_fail(e, "factored 1D kernel configuration");
   } else {
     e = fused1d_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "fused 1D kernel configuration");
@@ -709,7 +718,18 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
   std::vector<double> v;
   if (which == 0) {
     int L, row0 = 0, ld;
-    if (hp.ndim == 1) {
+    if (hp.ndim == 1 && hp.algo == 1) {
+      // factored 1D: axis 0 = F_8, 1 = twiddles w64^(ka lb) (8 x 8), 2 = w4096^(a c) (64 x 64)
+      if (axis < 0 || axis > 2) { set_error("axis must be 0 (F_8), 1 (w64) or 2 (w4096)"); return FFTSTENCIL_EINVAL; }
+      if (axis == 2) {
+        v.assign(hp.tw.begin(), hp.tw.end());
+        L = 0;
+      } else {
+        L = 8;
+      }
+      row0 = 8 * (axis & 1);
+      ld = 8;
+    } else if (hp.ndim == 1) {
       if (axis < 0 || axis > 1) { set_error("axis must be 0 (N1) or 1 (N2) for 1D"); return FFTSTENCIL_EINVAL; }
       L = axis == 0 ? hp.N1 : hp.N2;
       row0 = axis == 0 ? 0 : 8;
@@ -758,7 +778,7 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
       }
     }
   } else if (which == 3) {
-    if (hp.ndim != 1) { set_error("the PFA map exists for 1D plans only"); return FFTSTENCIL_EINVAL; }
+    if (hp.ndim != 1 || hp.crt.empty()) { set_error("the PFA map exists for 1D prime-factor plans only"); return FFTSTENCIL_EINVAL; }
     for (int l1 = 0; l1 < hp.N1; ++l1)
       for (int l2 = 0; l2 < hp.N2; ++l2) v.push_back((double)hp.crt[l1 * 8 + l2]);
   } else if (which == 4) {

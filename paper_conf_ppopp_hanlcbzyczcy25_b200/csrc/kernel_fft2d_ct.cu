@@ -25,129 +25,20 @@
 // Shared layout: plane[r][c] at r*64 + (c ^ 4(((c>>4) ^ (r>>4)) & 3) ^ (r & 3)) (XOR swizzle):
 // both the row pattern (c = 16q + 8j + g) and the column pattern (r = 16q + 8j + g) are
 // bank-conflict free per half-warp.
-#include "device_common.cuh"
+#include "ct_line.cuh"
 #include "kernels.cuh"
 #include "tma.cuh"
 
 namespace fstencil {
 namespace {
 
-using dev::dmma;
+using namespace ct;
 
-constexpr int L = 64;
 constexpr int PLANE = L * L;
-
-// XOR-swizzled dense layout: both fragment patterns (row r fixed, c = 16q + 8j + g; and
-// column c fixed, r = 16q + 8j + g) are conflict-free per half-warp (8-byte accesses are
-// served 16 lanes at a time: lanes 4g + q, g in one half), the optimal 2 wavefronts per 32
-// doubles; a permutation within each row; 64 KB for the two planes (3 CTAs / SM).
-__device__ __forceinline__ int sw(int r, int c) {
-  return r * L + (c ^ (((((c >> 4) & 3) ^ ((r >> 4) & 3))) << 2) ^ (r & 3));
-}
 
 __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
-}
-
-// B-route: C = F8 . B (F8 fragments f*, data fragments b*), CONJ -> conj(F8).
-template <bool CONJ>
-__device__ __forceinline__ void broute(double (&cr)[2], double (&ci)[2], const double (&fr)[2], const double (&fi)[2],
-                                       const double (&br)[2], const double (&bi)[2]) {
-  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
-#pragma unroll
-  for (int j = 0; j < 2; ++j) {
-    if (CONJ) {
-      dmma(cr, fr[j], br[j]);
-      dmma(ci, fr[j], bi[j]);
-      dmma(cr, fi[j], bi[j]);
-      dmma(ci, -fi[j], br[j]);
-    } else {
-      dmma(cr, fr[j], br[j]);
-      dmma(ci, fr[j], bi[j]);
-      dmma(cr, -fi[j], bi[j]);
-      dmma(ci, fi[j], br[j]);
-    }
-  }
-}
-
-// A-route: C = D . F8^T (data fragments d* as A, F8^T fragments = F8 fragments as B).
-template <bool CONJ>
-__device__ __forceinline__ void aroute(double (&cr)[2], double (&ci)[2], const double (&dr)[2], const double (&di)[2],
-                                       const double (&fr)[2], const double (&fi)[2]) {
-  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
-#pragma unroll
-  for (int j = 0; j < 2; ++j) {
-    if (CONJ) {
-      dmma(cr, dr[j], fr[j]);
-      dmma(ci, di[j], fr[j]);
-      dmma(cr, di[j], fi[j]);
-      dmma(ci, -dr[j], fi[j]);
-    } else {
-      dmma(cr, dr[j], fr[j]);
-      dmma(ci, di[j], fr[j]);
-      dmma(cr, -di[j], fi[j]);
-      dmma(ci, dr[j], fi[j]);
-    }
-  }
-}
-
-template <bool CONJ>
-__device__ __forceinline__ void twiddle(double (&cr)[2], double (&ci)[2], const double (&tr)[2], const double (&ti)[2]) {
-#pragma unroll
-  for (int j = 0; j < 2; ++j) {
-    const double t_i = CONJ ? -ti[j] : ti[j];
-    const double r = cr[j] * tr[j] - ci[j] * t_i;
-    const double i = cr[j] * t_i + ci[j] * tr[j];
-    cr[j] = r;
-    ci[j] = i;
-  }
-}
-
-// NL independent lines per warp, their DMMA chains interleaved for latency hiding.
-template <bool CONJ, int NL>
-__device__ __forceinline__ void broute_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&fr)[2],
-                                         const double (&fi)[2], const double (&br)[NL][2], const double (&bi)[NL][2]) {
-#pragma unroll
-  for (int u = 0; u < NL; ++u) cr[u][0] = cr[u][1] = ci[u][0] = ci[u][1] = 0.0;
-#pragma unroll
-  for (int j = 0; j < 2; ++j) {
-    const double nfi = CONJ ? fi[j] : -fi[j];   // coefficient of bi in cr
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(cr[u], fr[j], br[u][j]);
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(ci[u], fr[j], bi[u][j]);
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(cr[u], nfi, bi[u][j]);
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(ci[u], -nfi, br[u][j]);
-  }
-}
-
-template <bool CONJ, int NL>
-__device__ __forceinline__ void aroute_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&dr)[NL][2],
-                                         const double (&di)[NL][2], const double (&fr)[2], const double (&fi)[2]) {
-#pragma unroll
-  for (int u = 0; u < NL; ++u) cr[u][0] = cr[u][1] = ci[u][0] = ci[u][1] = 0.0;
-#pragma unroll
-  for (int j = 0; j < 2; ++j) {
-    const double nfi = CONJ ? fi[j] : -fi[j];
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(cr[u], dr[u][j], fr[j]);
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(ci[u], di[u][j], fr[j]);
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(cr[u], di[u][j], nfi);
-#pragma unroll
-    for (int u = 0; u < NL; ++u) dmma(ci[u], dr[u][j], -nfi);
-  }
-}
-
-template <bool CONJ, int NL>
-__device__ __forceinline__ void twiddle_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&tr)[2],
-                                          const double (&ti)[2]) {
-#pragma unroll
-  for (int u = 0; u < NL; ++u) twiddle<CONJ>(cr[u], ci[u], tr, ti);
 }
 
 // TMA = true: each tile arrives by one 64 x 64 TMA box (OOB -> 0) in a dense row-major

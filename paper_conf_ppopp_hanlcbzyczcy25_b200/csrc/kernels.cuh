@@ -56,12 +56,13 @@ struct Fft2dArgs {
   double* spec;          // unfused ablation only: [pair][re|im][k0][k1] spectrum in HBM
 };
 
-// One fused pass of the 1D prime-factor path (kernel_fft1d.cu).
+// One fused pass of the 1D path: prime-factor 8 x 7 tile (kernel_fft1d.cu) or the
+// factored 4096 = 64 x 64 tile (kernel_fft1d_ct.cu).
 struct Fft1dArgs {
   const double* src;
   double* dst;
   int64_t n;
-  int h, S, L;           // L = N1*N2 = 56
+  int h, S, L;           // L = N1*N2 = 56 (PFA) or 4096 (factored)
   int64_t ntiles;        // pair p holds tiles 2p and 2p+1
   Window win;
   Bound bd;
@@ -69,7 +70,8 @@ struct Fft1dArgs {
   const double* Fim;
   const double* Sre;     // 8 x 8 Ruritanian-ordered powered spectrum, zero-padded
   const double* Sim;
-  const int* crt;        // 64: tile position stored at (l1, l2), -1 = padding
+  const int* crt;        // PFA: 64 tile positions stored at (l1, l2), -1 = padding
+  const double* tw;      // factored: w4096^(a c) at [a][c], interleaved (re, im)
 };
 
 // One fused pass of the 3D path over every tile pair (kernel_fft3d.cu); 16^3 tiles.
@@ -136,6 +138,9 @@ cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, const CUtensorMap* tm
 constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused1d(const Fft1dArgs& a, int grid, cudaStream_t s);
+size_t fused1d_ct_smem();
+cudaError_t fused1d_ct_configure(int* max_blocks_per_sm);
+cudaError_t launch_fused1d_ct(const Fft1dArgs& a, int grid, cudaStream_t s);
 
 size_t fused3d_smem();
 cudaError_t fused3d_configure(int* max_blocks_per_sm);

@@ -106,6 +106,14 @@ static double model_flops_3d(int L, int S, int T) {
 static double model_flops_1d(int S, int T) {  // one 8x8 complex tile, 4 GEMMs of 8 DMMAs
   return 32.0 * 512.0 / (2.0 * S * (double)T);
 }
+static constexpr double kEff1d = 0.73;     // PFA 8x7: executed DMMA efficiency (profiles/r01_fft1d_ncu.txt)
+
+// Factored 1D tile (kernel_fft1d_ct.cu), per pair: 4 x 64 lines of DFT-64 (16 DMMA.8x8x4
+// each, 512 flops per DMMA) + 7 complex multiplies per element (2 w4096 twiddles, 4 w64
+// twiddles, S_T; 6 flops each).
+static double flops_pair_1d_ct() { return 512.0 * 4096.0 + 6.0 * 7.0 * 4096.0; }
+static double model_flops_1d_ct(int S, int T) { return flops_pair_1d_ct() / (2.0 * S * (double)T); }
+static constexpr double kEff1dCt = 0.70;   // assumed until measured
 
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
                     HostPlan& p, std::string& err, int nranks, int rank, int algo, int periodic) {
@@ -137,28 +145,41 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
 
   // ---- tile and depth selection (Eq. 5's role, re-derived: DESIGN.md §Plan) ----
   if (ndim == 1) {
-    p.N1 = kPfaN1;
-    p.N2 = kPfaN2;
-    const int L = p.N1 * p.N2;
-    const int hmax = std::min(hmax_grid, (L - 8) / 2);   // keep S >= 8
-    if (hmax < radius) { err = "grid or radius too small for the 1D tile"; return FFTSTENCIL_EINVAL; }
-    const int tmax = hmax / radius;
-    int bestT = 1;
-    if (T == 0) {
-      double best = 1e300;
-      for (int t = 1; t <= std::min(tmax, 64); ++t) {
-        const double f = model_flops_1d(L - 2 * radius * t, t);
-        if (f < best) { best = f; bestT = t; }
+    // candidates: the prime-factor 8 x 7 tile (the paper's, §3.2.1) and the factored
+    // 4096 = 64 x 64 tile (long tiles for deep temporal fusion, kernel_fft1d_ct.cu)
+    double best = 1e300;
+    int bT = 0, bA = 0;
+    for (int al = 0; al < 2; ++al) {
+      if (algo >= 0 && al != algo) continue;
+      const int L = al ? kCt1dL : kPfaN1 * kPfaN2;
+      const int smin = al ? 64 : 8;
+      const int hmax = std::min(hmax_grid, (L - smin) / 2);
+      if (hmax < radius) continue;
+      const int tmax = hmax / radius;
+      const int tlo = T == 0 ? 1 : std::min(T, tmax), thi = T == 0 ? (al ? tmax : std::min(tmax, 64)) : tlo;
+      for (int t = tlo; t <= thi; ++t) {
+        const int S = L - 2 * radius * t;
+        const double f = al ? model_flops_1d_ct(S, t) / kEff1dCt : model_flops_1d(S, t) / kEff1d;
+        if (f < best * (1 - 1e-12)) { best = f; bT = t; bA = al; }
       }
-    } else {
-      bestT = std::min(T, tmax);
     }
-    p.T = bestT;
+    if (bT == 0) { err = "grid or radius too small for the 1D tile"; return FFTSTENCIL_EINVAL; }
+    p.algo = bA;
+    p.N1 = bA ? 64 : kPfaN1;
+    p.N2 = bA ? 64 : kPfaN2;
+    const int L = bA ? kCt1dL : p.N1 * p.N2;
+    p.T = bT;
     p.h = radius * p.T;
     p.L[0] = L;
     p.S[0] = L - 2 * p.h;
-    p.flops_per_cell_step = (16.0 * p.N1 * p.N2 * (p.N1 + p.N2) + 6.0 * p.N1 * p.N2) / (2.0 * p.S[0] * p.T);
-    p.mma_flops_per_pair = 32.0 * 512.0;
+    if (bA) {
+      p.flops_per_cell_step = model_flops_1d_ct(p.S[0], p.T);
+      p.mma_flops_per_pair = 512.0 * 4096.0;
+      p.fused_smem = (size_t)2 * kCt1dL * sizeof(double);
+    } else {
+      p.flops_per_cell_step = (16.0 * p.N1 * p.N2 * (p.N1 + p.N2) + 6.0 * p.N1 * p.N2) / (2.0 * p.S[0] * p.T);
+      p.mma_flops_per_pair = 32.0 * 512.0;
+    }
   } else if (ndim == 2) {
     // candidates: dense L x L DFT tiles and the factored 64 = 8 x 8 tile (NEXT-1)
     static const int cand[] = {16, 24, 32, 40, 48, 56, 64};
@@ -303,7 +324,25 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   }
 
   // ---- DFT matrices (forward; the kernel conjugates for the inverse, L258/L278) ----
-  if (ndim == 1) {
+  if (ndim == 1 && p.algo == 1) {
+    // [F8 | twiddles w64^(ka lb)] as in 2D, and the four-step twiddles w4096^(a c)
+    p.Fre.assign(128, 0.0);
+    p.Fim.assign(128, 0.0);
+    fill_dft(8, 8, 0, 0, p.Fre, p.Fim);
+    for (int ka = 0; ka < 8; ++ka)
+      for (int lb = 0; lb < 8; ++lb) {
+        const cplx v = root((int64_t)ka * lb, 64);
+        p.Fre[64 + ka * 8 + lb] = v.real();
+        p.Fim[64 + ka * 8 + lb] = v.imag();
+      }
+    p.tw.assign(2 * kCt1dL, 0.0);
+    for (int a = 0; a < 64; ++a)
+      for (int c = 0; c < 64; ++c) {
+        const cplx v = root((int64_t)a * c, kCt1dL);
+        p.tw[2 * (a * 64 + c)] = v.real();
+        p.tw[2 * (a * 64 + c) + 1] = v.imag();
+      }
+  } else if (ndim == 1) {
     p.Fre.assign(2 * 64, 0.0);
     p.Fim.assign(2 * 64, 0.0);
     fill_dft(p.N1, 8, 0, 0, p.Fre, p.Fim);          // rows 0..7   : F_N1
@@ -340,23 +379,24 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   }
 
   // ---- powered spectra S_t, t = 1..T (Eq. 10) with 1/prod(L) folded in (Q7) ----
+  // Powers by repeated multiplication, v_t = v_{t-1} * sigma (reading Q6), kept running
+  // across t so the build is O(T vol), not O(T^2 vol).
   p.Sre.assign(p.T, {});
   p.Sim.assign(p.T, {});
-  if (ndim == 1) {
+  if (ndim == 1 && p.algo == 0) {
     const int L = p.N1 * p.N2;
-    std::vector<cplx> sig(L);
+    std::vector<cplx> sig(L), pw(L, cplx(1.0, 0.0));
     for (int k = 0; k < L; ++k) { int kk[1] = {k}; int LL[1] = {L}; sig[k] = symbol(p, kk, LL); }
     for (int t = 1; t <= p.T; ++t) {
       auto& re = p.Sre[t - 1];
       auto& im = p.Sim[t - 1];
       re.assign(64, 0.0);
       im.assign(64, 0.0);
+      for (int k = 0; k < L; ++k) pw[k] *= sig[k];
       for (int k1 = 0; k1 < p.N1; ++k1)
         for (int k2 = 0; k2 < p.N2; ++k2) {
           const int k = (k1 * p.N2 + k2 * p.N1) % L;   // Ruritanian order (Eq. 8, reading Q8)
-          cplx v(1.0, 0.0);
-          for (int s = 0; s < t; ++s) v *= sig[k];
-          v /= (double)L;
+          const cplx v = pw[k] / (double)L;
           re[k1 * 8 + k2] = v.real();
           im[k1 * 8 + k2] = v.imag();
         }
@@ -364,7 +404,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   } else {
     int64_t vol = 1;
     for (int a = 0; a < ndim; ++a) vol *= p.L[a];
-    std::vector<cplx> sig(vol);
+    std::vector<cplx> sig(vol), pw(vol, cplx(1.0, 0.0));
     for (int64_t i = 0; i < vol; ++i) {
       int k[3], rem = (int)i;
       for (int a = ndim - 1; a >= 0; --a) { k[a] = rem % p.L[a]; rem /= p.L[a]; }
@@ -376,13 +416,16 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       re.resize(vol);
       im.resize(vol);
       for (int64_t i = 0; i < vol; ++i) {
-        cplx v(1.0, 0.0);
-        for (int s = 0; s < t; ++s) v *= sig[i];
-        v /= (double)vol;
+        pw[i] *= sig[i];
+        const cplx v = pw[i] / (double)vol;
         // 2D: natural [k0][k1].  3D: [k1][k2][k0] -- the 3D kernel multiplies in C fragments
         // whose two adjacent columns are consecutive k0 (kernel_fft3d.cu phase 2).
         int64_t dst = i;
-        if (ndim == 3 && p.algo == 1) {
+        if (ndim == 1) {
+          // factored 1D: k = c + 64 d at [c][8 (d % 8) + d / 8] (row c, CT digit order of d)
+          const int64_t c = i % 64, d = i / 64;
+          dst = c * 64 + 8 * (d % 8) + d / 8;
+        } else if (ndim == 3 && p.algo == 1) {
           // factored 3D: [k1][k2][k0 % 8][k0 / 8] (the thread-local DFT-2 output pair)
           const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
           dst = (k12 * 8 + k0 % 8) * 2 + k0 / 8;

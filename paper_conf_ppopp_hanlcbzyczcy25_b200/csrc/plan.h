@@ -22,6 +22,7 @@ constexpr int kMaxRadius = 8;
 constexpr int kPfaN1 = 8;     // 1D prime-factor split (gcd(8,7) = 1), N2 padded to 8
 constexpr int kPfaN2 = 7;
 constexpr int k3DTile = 16;   // 3D tile side (a 16^3 complex tile is 64 KiB of SMEM)
+constexpr int kCt1dL = 4096;  // factored 1D tile (64 x 64 four-step Cooley-Tukey, 64 KiB per pair)
 
 struct Box {                   // half-open box in embedded 3-axis coordinates
   int64_t lo[3];
@@ -36,8 +37,9 @@ struct HostPlan {
   std::vector<double> w;           // (2r+1)^ndim weights
   int L[3] = {1, 1, 1};            // tile extent per user axis
   int S[3] = {1, 1, 1};            // valid extent per user axis
-  int N1 = 0, N2 = 0;              // 1D prime-factor split
-  int algo = 0;                    // 0 dense DFT GEMMs, 1 factored (2D CT 8x8, 3D 8x2), 2 unfused 2D ablation
+  int N1 = 0, N2 = 0;              // 1D split: prime-factor 8 x 7, or 64 x 64 (factored)
+  int algo = 0;                    // 0 dense DFT GEMMs (1D: PFA 8x7), 1 factored (1D 64x64 CT, 2D CT 8x8, 3D 8x2),
+                                   // 2 unfused 2D ablation
   int periodic = 0;                // 1: periodic boundary (no ring/band, wrap-around tiles)
   int64_t nt[3] = {1, 1, 1};       // tiles per user axis
   int64_t tiles = 0, pairs = 0;
@@ -57,6 +59,8 @@ struct HostPlan {
   std::vector<std::vector<double>> Sre, Sim;
   //   1D: crt[l1*8 + l2] = tile position l stored at (l1, l2), or -1 for padding.
   std::vector<int> crt;
+  //   factored 1D: w4096^(a c) at [a][c], interleaved (re, im), 2 x 4096 doubles.
+  std::vector<double> tw;
   std::vector<Box> ring_boxes;     // the fixed ring, partitioned exactly
   std::vector<Box> band_boxes;     // output boxes of the band kernel (exactly-once cover)
   std::vector<int32_t> band_blocks; // 7 ints per block: out lo[3], hi[3], face axis
@@ -68,7 +72,7 @@ struct HostPlan {
 
 // Builds the plan; returns 0 or a negative FFTSTENCIL_* code with `err` set.
 // nranks/rank select one slab of the outer-axis decomposition (1/0 = whole grid).
-// algo (2D only): -1 = choose by the cost model, 0 = dense, 1 = factored (CT 8 x 8).
+// algo: -1 = choose by the cost model, 0 = dense (1D: PFA 8 x 7), 1 = factored, 2 = unfused (2D).
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
                     HostPlan& p, std::string& err, int nranks = 1, int rank = 0, int algo = -1,
                     int periodic = 0);

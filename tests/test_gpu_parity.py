@@ -363,3 +363,78 @@ def test_full_size_3d_sampled(fs, name, T):
     assert np.abs(vals - ref).max() <= TOL * np.abs(u0).max()
     assert np.isfinite(got).all()
     assert got.min() >= u0.min() - 1e-9 and got.max() <= u0.max() + 1e-9
+
+
+# ---------------------------------------------------------------- factored 1D tile (4096 = 64 x 64)
+CT1D_CASES = [((20000,), 1, 1024, 2051), ((4200,), 1, 1024, 1500), ((9001,), 3, 0, None),
+              ((12345,), 2, 100, 250), ((300000,), 1, 500, 1003), ((70000,), 2, 37, 80), ((5000,), 1, 8, 3)]
+
+
+@pytest.mark.parametrize("ext,r,T,steps", CT1D_CASES)
+def test_factored_1d_parity(fs, monkeypatch, ext, r, T, steps):
+    """kernel_fft1d_ct.cu: ragged tile counts, an odd pair, remainder passes, deep T."""
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "factored")
+    w = wl.seeded_weights("star", 1, r)
+    u0 = wl.grid(ext, 31)
+    p = fs.Plan(ext, w, r, T)
+    info = p.info()
+    assert info["algo"] == "factored" and info["tile"] == [4096]
+    steps = steps or 2 * info["T"] + 3
+    got, _ = run_gpu(fs, u0, w, r, T, steps, plan=p)
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(got, ref) <= TOL, (rel_err(got, ref), info)
+    assert np.array_equal(got[:r], u0[:r]) and np.array_equal(got[-r:], u0[-r:])
+
+
+def test_factored_1d_default_plan_parity(fs):
+    """Auto plan on a long 1D grid: the factored tile at T = 1024, two full passes + a remainder."""
+    ext, r = (1 << 20,), 1
+    w = wl.seeded_weights("star", 1, r)
+    u0 = wl.grid(ext, 37)
+    got, p = run_gpu(fs, u0, w, r, 0, 2500)
+    assert p.info()["algo"] == "factored" and p.info()["T"] == 1024
+    ref = oracle.stencil_run(u0, w, r, 2500)
+    assert rel_err(got, ref) <= TOL
+
+
+@pytest.mark.parametrize("name", ["heat1d_512m", "1d7p_512m"])
+def test_full_size_1d_sampled(fs, name):
+    """Table 3's 1D size (2^29 cells), 1000 steps in the launch configuration bench.py times:
+    sampled cells (interior, tile seams, band, ring) against the single-cell oracle."""
+    wk = wl.CONFIGS[name]
+    w = wk.weights()
+    u0 = wk.grid()
+    steps = 1000
+    got, p = run_gpu(fs, u0, w, wk.radius, 0, steps)
+    info = p.info()
+    n = wk.extents[0]
+    h, S = info["halo"], info["valid"][0]
+    rng = np.random.default_rng(41)
+    cells = list(rng.integers(0, n, 120))
+    for k in (0, 1, 2, 1000, (n - 2 * h) // S - 1):
+        cells += [h + k * S - 1, h + k * S]
+    cells += [0, wk.radius - 1, wk.radius, h - 1, h, n - h - 1, n - h, n - 1, n // 2]
+    cells = np.clip(np.array(cells), 0, n - 1).reshape(-1, 1)
+    ref = oracle.stencil_point(u0, w, wk.radius, steps, cells)
+    vals = got[cells[:, 0]]
+    assert np.abs(vals - ref).max() <= TOL * np.abs(u0).max()
+    assert np.isfinite(got).all()
+    assert got.min() >= u0.min() - 1e-9 and got.max() <= u0.max() + 1e-9
+
+
+def test_periodic_plane_wave_1d_long(fs):
+    """Oracle-free pin of the periodic factored 1D path on 2^25 cells, 3000 steps."""
+    n, steps = 1 << 25, 3000
+    w = wl.CONFIGS["1d5p_512m"].weights()
+    r = 2
+    th = 2 * np.pi * 7 / n
+    c = np.arange(n, dtype=np.float64)
+    sig = sum(w[o] * np.exp(1j * (o - r) * th) for o in range(2 * r + 1))
+    p = fs.Plan((n,), w, r, 0, periodic=True)
+    assert p.info()["algo"] == "factored"
+    a = torch.from_numpy(np.cos(th * c)).cuda()
+    b = torch.empty_like(a)
+    p.run(a, b, steps)
+    torch.cuda.synchronize()
+    ref = np.real(sig ** steps * np.exp(1j * th * c))
+    assert np.abs(b.cpu().numpy() - ref).max() <= 1e-9

@@ -325,3 +325,75 @@ def test_periodic_tiles_cover_grid_exactly_once(ext, shape, r, T):
         sl = tuple(slice(idx[a] * S[a], min(idx[a] * S[a] + S[a], ext[a])) for a in range(nd))
         count[sl] += 1
     assert count.min() == 1 and count.max() == 1
+
+
+# ---------------------------------------------------------------- factored 1D (4096 = 64 x 64)
+def test_factored_1d_is_default_for_long_grids():
+    """The cost model takes the long tile for deep fusion: T = L / (4r) maximises S T."""
+    for r in (1, 2, 3):
+        info = fs.describe((1 << 24,), wl.seeded_weights("star", 1, r), r, 0)
+        assert info["algo"] == "factored" and info["tile"] == [4096] and info["pfa"] == [64, 64]
+        assert info["T"] == 1024 // r and info["valid"] == [4096 - 2 * r * (1024 // r)]
+    # BASELINE configs[0] (4096 cells, T = 8 fixed) keeps the paper's 8 x 7 prime-factor tile
+    assert fs.describe((4096,), wl.seeded_weights("star", 1, 1), 1, 8)["algo"] == "pfa"
+
+
+def _tables_1d(n, w, r, T):
+    F8 = fs.export_aux((n,), w, r, T, which=0, axis=0)
+    tw = fs.export_aux((n,), w, r, T, which=0, axis=1)
+    W = fs.export_aux((n,), w, r, T, which=0, axis=2)
+    c = lambda v, s: (v[0::2] + 1j * v[1::2]).reshape(s)   # noqa: E731
+    return c(F8, (8, 8)), c(tw, (8, 8)), c(W, (64, 64))
+
+
+def test_factored_1d_tables_vs_numpy(factored):
+    F8, tw, W = _tables_1d(20000, wl.seeded_weights("star", 1, 1), 1, 100)
+    np.testing.assert_allclose(F8, np.fft.fft(np.eye(8), axis=0), atol=1e-15)
+    np.testing.assert_allclose(tw, np.exp(-2j * np.pi * np.outer(np.arange(8), np.arange(8)) / 64), atol=1e-15)
+    np.testing.assert_allclose(W, np.exp(-2j * np.pi * np.outer(np.arange(64), np.arange(64)) / 4096), atol=1e-15)
+
+
+def _four_step_pass(x, F8, tw, W, G):
+    """numpy model of kernel_fft1d_ct.cu on one complex tile: the four-step DFT-4096 as the
+    kernel orders it (plane[b][a] = x[a + 64 b]), * S in the kernel's [c][8 g + m] order,
+    and the inverse steps backwards."""
+    P = x.reshape(64, 64)                                # [b][a]
+    Y = _ct_axis(P.T, F8, tw).T * W.T                    # phase 1: over b -> [c][a], * w4096^(a c)
+    X = _ct_axis(Y, F8, tw)                              # phase 2: over a -> [c][d]
+    m = np.arange(64)
+    d_of = (m // 8) + 8 * (m % 8)                        # device column 8 g + m' holds d = g + 8 m'
+    Sn = np.empty((64, 64), complex)
+    Sn[:, d_of] = G                                      # natural [c][d]
+    Z = _ct_axis(X * Sn, F8, tw, inverse=True)           # over d -> [c][a]
+    Z = Z * np.conj(W.T)                                 # phase 3: * w4096^(-a c)
+    return X, _ct_axis(Z.T, F8, tw, inverse=True).T      # over c -> [b][a]
+
+
+@pytest.mark.parametrize("r,T", [(1, 1024), (2, 300), (3, 17)])
+def test_factored_1d_four_step_model_matches_oracle(factored, r, T):
+    """The exported tables, run through the kernel's four-step order, give fft(x) at
+    k = c + 64 d, and one fused pass equals T direct steps (the oracle) on [h, 4096 - h)."""
+    n = 4096
+    w = wl.seeded_weights("star", 1, r)
+    info = fs.describe((n,), w, r, T)
+    assert info["tile"] == [4096] and info["T"] == T
+    h = info["halo"]
+    F8, tw, W = _tables_1d(n, w, r, T)
+    v = fs.export_aux((n,), w, r, T, which=1, t=T)
+    G = (v[0::2] + 1j * v[1::2]).reshape(64, 64)
+    u = wl.grid((n,), 7)
+    u2 = wl.grid((n,), 8)
+    X, y = _four_step_pass(u + 1j * u2, F8, tw, W, G)
+    ref = np.fft.fft(u + 1j * u2)
+    np.testing.assert_allclose(X, ref.reshape(64, 64).T, atol=1e-10)   # X[c][d] = fft[c + 64 d]
+    y = y.reshape(-1)
+    for part, src in ((y.real, u), (y.imag, u2)):
+        want = oracle.stencil_run(src, w, r, T)
+        err = np.abs(part[h:n - h] - want[h:n - h]).max()
+        assert err <= 1e-11 * np.abs(want).max(), err
+
+
+@pytest.mark.parametrize("ext,r,T", [((20000,), 1, 1024), ((9000,), 3, 200), ((5000,), 2, 0)])
+def test_factored_1d_tiles_band_ring_partition(factored, ext, r, T):
+    count, h = _cover(ext, r, T, "star")
+    assert count.min() == 1 and count.max() == 1
