@@ -109,6 +109,17 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
+def kernel_name(info) -> str:
+    """The fused kernel this plan launches (csrc/kernel_*.cu)."""
+    nd, algo, L = info["ndim"], info["algo"], info["tile"][0]
+    if nd == 1:
+        return "fft1d_ct_kernel (4096 = 64 x 64)" if algo == "factored" else "fft1d_kernel (PFA 8 x 7)"
+    if nd == 2:
+        return {"factored": "fft2d_ct_kernel (64 = 8 x 8 per axis)", "dense": f"fft2d_kernel<{L}>",
+                "unfused": f"fft2d_kernel<{L}> forward / spec_mul / inverse"}[algo]
+    return "fft3d_ct_kernel (16 = 8 x 2 per axis)" if algo == "factored" else "fft3d_kernel"
+
+
 def load_traffic(info: dict, workload: str):
     """DRAM bytes per fused launch from the committed ncu --set full capture, if it matches."""
     path = os.path.join(ROOT, "profiles", "ncu_fused_traffic.json")
@@ -259,7 +270,7 @@ def main():
     traffic = load_traffic(info, args.workload)
     roofline = {"bound": "tensor", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
                 "frac": achieved / FP64_PEAK_TFLOPS, "traffic": traffic,
-                "kernel": f"fft2d_kernel<{info['tile'][0]}>" if info["ndim"] == 2 else "fft1d_kernel",
+                "kernel": kernel_name(info),
                 "dtype": "f64 (DMMA.8x8x4)", "peak_source": FP64_PEAK_SOURCE,
                 "alg_flops_per_launch": alg_flops_launch,
                 "flops_per_cell_step": info["flops_per_cell_step"],
