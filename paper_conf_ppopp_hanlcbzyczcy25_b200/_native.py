@@ -9,7 +9,7 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(HERE, "libfftstencil.so")
+SO_PATH = os.environ.get("FFTSTENCIL_LIB") or os.path.join(HERE, "libfftstencil.so")   # override: ablation builds
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 PERIODIC = 1

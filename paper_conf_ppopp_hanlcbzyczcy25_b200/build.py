@@ -15,8 +15,12 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-BUILD = os.path.join(HERE, "_build")
-SO = os.path.join(HERE, "libfftstencil.so")
+# Ablation builds: FFTSTENCIL_NVCC_DEFS="-DNAME=V ..." compiles a variant into its own object
+# directory and .so (FFTSTENCIL_LIB selects it at load time, _native.py).
+DEFS = os.environ.get("FFTSTENCIL_NVCC_DEFS", "").split()
+_TAG = "".join(c if c.isalnum() else "_" for c in "".join(DEFS))
+BUILD = os.path.join(HERE, "_build" + ("_" + _TAG if _TAG else ""))
+SO = os.path.join(HERE, "libfftstencil.so" if not _TAG else f"libfftstencil_{_TAG}.so")
 INCLUDE = os.path.join(ROOT, "include")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
@@ -39,12 +43,12 @@ def _nccl_dirs():
 NCCL_INC, NCCL_LIB = _nccl_dirs()
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVFLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v", *ARCH,
-           "-I", INCLUDE, "-I", CSRC, "-I", NCCL_INC]
-CXXFLAGS = ["-O2", "-std=c++17", "-fPIC", "-I", INCLUDE, "-I", CSRC]
+           "-I", INCLUDE, "-I", CSRC, "-I", NCCL_INC, *DEFS]
+CXXFLAGS = ["-O2", "-std=c++17", "-fPIC", "-I", INCLUDE, "-I", CSRC, *DEFS]
 
 CU = ["capi.cu", "kernel_fft2d.cu", "kernel_fft2d_ct.cu", "kernel_fft1d.cu", "kernel_fft1d_ct.cu", "kernel_fft3d.cu", "kernel_fft3d_ct.cu", "kernel_band.cu"]
 CPP = ["plan.cpp"]
-HEADERS = ["plan.h", "kernels.cuh", "device_common.cuh", "tma.cuh"]
+HEADERS = ["plan.h", "kernels.cuh", "device_common.cuh", "tma.cuh", "ct_line.cuh"]
 
 
 def _stale(obj: str, src: str) -> bool:

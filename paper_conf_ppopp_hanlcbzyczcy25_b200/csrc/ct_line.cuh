@@ -82,9 +82,51 @@ __device__ __forceinline__ void twiddle(double (&cr)[2], double (&ci)[2], const 
 }
 
 // NL independent lines per warp, their DMMA chains interleaved for latency hiding.
-template <bool CONJ, int NL>
+// Complex 8x8x8 products as real DMMAs.  FFTSTENCIL_CMUL3 = 1 (default): the 3-multiply
+// form (Gauss / "3M"), P1 = Ar Br, P2 = Ai Bi, P3 = (Ar + Ai)(Br + Bi),
+// Re = P1 - P2, Im = P3 - P1 - P2 -- 6 DMMA.8x8x4 per product instead of 8, for 8 FP64
+// adds per thread; 0: the 4-multiply form.  The 1D and 2D factored kernels use it; the 3D one
+// (less tensor-bound, measured profiles/r01_cmul3.jsonl) keeps 4M (FFTSTENCIL_CMUL3_3D).
+#ifndef FFTSTENCIL_CMUL3
+#define FFTSTENCIL_CMUL3 1
+#endif
+#ifndef FFTSTENCIL_CMUL3_3D
+#define FFTSTENCIL_CMUL3_3D 0
+#endif
+
+template <int NL>
+__device__ __forceinline__ void finish3(double (&cr)[NL][2], double (&ci)[NL][2], const double (&p1)[NL][2],
+                                        const double (&p2)[NL][2], const double (&p3)[NL][2]) {
+#pragma unroll
+  for (int u = 0; u < NL; ++u)
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      cr[u][e] = p1[u][e] - p2[u][e];
+      ci[u][e] = p3[u][e] - p1[u][e] - p2[u][e];
+    }
+}
+
+// B-route: C = F8' . B with F8' = F8 (CONJ = false) or conj(F8).
+template <bool CONJ, int NL, bool M3 = FFTSTENCIL_CMUL3 != 0>
 __device__ __forceinline__ void broute_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&fr)[2],
                                          const double (&fi)[2], const double (&br)[NL][2], const double (&bi)[NL][2]) {
+  if constexpr (M3) {
+  double p1[NL][2], p2[NL][2], p3[NL][2];
+#pragma unroll
+  for (int u = 0; u < NL; ++u) p1[u][0] = p1[u][1] = p2[u][0] = p2[u][1] = p3[u][0] = p3[u][1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const double f_i = CONJ ? -fi[j] : fi[j];
+    const double fs = fr[j] + f_i;
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(p1[u], fr[j], br[u][j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(p2[u], f_i, bi[u][j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(p3[u], fs, br[u][j] + bi[u][j]);
+  }
+  finish3<NL>(cr, ci, p1, p2, p3);
+  } else {
 #pragma unroll
   for (int u = 0; u < NL; ++u) cr[u][0] = cr[u][1] = ci[u][0] = ci[u][1] = 0.0;
 #pragma unroll
@@ -99,11 +141,30 @@ __device__ __forceinline__ void broute_n(double (&cr)[NL][2], double (&ci)[NL][2
 #pragma unroll
     for (int u = 0; u < NL; ++u) dmma(ci[u], -nfi, br[u][j]);
   }
+  }
 }
 
-template <bool CONJ, int NL>
+// A-route: C = D . F8'^T.
+template <bool CONJ, int NL, bool M3 = FFTSTENCIL_CMUL3 != 0>
 __device__ __forceinline__ void aroute_n(double (&cr)[NL][2], double (&ci)[NL][2], const double (&dr)[NL][2],
                                          const double (&di)[NL][2], const double (&fr)[2], const double (&fi)[2]) {
+  if constexpr (M3) {
+  double p1[NL][2], p2[NL][2], p3[NL][2];
+#pragma unroll
+  for (int u = 0; u < NL; ++u) p1[u][0] = p1[u][1] = p2[u][0] = p2[u][1] = p3[u][0] = p3[u][1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    const double f_i = CONJ ? -fi[j] : fi[j];
+    const double fs = fr[j] + f_i;
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(p1[u], dr[u][j], fr[j]);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(p2[u], di[u][j], f_i);
+#pragma unroll
+    for (int u = 0; u < NL; ++u) dmma(p3[u], dr[u][j] + di[u][j], fs);
+  }
+  finish3<NL>(cr, ci, p1, p2, p3);
+  } else {
 #pragma unroll
   for (int u = 0; u < NL; ++u) cr[u][0] = cr[u][1] = ci[u][0] = ci[u][1] = 0.0;
 #pragma unroll
@@ -117,6 +178,7 @@ __device__ __forceinline__ void aroute_n(double (&cr)[NL][2], double (&ci)[NL][2
     for (int u = 0; u < NL; ++u) dmma(cr[u], di[u][j], nfi);
 #pragma unroll
     for (int u = 0; u < NL; ++u) dmma(ci[u], dr[u][j], -nfi);
+  }
   }
 }
 

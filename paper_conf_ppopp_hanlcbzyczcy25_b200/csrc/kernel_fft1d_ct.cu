@@ -50,7 +50,7 @@ __device__ __forceinline__ void cmul(double (&cr)[1][2], double (&ci)[1][2], con
 }
 
 template <bool WRAP>   // WRAP: periodic boundary (wrap-around tile loads)
-__global__ void __launch_bounds__(kThreads, 3) fft1d_ct_kernel(const Fft1dArgs a) {
+__global__ void __maxnreg__(72) fft1d_ct_kernel(const Fft1dArgs a) {
   extern __shared__ __align__(128) double smem[];
   double* sR = smem;           // tile 2p   (Re), then the transform's real parts
   double* sI = smem + PLANE;   // tile 2p+1 (Im)

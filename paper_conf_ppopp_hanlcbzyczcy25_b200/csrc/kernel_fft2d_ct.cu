@@ -45,7 +45,12 @@ __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool v
 // layout; phase 1 reads its rows there (4-way bank conflicts on that pass only) and, the
 // XOR swizzle being a permutation within a row, rewrites each row in place swizzled.
 template <int NW, int NL, bool TMA, bool WRAP = false>   // WRAP: periodic (cp.async path only)
-__global__ void __launch_bounds__(NW * 32, NL > 2 ? 2 : 3)
+// FFTSTENCIL_CT2D_REGS (80): three CTAs per SM (72 would admit a band CTA beside them, but
+// costs 1.5% in spills: profiles/r01_cmul3.jsonl)
+#ifndef FFTSTENCIL_CT2D_REGS
+#define FFTSTENCIL_CT2D_REGS 80
+#endif
+__global__ void __maxnreg__(NL > 2 ? 128 : (NW == 16 ? 40 : FFTSTENCIL_CT2D_REGS))
     fft2d_ct_kernel(const Fft2dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ __align__(128) double smem[];
   double* sR = smem;            // plane 0: tile 2j (Re), then Q/W real parts

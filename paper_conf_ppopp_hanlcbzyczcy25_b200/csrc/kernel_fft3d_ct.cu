@@ -24,7 +24,7 @@
 // 64 KB for both planes -> 3 CTAs / SM.  f permutes words within a 16-element row only, so
 // with TMA the tiles land as two dense 16^3 boxes and P1 (whose groups own whole rows)
 // reads them unswizzled and rewrites its rows swizzled in place.
-#include "device_common.cuh"
+#include "ct_line.cuh"
 #include "kernels.cuh"
 #include "tma.cuh"
 
@@ -33,7 +33,7 @@ namespace {
 
 using dev::dmma;
 
-constexpr int L = 16;
+constexpr int L = 16;   // (ct::L = 64 is the 2D line; unused here)
 constexpr int PLANE = L * L * L;
 constexpr int NWC = 8;
 
@@ -64,18 +64,14 @@ struct Lines {
   }
 };
 
+// C = F8' . B (B-route of ct_line.cuh, one group; 4M unless FFTSTENCIL_CMUL3_3D)
 template <bool CONJ>
 __device__ __forceinline__ void cgemm(double (&cr)[2], double (&ci)[2], const double (&fr)[2], const double (&fi)[2],
                                       const double (&br)[2], const double (&bi)[2]) {
-  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
-#pragma unroll
-  for (int j = 0; j < 2; ++j) {
-    const double nfi = CONJ ? fi[j] : -fi[j];
-    dmma(cr, fr[j], br[j]);
-    dmma(ci, fr[j], bi[j]);
-    dmma(cr, nfi, bi[j]);
-    dmma(ci, -nfi, br[j]);
-  }
+  double r[1][2], i[1][2];
+  const double b_r[1][2] = {{br[0], br[1]}}, b_i[1][2] = {{bi[0], bi[1]}};
+  ct::broute_n<CONJ, 1, FFTSTENCIL_CMUL3_3D != 0>(r, i, fr, fi, b_r, b_i);
+  cr[0] = r[0][0]; cr[1] = r[0][1]; ci[0] = i[0][0]; ci[1] = i[0][1];
 }
 
 struct Regs {
@@ -148,7 +144,7 @@ __device__ __forceinline__ void inv_group(double* sR, double* sI, const LN& ln, 
 }
 
 template <bool TMA, bool WRAP = false>   // WRAP: periodic boundary (cp.async path only)
-__global__ void __launch_bounds__(NWC * 32, 3) fft3d_ct_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
+__global__ void __maxnreg__(72) fft3d_ct_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ __align__(128) double smem[];
   double* sR = smem;
   double* sI = smem + PLANE;

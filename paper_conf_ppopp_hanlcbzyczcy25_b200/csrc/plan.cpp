@@ -61,11 +61,12 @@ double model_flops_2d(int L, int S, int T) {
   return 8.0 * dm / (2.0 * S * (double)S * T);
 }
 
-// Factored tile (kernel_fft2d_ct.cu), per pair: DMMA.8x8x4 x 512 flops for 64 rows x 2
-// stages + 64 columns x 4 stages + S rows x 2 stages (8 DMMA per stage and line), twiddles
-// (6 flops per element, 192 + S lines of 64) and the S_T multiply (6 flops per element).
+// Factored tile (kernel_fft2d_ct.cu), per pair: complex 8x8x8 products (kProdFlops each)
+// for 64 rows x 2 stages + 64 columns x 4 stages + S rows x 2 stages, twiddles (6 flops per
+// element, 192 + S lines of 64) and the S_T multiply (6 flops per element).
+static double products_2d_ct(int S) { return 384.0 + 2.0 * S; }
 double model_flops_2d_ct(int S, int T) {
-  const double f = 512.0 * (3072.0 + 16.0 * S) + 384.0 * (192.0 + S) + 6.0 * 4096.0;
+  const double f = kProdFlops * products_2d_ct(S) + 384.0 * (192.0 + S) + 6.0 * 4096.0;
   return f / (2.0 * S * (double)S * T);
 }
 
@@ -89,10 +90,10 @@ static double eff_2d(int L) {
 
 // Factored 3D tile (kernel_fft3d_ct.cu): line groups of 4 per pair (64 per forward axis,
 // 64 for the inverse axis 0, 4S for inverse axis 1, S ceil(S/4) for inverse axis 2), each
-// 8 DMMA.8x8x4 (4096 flops) + twiddle (32 x 6) + DFT-2 (64 x 2); + S_T (6 per element).
+// one complex 8x8x8 product (kProdFlops) + twiddle (32 x 6) + DFT-2 (64 x 2); + S_T.
 static double groups_3d_ct(int S) { return 256.0 + 4.0 * S + S * (double)((S + 3) / 4); }
 static double model_flops_3d_ct(int S, int T) {
-  return (4416.0 * groups_3d_ct(S) + 6.0 * 4096.0) / (2.0 * S * (double)S * S * T);
+  return ((prod_flops(kCmul3_3d) + 320.0) * groups_3d_ct(S) + 6.0 * 4096.0) / (2.0 * S * (double)S * S * T);
 }
 static constexpr double kEff3d = 0.70;     // dense 3D: executed DMMA efficiency (profiles/r01_sweep.txt)
 static constexpr double kEff3dCt = 0.60;   // factored 3D: assumed until measured
@@ -108,10 +109,10 @@ static double model_flops_1d(int S, int T) {  // one 8x8 complex tile, 4 GEMMs o
 }
 static constexpr double kEff1d = 0.73;     // PFA 8x7: executed DMMA efficiency (profiles/r01_fft1d_ncu.txt)
 
-// Factored 1D tile (kernel_fft1d_ct.cu), per pair: 4 x 64 lines of DFT-64 (16 DMMA.8x8x4
-// each, 512 flops per DMMA) + 7 complex multiplies per element (2 w4096 twiddles, 4 w64
-// twiddles, S_T; 6 flops each).
-static double flops_pair_1d_ct() { return 512.0 * 4096.0 + 6.0 * 7.0 * 4096.0; }
+// Factored 1D tile (kernel_fft1d_ct.cu), per pair: 4 x 64 lines of DFT-64 (2 complex 8x8x8
+// products each) + 7 complex multiplies per element (2 w4096 twiddles, 4 w64 twiddles, S_T;
+// 6 flops each).
+static double flops_pair_1d_ct() { return kProdFlops * 512.0 + 6.0 * 7.0 * 4096.0; }
 static double model_flops_1d_ct(int S, int T) { return flops_pair_1d_ct() / (2.0 * S * (double)T); }
 static constexpr double kEff1dCt = 0.70;   // assumed until measured
 
@@ -174,7 +175,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     p.S[0] = L - 2 * p.h;
     if (bA) {
       p.flops_per_cell_step = model_flops_1d_ct(p.S[0], p.T);
-      p.mma_flops_per_pair = 512.0 * 4096.0;
+      p.mma_flops_per_pair = kProdDmmaFlops * 512.0;
       p.fused_smem = (size_t)2 * kCt1dL * sizeof(double);
     } else {
       p.flops_per_cell_step = (16.0 * p.N1 * p.N2 * (p.N1 + p.N2) + 6.0 * p.N1 * p.N2) / (2.0 * p.S[0] * p.T);
@@ -222,7 +223,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       p.fused_smem = (size_t)(bL >= 56 ? 48 : 32) * bL * (bL + 4);   // F + pair buffer(s)
     } else {
       p.flops_per_cell_step = model_flops_2d_ct(p.S[0], bT);
-      p.mma_flops_per_pair = 512.0 * (3072.0 + 16.0 * S);
+      p.mma_flops_per_pair = kProdDmmaFlops * products_2d_ct(p.S[0]);
       p.fused_smem = (size_t)2 * 64 * 64 * sizeof(double);
     }
   } else {
@@ -259,7 +260,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       p.fused_smem = (size_t)(2 * 16 * 20 + 2 * 16 * (16 * 20 + 4)) * sizeof(double);
     } else {
       p.flops_per_cell_step = model_flops_3d_ct(p.S[0], bestT);
-      p.mma_flops_per_pair = 4096.0 * groups_3d_ct(p.S[0]);
+      p.mma_flops_per_pair = prod_dmma_flops(kCmul3_3d) * groups_3d_ct(p.S[0]);
       p.fused_smem = (size_t)2 * 16 * 16 * 16 * sizeof(double);
     }
   }

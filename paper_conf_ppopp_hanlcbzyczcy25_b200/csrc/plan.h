@@ -19,6 +19,21 @@
 namespace fstencil {
 
 constexpr int kMaxRadius = 8;
+
+// Complex 8x8x8 products of the factored kernels (ct_line.cuh): the 3-multiply form by
+// default (6 DMMA.8x8x4 + 256 FP64 adds per product of 64 outputs), else 4-multiply (8 DMMA).
+#ifndef FFTSTENCIL_CMUL3
+#define FFTSTENCIL_CMUL3 1
+#endif
+#ifndef FFTSTENCIL_CMUL3_3D
+#define FFTSTENCIL_CMUL3_3D 0
+#endif
+constexpr bool kCmul3 = FFTSTENCIL_CMUL3 != 0;        // factored 1D and 2D kernels
+constexpr bool kCmul3_3d = FFTSTENCIL_CMUL3_3D != 0;  // factored 3D kernel
+constexpr double prod_dmma_flops(bool m3) { return m3 ? 6 * 512.0 : 8 * 512.0; }   // executed on the tensor pipe
+constexpr double prod_flops(bool m3) { return m3 ? 6 * 512.0 + 256.0 : 8 * 512.0; }
+constexpr double kProdDmmaFlops = prod_dmma_flops(kCmul3);
+constexpr double kProdFlops = prod_flops(kCmul3);
 constexpr int kPfaN1 = 8;     // 1D prime-factor split (gcd(8,7) = 1), N2 padded to 8
 constexpr int kPfaN2 = 7;
 constexpr int k3DTile = 16;   // 3D tile side (a 16^3 complex tile is 64 KiB of SMEM)
