@@ -41,6 +41,32 @@ __global__ void dfma_loop(double* out, int iters, double a0, double b0) {
   out[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
 
+// DMMA and DFMA interleaved in one warp stream (independent accumulators): tells whether
+// the tensor DMMA path and the FP64 FMA units share throughput on this GPU.
+template <int CH, int NF>
+__global__ void mix_loop(double* out, int iters, double a0, double b0) {
+  double c[CH][2], f[NF > 0 ? NF : 1];
+#pragma unroll
+  for (int i = 0; i < CH; ++i) { c[i][0] = 0; c[i][1] = 0; }
+#pragma unroll
+  for (int i = 0; i < NF; ++i) f[i] = threadIdx.x * 1e-3 + i;
+  double a = a0 * threadIdx.x, b = b0;
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int i = 0; i < CH; ++i) {
+      dmma(c[i][0], c[i][1], a, b);
+#pragma unroll
+      for (int k = 0; k < NF / CH; ++k) f[i * (NF / CH) + k] = fma(f[i * (NF / CH) + k], a0, b0);
+    }
+  }
+  double s = 0;
+#pragma unroll
+  for (int i = 0; i < CH; ++i) s += c[i][0] + c[i][1];
+#pragma unroll
+  for (int i = 0; i < NF; ++i) s += f[i];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
 __global__ void layout_probe(double* A, double* B, double* C) {
   int lane = threadIdx.x;
   // A[8][4] row-major, B[4][8] row-major (k, n), fragment per documented layout
@@ -80,6 +106,25 @@ int main() {
       double flops = 2.0 * 8 * (double)iters * blocks * wpb * 32;
       if (rep) printf("DFMA: warps/block %d blocks %d -> %.2f TFLOP/s (%.3f ms)\n", wpb, blocks, flops / ms / 1e9, ms);
     }
+  }
+  // shared or separate FP64 throughput: CH DMMA + NF DFMA per iteration and warp
+  {
+    const int wpb = 16, blocks = sms * 2;
+    auto run = [&](auto kern, const char* name, double dm_flops, double fm_flops) {
+      for (int rep = 0; rep < 2; ++rep) {
+        cudaEventRecord(e0);
+        kern<<<blocks, wpb * 32>>>(out, iters, 1.0000001, 1e-9);
+        cudaEventRecord(e1); cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        const double w = (double)iters * blocks * wpb;
+        if (rep) printf("%s: %.3f ms  DMMA %.2f TF + DFMA %.2f TF = %.2f TF\n", name, ms, dm_flops * w / ms / 1e9,
+                        fm_flops * w / ms / 1e9, (dm_flops + fm_flops) * w / ms / 1e9);
+      }
+    };
+    run(mix_loop<8, 0>, "mix DMMA x8 only      ", 2.0 * 256 * 8, 0.0);
+    run(mix_loop<8, 64>, "mix DMMA x8 + DFMA x64", 2.0 * 256 * 8, 2.0 * 32 * 64);
+    run(mix_loop<8, 32>, "mix DMMA x8 + DFMA x32", 2.0 * 256 * 8, 2.0 * 32 * 32);
+    run(mix_loop<8, 16>, "mix DMMA x8 + DFMA x16", 2.0 * 256 * 8, 2.0 * 32 * 16);
   }
   // layout probe
   double hA[32], hB[32], hC[64], ref[64];
