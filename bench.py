@@ -32,6 +32,9 @@ sys.path.insert(0, ROOT)
 from synth import workloads as wl  # noqa: E402
 
 FP64_PEAK_TFLOPS = 37.18   # measured DMMA.8x8x4 peak on this pool's B200 (profiles/r01_fp64_peak.txt)
+FP64_ALU_PEAK_TOPS = 34.13 / 2   # measured DFMA 34.13 TF/s = 17.07 T FP64 instructions/s
+FP64_ALU_PEAK_SOURCE = ("measured: tools/fp64_peak.cu DFMA microbenchmark 34.13 TFLOP/s / 2 flops per DFMA "
+                        "(profiles/r01_fp64_peak.txt); one DADD/DMUL/DFMA = one FP64 pipe slot")
 FP64_PEAK_SOURCE = ("measured: tools/fp64_peak.cu DMMA m8n8k4 microbenchmark, 148 SMs x 64 FMA/clk x 1.965 GHz "
                     "(profiles/r01_fp64_peak.txt); MEASURED_PEAKS.json carries no FP64 figure")
 
@@ -115,9 +118,14 @@ def kernel_name(info) -> str:
     if nd == 1:
         return "fft1d_ct_kernel (4096 = 64 x 64)" if algo == "factored" else "fft1d_kernel (PFA 8 x 7)"
     if nd == 2:
+        if algo == "factored" and info.get("engine") == "alu":
+            return "fft2d_bf_kernel (64 = 8 x 8 radix-8 FFT per axis, FP64 ALU)"
         return {"factored": "fft2d_ct_kernel (64 = 8 x 8 per axis)", "dense": f"fft2d_kernel<{L}>",
                 "unfused": f"fft2d_kernel<{L}> forward / spec_mul / inverse"}[algo]
-    return "fft3d_ct_kernel (16 = 8 x 2 per axis)" if algo == "factored" else "fft3d_kernel"
+    if algo == "factored":
+        return ("fft3d_bf_kernel (16 = 4 x 4 radix-4 FFT per line, FP64 ALU)" if info.get("engine") == "alu"
+                else "fft3d_ct_kernel (16 = 8 x 2 per axis)")
+    return "fft3d_kernel"
 
 
 def load_traffic(info: dict, workload: str):
@@ -279,6 +287,14 @@ def main():
                 "fused_ms_avg": fused_avg_s * 1e3, "fused_share_of_step": prof["fused_ms"] / max(ms, 1e-9),
                 "fused_launches": prof["fused_launches"], "passes": passes,
                 "band_ms_avg": prof["band_ms"] / max(1, prof["band_launches"])}
+    if info.get("engine") == "alu":
+        # FP64 ALU engine: the binding unit is the FP64 pipe's issue rate (adds, multiplies and
+        # FMAs each take one slot); peak = the measured DFMA rate / 2 (profiles/r01_fp64_peak.txt)
+        ops = info["alu_ops_per_pass"] / fused_avg_s / 1e12
+        roofline.update({"bound": "alu", "achieved": ops, "peak": FP64_ALU_PEAK_TOPS, "unit": "Top/s",
+                         "frac": ops / FP64_ALU_PEAK_TOPS, "dtype": "f64 (DADD/DMUL/DFMA)",
+                         "peak_source": FP64_ALU_PEAK_SOURCE, "alu_ops_per_launch": info["alu_ops_per_pass"],
+                         "alg_tflops": achieved})
 
     # ---- end to end through the host-buffer C-ABI entry point ----
     e2e = None

@@ -90,6 +90,11 @@ typedef struct {
                                    (FFTSTENCIL_ALGO=unfused: forward / multiply / inverse as
                                    three kernels with the spectrum in HBM)                  */
   int periodic;                 /* 1 for a FFTSTENCIL_PERIODIC plan                      */
+  int engine;                   /* line-DFT engine of the factored 3D tile: 0 DFT-8 GEMMs on
+                                   the FP64 tensor pipe (DMMA), 1 radix-4 FFTs in registers on
+                                   the FP64 ALU (default; FFTSTENCIL_ENGINE=dmma|alu)         */
+  double alu_ops_per_pass;      /* engine 1: FP64 ALU instructions one fused launch executes
+                                   (adds, multiplies and FMAs, each one)                    */
 } fftstencil_info;
 
 /* Plan creation flags (fftstencil_plan_create_ex / fftstencil_describe_ex). */

@@ -55,6 +55,8 @@ class Info(ctypes.Structure):
         ("ghost_hi", ctypes.c_int64),
         ("algo", ctypes.c_int),
         ("periodic", ctypes.c_int),
+        ("engine", ctypes.c_int),
+        ("alu_ops_per_pass", ctypes.c_double),
     ]
 
     def as_dict(self) -> dict:
@@ -72,6 +74,7 @@ class Info(ctypes.Structure):
             "interior_end": self.interior_end, "ghost_lo": self.ghost_lo, "ghost_hi": self.ghost_hi,
             "algo": ("dense", "factored", "unfused")[self.algo] if nd >= 2 else ("pfa", "factored")[self.algo],
             "periodic": bool(self.periodic),
+            "engine": ("dmma", "alu")[self.engine], "alu_ops_per_pass": self.alu_ops_per_pass,
         }
 
 

@@ -189,6 +189,8 @@ void fill_info(const HostPlan& hp, fftstencil_info* info) {
   info->ghost_hi = hp.g1 - hp.row_hi;
   info->algo = hp.algo;
   info->periodic = hp.periodic;
+  info->engine = hp.engine;
+  info->alu_ops_per_pass = hp.alu_ops_per_pair * (double)(hp.pair_hi - hp.pair_lo);
 }
 
 // Profiling: a (start, end) event pair around one launch; returns the pair index or -1.
@@ -268,9 +270,13 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
       a.Fim = p->dF + 128;
       CUtensorMap tm;
       const uint64_t dims[2] = {(uint64_t)hp.ext[1], (uint64_t)(hp.g1 - hp.g0)};
-      const uint32_t box[2] = {64, 64};
-      const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 2, dims, box);
-      e = launch_fused2d_ct(p->ct_cfg, a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+      const uint32_t box[2] = {64, 64}, box_bf[2] = {16, 64};
+      const bool bf = hp.engine == 1;
+      const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 2, dims, bf ? box_bf : box, bf);
+      if (bf)
+        e = launch_fused2d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+      else
+        e = launch_fused2d_ct(p->ct_cfg, a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
       e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(p->fused_grid, np), s);
@@ -320,8 +326,11 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
       CUtensorMap tm;
       const uint64_t dims[3] = {(uint64_t)hp.ext[2], (uint64_t)hp.ext[1], (uint64_t)(hp.g1 - hp.g0)};
       const uint32_t box[3] = {16, 16, 16};
-      const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 3, dims, box);
-      e = launch_fused3d_ct(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+      const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 3, dims, box, hp.engine == 1);
+      if (hp.engine == 1)
+        e = launch_fused3d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+      else
+        e = launch_fused3d_ct(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
       e = launch_fused3d(a, (int)std::min<int64_t>(p->fused_grid, np), s);
@@ -591,7 +600,7 @@ int setup_device(fftstencil_plan* p) {
   if (hp.ndim == 2 && hp.algo == 1) {
     if (const char* v = std::getenv("FFTSTENCIL_CT_CFG")) p->ct_cfg = std::atoi(v);
     if (const char* v = std::getenv("FFTSTENCIL_TMA")) p->use_tma = std::atoi(v) != 0;
-    e = fused2d_ct_configure(p->ct_cfg, &occ);
+    e = hp.engine == 1 ? fused2d_bf_configure(&occ) : fused2d_ct_configure(p->ct_cfg, &occ);
     if (e == cudaErrorInvalidValue) {
       set_error("FFTSTENCIL_CT_CFG must be one of 81, 82, 84, 161, 162");
       return FFTSTENCIL_EINVAL;
@@ -616,7 +625,7 @@ int setup_device(fftstencil_plan* p) {
     if (e != cudaSuccess) return cuda_fail(e, "fused 2D kernel configuration");
   } else if (hp.ndim == 3 && hp.algo == 1) {
     if (const char* v = std::getenv("FFTSTENCIL_TMA")) p->use_tma = std::atoi(v) != 0;
-    e = fused3d_ct_configure(&occ);
+    e = hp.engine == 1 ? fused3d_bf_configure(&occ) : fused3d_ct_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "factored 3D kernel configuration");
   } else if (hp.ndim == 3) {
     e = fused3d_configure(&occ);
@@ -653,7 +662,8 @@ int setup_device(fftstencil_plan* p) {
 }  // namespace
 
 namespace fstencil {
-bool encode_tensor_map(CUtensorMap* map, const void* base, int rank, const uint64_t* dims, const uint32_t* box) {
+bool encode_tensor_map(CUtensorMap* map, const void* base, int rank, const uint64_t* dims, const uint32_t* box,
+                       bool swizzle128) {
   EncodeTiledFn fn = encode_fn();
   if (!fn || rank < 1 || rank > 3 || (reinterpret_cast<uintptr_t>(base) & 15)) return false;
   cuuint64_t gdim[3], gstride[2];
@@ -669,7 +679,8 @@ bool encode_tensor_map(CUtensorMap* map, const void* base, int rank, const uint6
     stride *= dims[i];
   }
   return fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)rank, const_cast<void*>(base), gdim, gstride, bdim, es,
-            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_INTERLEAVE_NONE,
+            swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 }  // namespace fstencil
@@ -734,6 +745,11 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
       L = axis == 0 ? hp.N1 : hp.N2;
       row0 = axis == 0 ? 0 : 8;
       ld = 8;
+    } else if (hp.ndim == 2 && hp.algo == 1 && hp.engine == 1) {
+      // radix-8 ALU engine: axis 0 = the w64^m table, m = 0..63
+      if (axis != 0) { set_error("axis must be 0 (w64^m) for the ALU engine"); return FFTSTENCIL_EINVAL; }
+      for (int m = 0; m < 64; ++m) { v.push_back(hp.Fre[m]); v.push_back(hp.Fim[m]); }
+      L = 0;
     } else if (hp.ndim == 2 && hp.algo == 1) {
       if (axis < 0 || axis > 1) { set_error("axis must be 0 (F_8) or 1 (twiddles)"); return FFTSTENCIL_EINVAL; }
       L = 8;

@@ -1,0 +1,280 @@
+// Fused 3D FFT-stencil tile kernel with register-resident radix-4 FFTs on the FP64 ALU
+// (sm_100a).  One thread owns one whole 16-point line per pass.
+//
+// Same fused pass as kernel_fft3d_ct.cu (Algorithm 1 L252-L258 on 16^3 overlap-save
+// tiles, Double-layer Filling Eq. 9, temporal fusion Eq. 10, Stitching Eq. 7; 3D handled axis
+// by axis as in §3.2.1), with each length-16 axis DFT evaluated as a 4 x 4 Cooley-Tukey
+// FFT in registers (fft_radix.cuh: 160 FP64 instructions per line) instead of DFT-8 GEMMs on
+// the tensor pipe (kernel_fft3d_ct.cu: 8 DMMA.8x8x4 = 2048 FMA per 4 lines, i.e. ~512 FP64
+// pipe operations per line on a pipe B200 shares between DMMA and DFMA).
+//
+// Per tile pair, five shared-memory passes, each thread reading one line and rewriting it in
+// place (no intra-pass exchange):
+//   P1 forward axis 2 | P2 forward axis 1 | P3 forward axis 0, * S_T, inverse axis 0 (writes
+//   only the S output planes) | P4 inverse axis 1 on those planes (writes only the S output
+//   rows) | P5 inverse axis 2 on the S x S output rows -> store the S^3 window.
+// Shared layout = the TMA SWIZZLE_128B image of a dense 16^3 box: element (l0, l1, l2) at
+// word 256 l0 + 16 l1 + (l2 ^ 2 (l1 & 7)) (the 16-byte chunk index XOR row mod 8).  Bank
+// check (8-byte words, a half-warp per wavefront; 16-byte words, a quarter-warp):
+//   P1/P5 (thread = (l0, l1), 16-byte loads of chunk c): lanes l1 = 0..7 -> chunks c ^ l1
+//         distinct.  P2/P4 (thread = (l0, l2), element l1 = p): lanes l2 = 0..15 -> words
+//         l2 ^ 2 (p & 7) distinct.  P3 (thread = (l1, l2), element l0 = p): lanes l2 = 0..15
+//         distinct.  All conflict-free except P5's ragged quarter-warps.
+// The spectrum S_T is in natural [k0][k1][k2] order (read coalesced across lanes in P3).
+#include "fft_radix.cuh"
+#include "kernels.cuh"
+#include "tma.cuh"
+
+namespace fstencil {
+namespace {
+
+constexpr int L = 16;
+constexpr int PLANE = L * L * L;
+constexpr int NT = 256;                 // threads per CTA: one per line of a full pass
+constexpr int kAlign = 1024;            // SWIZZLE_128B destinations are 1024-byte aligned
+
+__device__ __forceinline__ int wofs(int l0, int l1, int l2) { return (l0 << 8) | (l1 << 4) | (l2 ^ ((l1 & 7) << 1)); }
+
+__device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
+}
+
+// Row lines (along l2) at row (l0, l1): 16-byte chunk c holds l2 = 2c, 2c + 1 at chunk c ^ (l1 & 7).
+__device__ __forceinline__ void load_row(const double* sR, const double* sI, int l0, int l1, double (&xr)[16],
+                                         double (&xi)[16]) {
+  const int base = (l0 << 8) | (l1 << 4), s = l1 & 7;
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    const int o = base + ((c ^ s) << 1);
+    const double2 r = *reinterpret_cast<const double2*>(sR + o);
+    const double2 i = *reinterpret_cast<const double2*>(sI + o);
+    xr[2 * c] = r.x; xr[2 * c + 1] = r.y;
+    xi[2 * c] = i.x; xi[2 * c + 1] = i.y;
+  }
+}
+__device__ __forceinline__ void store_row(double* sR, double* sI, int l0, int l1, const double (&xr)[16],
+                                          const double (&xi)[16]) {
+  const int base = (l0 << 8) | (l1 << 4), s = l1 & 7;
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    const int o = base + ((c ^ s) << 1);
+    *reinterpret_cast<double2*>(sR + o) = make_double2(xr[2 * c], xr[2 * c + 1]);
+    *reinterpret_cast<double2*>(sI + o) = make_double2(xi[2 * c], xi[2 * c + 1]);
+  }
+}
+
+// Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
+__device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
+
+struct PairGeom {
+  int64_t o0, o1, oa2, ob2;
+  bool has_b;
+};
+__device__ __forceinline__ PairGeom pair_geom(const Fft3dArgs& a, int64_t p) {
+  const int S = a.S;
+  const int64_t line = p / a.npr, pj = p - line * a.npr;
+  const int64_t t0 = line / a.nt1, t1 = line - t0 * a.nt1;
+  PairGeom g;
+  g.o0 = t0 * S + a.bd.shift;
+  g.o1 = t1 * S + a.bd.shift;
+  g.oa2 = 2 * pj * S + a.bd.shift;
+  g.ob2 = g.oa2 + S;
+  g.has_b = 2 * pj + 1 < a.nt2;
+  return g;
+}
+
+// One CTA per SM = two independent 256-thread groups, each transforming its own sequence of
+// tile pairs in its own 64 KB buffer (the other group's work hides a group's TMA latency and
+// barrier waits); S_T (64 KB) is staged once and shared: 192 KB.  Thread t of a group owns
+// line (t >> 4, t & 15) of every pass, so a warp's P1 rows and P2 lines lie in the same two
+// l0-planes (P1 -> P2 needs only __syncwarp), and likewise P4 -> P5 on the output planes.
+// TMA = false: cp.async loads (periodic wrap-around, or a pitch TMA cannot describe).
+template <bool TMA, bool WRAP = false>
+__global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
+  extern __shared__ unsigned char smem_raw[];
+  const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
+  double* base = reinterpret_cast<double*>(smem_raw + (mis ? kAlign - mis : 0));   // stays in the shared window
+  const double* sSr = base + 4 * PLANE;
+  const double* sSi = sSr + PLANE;
+  __shared__ __align__(8) uint64_t bar[3];
+  const int grp = threadIdx.x >> 8, tid = threadIdx.x & (NT - 1);
+  const int hi = tid >> 4, lo = tid & 15;
+  const int S = a.S, h = a.h;
+  double* sR = base + grp * 2 * PLANE;
+  double* sI = sR + PLANE;
+  if (threadIdx.x == 0) {
+    tma::mbar_init(&bar[0], 1);
+    tma::mbar_init(&bar[1], 1);
+    tma::mbar_init(&bar[2], 1);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {   // S_T once per launch (planes are 4096 doubles each, contiguous re | im)
+    tma::mbar_expect_tx(&bar[2], 2u * PLANE * 8u);
+    tma::load_bulk(base + 4 * PLANE, a.Sre, PLANE * 8u, &bar[2]);
+    tma::load_bulk(base + 5 * PLANE, a.Sim, PLANE * 8u, &bar[2]);
+  }
+  const int64_t stride = 2 * (int64_t)gridDim.x;
+  const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
+  auto issue = [&](int64_t p) {
+    const PairGeom g = pair_geom(a, p);
+    tma::mbar_expect_tx(&bar[grp], (g.has_b ? 2u : 1u) * PLANE * 8u);
+    tma::load_3d(sR, &tm, (int)g.oa2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
+    if (g.has_b) tma::load_3d(sI, &tm, (int)g.ob2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
+  };
+  if (TMA && tid == 0 && p0 < a.win.p_end) issue(p0);
+  tma::mbar_wait(&bar[2], 0);
+
+  uint32_t parity = 0;
+  for (int64_t p = p0; p < a.win.p_end; p += stride) {
+    const PairGeom g = pair_geom(a, p);
+    if (TMA) {
+      tma::mbar_wait(&bar[grp], parity);
+      parity ^= 1;
+      if (!g.has_b) {
+        for (int e = tid; e < PLANE; e += NT) sI[e] = 0.0;
+        group_sync(grp);
+      }
+    } else {
+      for (int e = tid; e < 2 * PLANE; e += NT) {
+        const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
+        int64_t g0 = g.o0 + l0, g1 = g.o1 + l1, g2 = (t ? g.ob2 : g.oa2) + l2;
+        if (WRAP) { g0 = wrap_index(g0, a.n0); g1 = wrap_index(g1, a.n1); g2 = wrap_index(g2, a.n2); }
+        const int64_t lg0 = g0 - a.win.g0;
+        const bool valid = (t == 0 || g.has_b) && g0 < a.n0 && lg0 >= 0 && lg0 < a.win.gn && g1 >= 0 && g1 < a.n1 &&
+                           g2 >= 0 && g2 < a.n2;
+        cp_async8((t ? sI : sR) + wofs(l0, l1, l2), valid ? a.src + (lg0 * a.n1 + g1) * a.n2 + g2 : a.src, valid);
+      }
+      asm volatile("cp.async.commit_group;\n" ::);
+      asm volatile("cp.async.wait_all;\n" ::: "memory");
+      group_sync(grp);
+    }
+    double xr[16], xi[16];
+    // ---- P1: forward axis 2 (thread = row (l0, l1) = (hi, lo)) ----
+    load_row(sR, sI, hi, lo, xr, xi);
+    radix::fft16<false>(xr, xi);
+    store_row(sR, sI, hi, lo, xr, xi);
+    __syncwarp();
+    // ---- P2: forward axis 1 (thread = (l0, l2) = (hi, lo)); same planes as the warp's P1 rows ----
+    {
+      const int b = hi << 8;
+#pragma unroll
+      for (int l1 = 0; l1 < 16; ++l1) {
+        const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
+        xr[l1] = sR[o];
+        xi[l1] = sI[o];
+      }
+      radix::fft16<false>(xr, xi);
+#pragma unroll
+      for (int l1 = 0; l1 < 16; ++l1) {
+        const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
+        sR[o] = xr[l1];
+        sI[o] = xi[l1];
+      }
+    }
+    group_sync(grp);
+    // ---- P3: forward axis 0, * S_T, inverse axis 0 (thread = (k1, k2) = (hi, lo)) ----
+    {
+      const int b = wofs(0, hi, lo);
+#pragma unroll
+      for (int l0 = 0; l0 < 16; ++l0) {
+        xr[l0] = sR[b + (l0 << 8)];
+        xi[l0] = sI[b + (l0 << 8)];
+      }
+      radix::fft16<false>(xr, xi);
+#pragma unroll
+      for (int k0 = 0; k0 < 16; ++k0) radix::cmul(xr[k0], xi[k0], sSr[(k0 << 8) + tid], sSi[(k0 << 8) + tid]);
+      radix::fft16<true>(xr, xi);
+#pragma unroll
+      for (int l0 = 0; l0 < 16; ++l0)
+        if (l0 >= h && l0 < h + S) {
+          sR[b + (l0 << 8)] = xr[l0];
+          sI[b + (l0 << 8)] = xi[l0];
+        }
+    }
+    group_sync(grp);
+    // ---- P4: inverse axis 1 on the S output planes (thread = (l0 - h, l2)) ----
+    if (hi < S) {
+      const int b = (h + hi) << 8;
+#pragma unroll
+      for (int l1 = 0; l1 < 16; ++l1) {
+        const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
+        xr[l1] = sR[o];
+        xi[l1] = sI[o];
+      }
+      radix::fft16<true>(xr, xi);
+#pragma unroll
+      for (int l1 = 0; l1 < 16; ++l1)
+        if (l1 >= h && l1 < h + S) {
+          const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
+          sR[o] = xr[l1];
+          sI[o] = xi[l1];
+        }
+    }
+    __syncwarp();
+    // ---- P5: inverse axis 2 on the output rows (thread = (l0 - h, l1 - h)), same planes as P4 ----
+    const bool p5 = hi < S && lo < S;
+    if (p5) load_row(sR, sI, h + hi, h + lo, xr, xi);
+    // the buffer is free: order this thread's shared accesses before the next TMA write, then
+    // refill it while the last transform and the stores run
+    if (TMA) tma::fence_proxy_async();
+    group_sync(grp);
+    if (TMA && tid == 0 && p + stride < a.win.p_end) issue(p + stride);
+    if (p5) {
+      const int l0 = h + hi, l1 = h + lo;
+      radix::fft16<true>(xr, xi);
+      const int64_t c0 = g.o0 + l0, c1 = g.o1 + l1;
+      if (!(c0 >= a.bd.lim0 || c0 < a.win.w_lo || c0 >= a.win.w_hi || c1 >= a.bd.lim1)) {
+        double* drow = a.dst + ((c0 - a.win.g0) * a.n1 + c1) * a.n2;
+        // 16-byte stores of (l2, l2 + 1) when the row and window are aligned
+        const bool vec = ((g.oa2 | h | a.n2 | S) & 1) == 0 && (reinterpret_cast<uintptr_t>(a.dst) & 15) == 0 &&
+                         g.oa2 + h + S <= a.bd.lim2 && (!g.has_b || g.ob2 + h + S <= a.bd.lim2);
+        if (vec) {
+#pragma unroll
+          for (int l2 = 0; l2 < 16; l2 += 2)
+            if (l2 >= h && l2 < h + S) {
+              *reinterpret_cast<double2*>(drow + g.oa2 + l2) = make_double2(xr[l2], xr[l2 + 1]);
+              if (g.has_b) *reinterpret_cast<double2*>(drow + g.ob2 + l2) = make_double2(xi[l2], xi[l2 + 1]);
+            }
+        } else {
+#pragma unroll
+          for (int l2 = 0; l2 < 16; ++l2)
+            if (l2 >= h && l2 < h + S) {
+              int64_t c2 = g.oa2 + l2;
+              if (c2 < a.bd.lim2) drow[c2] = xr[l2];
+              c2 = g.ob2 + l2;
+              if (g.has_b && c2 < a.bd.lim2) drow[c2] = xi[l2];
+            }
+        }
+      }
+    }
+  }
+}
+
+}  // namespace
+
+// Two group buffers + S_T.
+size_t fused3d_bf_smem(bool) { return (size_t)6 * PLANE * sizeof(double) + kAlign; }
+
+cudaError_t fused3d_bf_configure(int* max_blocks) {
+  const int st = (int)fused3d_bf_smem(true), sc = (int)fused3d_bf_smem(false);
+  cudaError_t e = cudaFuncSetAttribute(fft3d_bf_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, st);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(fft3d_bf_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft3d_bf_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_bf_kernel<true>, 2 * NT, st);
+}
+
+cudaError_t launch_fused3d_bf(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s) {
+  static const CUtensorMap none = {};
+  if (tm)
+    fft3d_bf_kernel<true><<<grid, 2 * NT, fused3d_bf_smem(true), s>>>(a, *tm);
+  else if (a.bd.wrap)
+    fft3d_bf_kernel<false, true><<<grid, 2 * NT, fused3d_bf_smem(false), s>>>(a, none);
+  else
+    fft3d_bf_kernel<false><<<grid, 2 * NT, fused3d_bf_smem(false), s>>>(a, none);
+  return cudaGetLastError();
+}
+
+}  // namespace fstencil

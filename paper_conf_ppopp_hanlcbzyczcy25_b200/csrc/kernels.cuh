@@ -153,6 +153,20 @@ cudaError_t fused3d_ct_configure(int* max_blocks_per_sm);
 // tm: tensor map of the source buffer (dims {n2, n1, gn}, box {16, 16, 16}) or null (cp.async).
 cudaError_t launch_fused3d_ct(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
 
+// Radix-8 ALU engine of the factored 2D tile (kernel_fft2d_bf.cu): 64 = 8 x 8 Cooley-Tukey with
+// DFT-8 butterflies in registers.  Fre/Fim[0..63] = w64^m; Sre/Sim = S_T in position order
+// (position 8a + b <-> frequency a + 8b per axis).  tm: dims {n1, gn}, box {16, 64}, SWIZZLE_128B.
+size_t fused2d_bf_smem(bool tma);
+cudaError_t fused2d_bf_configure(int* max_blocks_per_sm);
+cudaError_t launch_fused2d_bf(const Fft2dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
+
+// Radix-4 ALU engine of the factored 3D tile (kernel_fft3d_bf.cu): 16-point line FFTs in
+// registers; Sre/Sim = S_T in natural [k0][k1][k2] order.  tm: as for fft3d_ct but encoded with
+// SWIZZLE_128B.
+size_t fused3d_bf_smem(bool tma);
+cudaError_t fused3d_bf_configure(int* max_blocks_per_sm);
+cudaError_t launch_fused3d_bf(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
+
 constexpr int kBandThreads = 256;
 cudaError_t band_configure(size_t smem);
 cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s);

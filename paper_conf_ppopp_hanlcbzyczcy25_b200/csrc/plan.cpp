@@ -3,6 +3,8 @@
 #include "plan.h"
 
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
 #include <cmath>
 #include <complex>
 
@@ -72,6 +74,17 @@ double model_flops_2d_ct(int S, int T) {
 
 static constexpr double kEffCt = 0.70;   // assumed until measured (profiles/)
 
+// Radix-8 ALU engine (kernel_fft2d_bf.cu), per pair: DFT-8 chunks of 56 instructions/flops --
+// 512 in each of R1, R2, C1, C3, 1024 in C2, 8 S in each of R3, R4 -- twiddled chunks (7 complex
+// multiplies of 6 flops / 4 instructions: R1, C1, C2, R3) and S_T (one complex multiply per
+// element).
+static double chunks_2d_bf(int S) { return 3072.0 + 16.0 * S; }
+static double tw_chunks_2d_bf(int S) { return 1536.0 + 8.0 * S; }
+static double flops_pair_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 42.0 * tw_chunks_2d_bf(S) + 6.0 * 4096.0; }
+static double alu_ops_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 28.0 * tw_chunks_2d_bf(S) + 4.0 * 4096.0; }
+static double model_flops_2d_bf(int S, int T) { return flops_pair_2d_bf(S) / (2.0 * S * (double)S * T); }
+static constexpr double kEff2dBf = 0.35;   // flops per FP64-pipe slot-flop x pipe efficiency (assumed)
+
 // Measured DMMA issue efficiency of the fused 2D kernel per tile side (fraction of the
 // 37.18 TF/s peak, B200, profiles/r01_sweep.txt / r01_variants.txt): the plan minimises
 // executed flops / efficiency, i.e. predicted time per cell-step (the role of Eq. 5's
@@ -95,6 +108,25 @@ static double groups_3d_ct(int S) { return 256.0 + 4.0 * S + S * (double)((S + 3
 static double model_flops_3d_ct(int S, int T) {
   return ((prod_flops(kCmul3_3d) + 320.0) * groups_3d_ct(S) + 6.0 * 4096.0) / (2.0 * S * (double)S * S * T);
 }
+// Radix-4 ALU engine (kernel_fft3d_bf.cu), per pair: 16-point line FFTs -- 256 per forward
+// axis, 256 inverse axis 0, 16 S inverse axis 1, S^2 inverse axis 2 -- of 168 flops
+// (160 FP64 instructions, fft_radix.cuh) each, + S_T (6 flops, 4 instructions per element).
+static double lines_3d_bf(int S) { return 1024.0 + 16.0 * S + (double)S * S; }
+static double model_flops_3d_bf(int S, int T) {
+  return (168.0 * lines_3d_bf(S) + 6.0 * 4096.0) / (2.0 * S * (double)S * S * T);
+}
+static double alu_ops_3d_bf(int S) { return 160.0 * lines_3d_bf(S) + 4.0 * 4096.0; }
+// Relative cost of one executed flop on the ALU engine vs a DMMA flop: both share the FP64
+// pipe (profiles/r01_fp64_shared.txt); adds cost a full FMA slot (~0.55 flop per slot-flop)
+// and the passes are shared-memory heavy -- assumed until measured.
+static constexpr double kEff3dBf = 0.45;
+// FFTSTENCIL_ENGINE=dmma|alu pins the line engine of the factored 2D and 3D tiles (ablation);
+// default alu.
+static int env_engine() {
+  const char* v = std::getenv("FFTSTENCIL_ENGINE");
+  if (v && !std::strcmp(v, "dmma")) return 0;
+  return 1;
+}
 static constexpr double kEff3d = 0.70;     // dense 3D: executed DMMA efficiency (profiles/r01_sweep.txt)
 static constexpr double kEff3dCt = 0.60;   // factored 3D: assumed until measured
 
@@ -115,6 +147,8 @@ static constexpr double kEff1d = 0.73;     // PFA 8x7: executed DMMA efficiency 
 static double flops_pair_1d_ct() { return kProdFlops * 512.0 + 6.0 * 7.0 * 4096.0; }
 static double model_flops_1d_ct(int S, int T) { return flops_pair_1d_ct() / (2.0 * S * (double)T); }
 static constexpr double kEff1dCt = 0.70;   // assumed until measured
+
+static int env_engine();
 
 int build_host_plan(int ndim, const int64_t* extents, const double* weights, int radius, int T,
                     HostPlan& p, std::string& err, int nranks, int rank, int algo, int periodic) {
@@ -184,8 +218,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   } else if (ndim == 2) {
     // candidates: dense L x L DFT tiles and the factored 64 = 8 x 8 tile (NEXT-1)
     static const int cand[] = {16, 24, 32, 40, 48, 56, 64};
+    const int engine = env_engine();
     auto cost = [&](int al, int L, int S, int t) {
-      return al ? model_flops_2d_ct(S, t) / kEffCt : model_flops_2d(L, S, t) / eff_2d(L);
+      return al ? (engine ? model_flops_2d_bf(S, t) / kEff2dBf : model_flops_2d_ct(S, t) / kEffCt)
+                : model_flops_2d(L, S, t) / eff_2d(L);
     };
     double best = 1e300;
     int bL = 0, bT = 0, bA = 0;
@@ -221,6 +257,12 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       const double Sp = round8(p.S[0]);
       p.mma_flops_per_pair = 8.0 * (2.0 * L * L * L + Sp * L * L + Sp * Sp * L);
       p.fused_smem = (size_t)(bL >= 56 ? 48 : 32) * bL * (bL + 4);   // F + pair buffer(s)
+    } else if (engine) {
+      p.engine = 1;
+      p.flops_per_cell_step = model_flops_2d_bf(p.S[0], bT);
+      p.mma_flops_per_pair = 0;
+      p.alu_ops_per_pair = alu_ops_2d_bf(p.S[0]);
+      p.fused_smem = (size_t)6 * 64 * 64 * sizeof(double) + 64 * 16 + 1024;   // 2 pair buffers + S_T + w64
     } else {
       p.flops_per_cell_step = model_flops_2d_ct(p.S[0], bT);
       p.mma_flops_per_pair = kProdDmmaFlops * products_2d_ct(p.S[0]);
@@ -232,6 +274,7 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     const int hmax = std::min(hmax_grid, (L - 2) / 2);
     const int tmax = hmax / radius;
     if (tmax < 1) { err = "radius too large for the 16^3 3D tile"; return FFTSTENCIL_EINVAL; }
+    const int engine = env_engine();
     double best = 1e300;
     int bestT = 1, bA = 0;
     for (int t = 1; t <= tmax; ++t) {
@@ -239,7 +282,8 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       for (int al = 0; al < 2; ++al) {
         if (algo >= 0 && al != algo) continue;
         const int S = L - 2 * radius * t;
-        const double f = al ? model_flops_3d_ct(S, t) / kEff3dCt : model_flops_3d(L, S, t) / kEff3d;
+        const double f = !al ? model_flops_3d(L, S, t) / kEff3d
+                         : engine ? model_flops_3d_bf(S, t) / kEff3dBf : model_flops_3d_ct(S, t) / kEff3dCt;
         if (f < best) { best = f; bestT = t; bA = al; }
       }
     }
@@ -258,6 +302,12 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       const double mt = Sp / 8.0;
       p.mma_flops_per_pair = 512.0 * (16 * 128 + 32 * (32 + 16 * mt) + S * (64 * mt + 16 * mt * mt));
       p.fused_smem = (size_t)(2 * 16 * 20 + 2 * 16 * (16 * 20 + 4)) * sizeof(double);
+    } else if (engine) {
+      p.engine = 1;
+      p.flops_per_cell_step = model_flops_3d_bf(p.S[0], bestT);
+      p.mma_flops_per_pair = 0;
+      p.alu_ops_per_pair = alu_ops_3d_bf(p.S[0]);
+      p.fused_smem = (size_t)6 * 16 * 16 * 16 * sizeof(double) + 1024;   // 2 pair buffers + S_T
     } else {
       p.flops_per_cell_step = model_flops_3d_ct(p.S[0], bestT);
       p.mma_flops_per_pair = prod_dmma_flops(kCmul3_3d) * groups_3d_ct(p.S[0]);
@@ -361,6 +411,15 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       p.Fre[64 + k] = v.real();
       p.Fim[64 + k] = v.imag();
     }
+  } else if (ndim == 2 && p.algo == 1 && p.engine == 1) {
+    // w64^m, m = 0..63 (kernel_fft2d_bf.cu twiddle table)
+    p.Fre.assign(128, 0.0);
+    p.Fim.assign(128, 0.0);
+    for (int m = 0; m < 64; ++m) {
+      const cplx v = root(m, 64);
+      p.Fre[m] = v.real();
+      p.Fim[m] = v.imag();
+    }
   } else if (ndim == 2 && p.algo == 1) {
     // [F8 | twiddles w64^(ka lb)], 8 x 8 each (kernel_fft2d_ct.cu)
     p.Fre.assign(128, 0.0);
@@ -426,6 +485,8 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
           // factored 1D: k = c + 64 d at [c][8 (d % 8) + d / 8] (row c, CT digit order of d)
           const int64_t c = i % 64, d = i / 64;
           dst = c * 64 + 8 * (d % 8) + d / 8;
+        } else if (ndim == 3 && p.algo == 1 && p.engine == 1) {
+          // radix-4 ALU engine: natural [k0][k1][k2]
         } else if (ndim == 3 && p.algo == 1) {
           // factored 3D: [k1][k2][k0 % 8][k0 / 8] (the thread-local DFT-2 output pair)
           const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
@@ -433,6 +494,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         } else if (ndim == 3) {
           const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
           dst = k12 * L + k0;
+        } else if (p.algo == 1 && p.engine == 1) {
+          // radix-8 ALU engine: position order on both axes, position 8a + b <-> frequency a + 8b
+          const int64_t k0 = i / 64, k1 = i % 64;
+          dst = (8 * (k0 % 8) + k0 / 8) * 64 + 8 * (k1 % 8) + k1 / 8;
         } else if (p.algo == 1) {
           // factored 2D: [k1][8 g + c] holds k0 = g + 8 c (digit order of the CT output)
           const int64_t k0 = i / 64, k1 = i % 64;

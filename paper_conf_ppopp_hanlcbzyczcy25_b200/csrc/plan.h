@@ -56,6 +56,10 @@ struct HostPlan {
   int algo = 0;                    // 0 dense DFT GEMMs (1D: PFA 8x7), 1 factored (1D 64x64 CT, 2D CT 8x8, 3D 8x2),
                                    // 2 unfused 2D ablation
   int periodic = 0;                // 1: periodic boundary (no ring/band, wrap-around tiles)
+  int engine = 0;                  // line-DFT engine of the factored 3D tile: 0 DFT-8 GEMMs on the
+                                   // FP64 tensor pipe (kernel_fft3d_ct.cu), 1 radix-4 FFTs on the
+                                   // FP64 ALU (kernel_fft3d_bf.cu); FFTSTENCIL_ENGINE=dmma|alu
+  double alu_ops_per_pair = 0;     // FP64 ALU instructions per pair (engine 1: adds, muls, FMAs)
   int64_t nt[3] = {1, 1, 1};       // tiles per user axis
   int64_t tiles = 0, pairs = 0;
   int64_t npr = 1;                 // pairs per outer tile row (2D) / tile line (3D)

@@ -58,10 +58,21 @@ __device__ __forceinline__ void load_3d(void* smem_dst, const CUtensorMap* map, 
       : "memory");
 }
 
+// 1D bulk copy of `bytes` (multiple of 16; both addresses 16-byte aligned) global -> shared.
+__device__ __forceinline__ void load_bulk(void* smem_dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(smem_addr(smem_dst)),
+      "l"(reinterpret_cast<uint64_t>(src)), "r"(bytes), "r"(smem_addr(bar))
+      : "memory");
+}
+
 }  // namespace tma
 
 // Host: encode a row-major FP64 tensor map (rank 2 or 3; dims/box innermost first).
 // Returns false if TMA cannot describe it (alignment) or the driver entry point is missing.
-bool encode_tensor_map(CUtensorMap* map, const void* base, int rank, const uint64_t* dims, const uint32_t* box);
+// swizzle128: CU_TENSOR_MAP_SWIZZLE_128B (16-byte chunk c of each 128-byte box row r lands at
+// chunk c ^ (r & 7); the destination must be 1024-byte aligned, the inner box 128 bytes).
+bool encode_tensor_map(CUtensorMap* map, const void* base, int rank, const uint64_t* dims, const uint32_t* box,
+                       bool swizzle128 = false);
 
 }  // namespace fstencil

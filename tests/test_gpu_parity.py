@@ -438,3 +438,44 @@ def test_periodic_plane_wave_1d_long(fs):
     torch.cuda.synchronize()
     ref = np.real(sig ** steps * np.exp(1j * th * c))
     assert np.abs(b.cpu().numpy() - ref).max() <= 1e-9
+
+
+CASES_3D = [c for c in CASES if len(c[0]) == 3]
+
+
+@pytest.mark.parametrize("engine,tma", [("dmma", "1"), ("alu", "1"), ("alu", "0")])
+@pytest.mark.parametrize("ext,shape,r,T,steps,kind", CASES_3D)
+def test_parity_3d_engines(fs, monkeypatch, engine, tma, ext, shape, r, T, steps, kind):
+    """Both line-DFT engines of the factored 3D tile (DFT-8 GEMMs on DMMA; radix-4 FFTs on the
+    FP64 ALU, TMA-swizzled and cp.async staging) against the oracle."""
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "factored")
+    monkeypatch.setenv("FFTSTENCIL_ENGINE", engine)
+    monkeypatch.setenv("FFTSTENCIL_TMA", tma)
+    w = wl.stencil_weights(shape, len(ext), r, kind)
+    u0 = wl.grid(ext, 12)
+    got, p = run_gpu(fs, u0, w, r, T, steps)
+    assert p.info()["engine"] == engine
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(got, ref) <= TOL, (rel_err(got, ref), p.info())
+
+
+CASES_2D = [c for c in CASES if len(c[0]) == 2]
+
+
+@pytest.mark.parametrize("engine,tma", [("dmma", "1"), ("alu", "1"), ("alu", "0")])
+@pytest.mark.parametrize("ext,shape,r,T,steps,kind", CASES_2D)
+def test_parity_2d_engines(fs, monkeypatch, engine, tma, ext, shape, r, T, steps, kind):
+    """Both line-DFT engines of the factored 2D tile (DFT-8 GEMMs on DMMA; radix-8 butterflies on
+    the FP64 ALU, TMA-swizzled and cp.async staging) against the oracle."""
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "factored")
+    monkeypatch.setenv("FFTSTENCIL_ENGINE", engine)
+    monkeypatch.setenv("FFTSTENCIL_TMA", tma)
+    w = wl.stencil_weights(shape, len(ext), r, kind)
+    u0 = wl.grid(ext, 13)
+    try:
+        got, p = run_gpu(fs, u0, w, r, T, steps)
+    except Exception as e:   # a tile too small for the requested T: the factored 64-tile needs S >= 8
+        pytest.skip(str(e))
+    assert p.info()["engine"] == engine
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(got, ref) <= TOL, (rel_err(got, ref), p.info())

@@ -52,7 +52,16 @@ def dense(monkeypatch):
 
 @pytest.fixture
 def factored(monkeypatch):
+    """The factored tile with its DFT-8-GEMM (DMMA) line engine."""
     monkeypatch.setenv("FFTSTENCIL_ALGO", "factored")
+    monkeypatch.setenv("FFTSTENCIL_ENGINE", "dmma")
+
+
+@pytest.fixture
+def alu(monkeypatch):
+    """The factored tile with its radix butterfly (FP64 ALU) line engine (the default)."""
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "factored")
+    monkeypatch.setenv("FFTSTENCIL_ENGINE", "alu")
 
 
 @pytest.mark.parametrize("r,T,L", [(1, 8, 48), (1, 1, 16), (1, 4, 24), (3, 4, 64)])
@@ -397,3 +406,96 @@ def test_factored_1d_four_step_model_matches_oracle(factored, r, T):
 def test_factored_1d_tiles_band_ring_partition(factored, ext, r, T):
     count, h = _cover(ext, r, T, "star")
     assert count.min() == 1 and count.max() == 1
+
+
+# ---------------------------------------------------------------- ALU engine (radix butterflies) tables
+def test_alu_engine_is_the_default_for_2d_and_3d():
+    for ext, shape, r in (((10240, 10240), "star", 1), ((1024, 1024, 1024), "star", 1)):
+        info = fs.describe(ext, wl.seeded_weights(shape, len(ext), r), r, 0)
+        assert info["algo"] == "factored" and info["engine"] == "alu", info
+        assert info["mma_flops_per_pass"] == 0 and info["alu_ops_per_pass"] > 0
+
+
+def test_alu_w64_table_vs_numpy(alu):
+    w = wl.seeded_weights("box", 2, 1)
+    v = fs.export_aux((1000, 1000), w, 1, 8, which=0, axis=0)
+    tw = v[0::2] + 1j * v[1::2]
+    np.testing.assert_allclose(tw, np.fft.fft(np.eye(64)[1]), atol=1e-15)   # w64^m = exp(-2 pi i m / 64)
+
+
+def _pos(m):
+    """Position of frequency m on an axis of the radix-8 engine: p = 8 (m % 8) + m // 8."""
+    return 8 * (m % 8) + m // 8
+
+
+@pytest.mark.parametrize("shape,r,T", [("box", 1, 8), ("star", 3, 4)])
+def test_alu_2d_spectrum_position_order(alu, shape, r, T):
+    w = wl.seeded_weights(shape, 2, r)
+    info = fs.describe((3000, 3000), w, r, T)
+    for t in (1, info["T"]):
+        v = fs.export_aux((3000, 3000), w, r, T, which=1, t=t)
+        G = (v[0::2] + 1j * v[1::2]).reshape(64, 64)
+        ref = spectrum.powered_spectrum(w, r, (64, 64), t)    # [k0][k1], 1/4096 folded in
+        m = np.arange(64)
+        np.testing.assert_allclose(G[np.ix_(_pos(m), _pos(m))], ref, atol=1e-15)
+
+
+def test_alu_3d_spectrum_natural_order(alu):
+    w = wl.seeded_weights("box", 3, 1)
+    v = fs.export_aux((200, 200, 200), w, 1, 2, which=1, t=2)
+    G = (v[0::2] + 1j * v[1::2]).reshape(16, 16, 16)
+    np.testing.assert_allclose(G, spectrum.powered_spectrum(w, 1, (16, 16, 16), 2), atol=1e-15)
+
+
+def _dft8(x, axis, inverse=False):
+    """DFT-8 along `axis` (numpy's definition; conj kernel unnormalised for the inverse)."""
+    return np.fft.ifft(x, axis=axis) * 8 if inverse else np.fft.fft(x, axis=axis)
+
+
+def _alu_2d_tile(Z, tw, Sp, h, S):
+    """The radix-8 engine's seven stages on one complex 64 x 64 tile, index for index
+    (kernel_fft2d_bf.cu): positions 8 a + b, twiddles from the exported w64 table."""
+    W = lambda e: tw[np.mod(e, 64)]
+    j = np.arange(8)
+    X = Z.reshape(64, 8, 8).copy()                              # [r][n1][n2]: column 8 n1 + n2
+    # R1: DFT-8 over n1, * w64^(n2 k1)                           -> [r][k1][n2]
+    X = _dft8(X, 1) * W(np.outer(j, j))[None]
+    # R2: DFT-8 over n2 -> column 8 k1 + k2 holds frequency k1 + 8 k2
+    X = _dft8(X, 2).reshape(64, 64)
+    Y = X.reshape(8, 8, 64)                                      # [n1][n2][c]: row 8 n1 + n2
+    # C1: DFT-8 over n1, * w64^(n2 k1)                           -> [k1][n2][c]
+    Y = _dft8(Y, 0) * W(np.outer(j, j))[:, :, None]
+    # C2: DFT-8 over n2 (-> k2), * S at position (8 k1 + k2, c), IDFT-8 over k2, * conj w64^(n2 k1)
+    Y = _dft8(Y, 1) * Sp.reshape(8, 8, 64)
+    Y = _dft8(Y, 1, inverse=True) * np.conj(W(np.outer(j, j)))[:, :, None]
+    # C3: IDFT-8 over k1 -> rows 8 n1 + n2
+    Y = _dft8(Y, 0, inverse=True).reshape(64, 64)[h:h + S]
+    # R3: IDFT-8 over k2 (columns 8 k1 + k2), * conj w64^(n2 k1); R4: IDFT-8 over k1
+    R = Y.reshape(S, 8, 8)                                       # [r][k1][k2]
+    R = _dft8(R, 2, inverse=True) * np.conj(W(np.outer(j, j)))[None]
+    R = _dft8(R, 1, inverse=True).reshape(S, 64)                 # column 8 n1 + n2
+    return R[:, h:h + S]
+
+
+@pytest.mark.parametrize("shape,r,T", [("box", 1, 11), ("star", 3, 4), ("box", 2, 5)])
+def test_alu_2d_stage_model_vs_overlap_save(alu, shape, r, T):
+    """The stage sequence with the exported tables equals the tile's T-step circular
+    convolution (ifft2(fft2(x) sigma^T)) on the valid window, for two packed real tiles."""
+    w = wl.seeded_weights(shape, 2, r)
+    ext = (3000, 3000)
+    info = fs.describe(ext, w, r, T)
+    h, S, T = info["halo"], info["valid"][0], info["T"]
+    v = fs.export_aux(ext, w, r, T, which=0, axis=0)
+    tw = v[0::2] + 1j * v[1::2]
+    v = fs.export_aux(ext, w, r, T, which=1, t=T)
+    Sp = (v[0::2] + 1j * v[1::2]).reshape(64, 64)
+    rng = np.random.default_rng(5)
+    xa, xb = rng.random((64, 64)), rng.random((64, 64))
+    got = _alu_2d_tile(xa + 1j * xb, tw, Sp, h, S)
+    sig = spectrum.powered_spectrum(w, r, (64, 64), T) * 4096
+    for x, part in ((xa, got.real), (xb, got.imag)):
+        ref = np.fft.ifft2(np.fft.fft2(x) * sig).real[h:h + S, h:h + S]
+        np.testing.assert_allclose(part, ref, atol=1e-12)
+        # and the direct-stencil oracle on the tile (valid window = exact T-step result)
+        direct = oracle.stencil_run(np.pad(x, 0), w, r, T, periodic=True)[h:h + S, h:h + S]
+        np.testing.assert_allclose(part, direct, atol=1e-11)
