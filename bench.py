@@ -135,7 +135,8 @@ def load_traffic(info: dict, workload: str):
         with open(path) as f:
             d = json.load(f)
         e = d.get(workload)
-        if e and e.get("T") == info["T"] and e.get("tile") == info["tile"]:
+        if (e and e.get("T") == info["T"] and e.get("tile") == info["tile"]
+                and e.get("engine", "dmma") == info.get("engine", "dmma")):
             return float(e["dram_bytes_per_launch"])
     except Exception:
         pass

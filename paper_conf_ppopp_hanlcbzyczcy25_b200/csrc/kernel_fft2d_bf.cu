@@ -56,6 +56,35 @@ __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool v
 using radix::cmul;
 using radix::fft8;
 
+// Tuning switches (ablation builds via FFTSTENCIL_NVCC_DEFS): BF_TW_POW = 0 twiddles from the
+// shared table, 1 the lane-varying R1 twiddles as powers of w64^n2 in registers, 2 every twiddle
+// as powers (default: +6% on B200, fewer shared-memory wavefronts and no spills,
+// profiles/r01_s2_ab2d.txt); BF_UNROLL = chunks per thread in flight in the column/row-b stages.
+#ifndef BF_TW_POW
+#define BF_TW_POW 2
+#endif
+#ifndef BF_UNROLL
+#define BF_UNROLL 1
+#endif
+constexpr int kUnroll = BF_UNROLL;
+
+// x[j] *= w^(+-j) for j = 1..7 with w = (wr, wi) = w64^t: powers by repeated multiplication
+// (6 complex multiplies; error ~ j ulp).
+template <bool INV>
+__device__ __forceinline__ void twiddle_pow(double (&xr)[8], double (&xi)[8], double wr, double wi) {
+  if (INV) wi = -wi;
+  double pr = wr, pi = wi;
+#pragma unroll
+  for (int j = 1; j < 8; ++j) {
+    cmul(xr[j], xi[j], pr, pi);
+    if (j < 7) {
+      const double t = pr * wr - pi * wi;
+      pi = fma(pr, wi, pi * wr);
+      pr = t;
+    }
+  }
+}
+
 // twiddle x[j] *= w64^(+-t j), j = 1..7; tw[8 j + t] = w64^(j t) (shared, 1 KB): a warp-uniform
 // t is a broadcast, t = lane & 7 hits 8 distinct 16-byte chunks per quarter-warp.
 template <bool INV>
@@ -114,7 +143,7 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
   const int S = a.S, h = a.h;
   // ---- R1: rows, stage a; chunk (r, n2), n2 = lane & 7; a half-warp covers rows r0, r0 + 4
   // (8-byte words ((8 n1 + n2) & 15) ^ 2 (r & 7): the two rows land in opposite bank halves) ----
-#pragma unroll 1
+#pragma unroll kUnroll
   for (int u = 0; u < 2; ++u) {
     const int r = row_of(warp, lane, u), n2 = lane & 7;
     double xr[8], xi[8];
@@ -125,7 +154,12 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
       xi[n1] = sI[o];
     }
     fft8<false>(xr, xi);
-    twiddle_chunk<false>(xr, xi, tw, n2);
+    if (BF_TW_POW >= 1) {
+      const double2 w = tw[8 + n2];   // w64^n2
+      twiddle_pow<false>(xr, xi, w.x, w.y);
+    } else {
+      twiddle_chunk<false>(xr, xi, tw, n2);
+    }
 #pragma unroll
     for (int k1 = 0; k1 < 8; ++k1) {
       const int o = wd(r, 8 * k1 + n2);
@@ -135,7 +169,7 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
   }
   group_sync(grp);
   // ---- R2: rows, stage b; chunk (r, k1): columns 8 k1 + n2 (4 x 16-byte words) ----
-#pragma unroll 1
+#pragma unroll kUnroll
   for (int u = 0; u < 2; ++u) {
     const int task = warp + NW * u, r = lane + 32 * (task & 1), k1 = task >> 1;
     double xr[8], xi[8];
@@ -156,7 +190,7 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
   }
   group_sync(grp);
   // ---- C1: columns, stage a; chunk (c, n2): rows 8 n1 + n2 ----
-#pragma unroll 1
+#pragma unroll kUnroll
   for (int u = 0; u < 2; ++u) {
     const int task = warp + NW * u, c = lane + 32 * (task & 1), n2 = task >> 1;
     double xr[8], xi[8];
@@ -167,7 +201,12 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
       xi[n1] = sI[o];
     }
     fft8<false>(xr, xi);
-    twiddle_chunk<false>(xr, xi, tw, n2);
+    if (BF_TW_POW >= 2) {
+      const double2 w = tw[8 + n2];
+      twiddle_pow<false>(xr, xi, w.x, w.y);
+    } else {
+      twiddle_chunk<false>(xr, xi, tw, n2);
+    }
 #pragma unroll
     for (int k1 = 0; k1 < 8; ++k1) {
       const int o = wd(8 * k1 + n2, c);
@@ -177,7 +216,7 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
   }
   group_sync(grp);
   // ---- C2: columns, stage b, * S_T, inverse stage b; chunk (c, k1): rows 8 k1 + n2 ----
-#pragma unroll 1
+#pragma unroll kUnroll
   for (int u = 0; u < 2; ++u) {
     const int task = warp + NW * u, c = lane + 32 * (task & 1), k1 = task >> 1;
     double xr[8], xi[8];
@@ -194,7 +233,12 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
       cmul(xr[k2], xi[k2], sSr[so], sSi[so]);
     }
     fft8<true>(xr, xi);    // slot n2
-    twiddle_chunk<true>(xr, xi, tw, k1);
+    if (BF_TW_POW >= 2) {
+      const double2 w = tw[8 + k1];
+      twiddle_pow<true>(xr, xi, w.x, w.y);
+    } else {
+      twiddle_chunk<true>(xr, xi, tw, k1);
+    }
 #pragma unroll
     for (int n2 = 0; n2 < 8; ++n2) {
       const int o = wd(8 * k1 + n2, c);
@@ -204,7 +248,7 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
   }
   group_sync(grp);
   // ---- C3: columns, inverse stage a; chunk (c, n2): rows 8 k1 + n2 -> rows 8 n1 + n2 (S kept) ----
-#pragma unroll 1
+#pragma unroll kUnroll
   for (int u = 0; u < 2; ++u) {
     const int task = warp + NW * u, c = lane + 32 * (task & 1), n2 = task >> 1;
     double xr[8], xi[8];
@@ -241,7 +285,12 @@ __device__ __forceinline__ void tile_stages(double* sR, double* sI, const double
         xr[2 * j] = vr.x; xr[2 * j + 1] = vr.y; xi[2 * j] = vi.x; xi[2 * j + 1] = vi.y;
       }
       fft8<true>(xr, xi);
-      twiddle_chunk<true>(xr, xi, tw, k1);
+      if (BF_TW_POW >= 2) {
+        const double2 w = tw[8 + k1];
+        twiddle_pow<true>(xr, xi, w.x, w.y);
+      } else {
+        twiddle_chunk<true>(xr, xi, tw, k1);
+      }
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         const int o = wd(r, 8 * k1 + 2 * j);

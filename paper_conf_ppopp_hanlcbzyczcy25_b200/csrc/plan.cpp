@@ -75,13 +75,13 @@ double model_flops_2d_ct(int S, int T) {
 static constexpr double kEffCt = 0.70;   // assumed until measured (profiles/)
 
 // Radix-8 ALU engine (kernel_fft2d_bf.cu), per pair: DFT-8 chunks of 56 instructions/flops --
-// 512 in each of R1, R2, C1, C3, 1024 in C2, 8 S in each of R3, R4 -- twiddled chunks (7 complex
-// multiplies of 6 flops / 4 instructions: R1, C1, C2, R3) and S_T (one complex multiply per
-// element).
+// 512 in each of R1, R2, C1, C3, 1024 in C2, 8 S in each of R3, R4 -- twiddled chunks (R1, C1,
+// C2, R3: 7 complex multiplies by w^j plus the 6 that form the powers w^2..w^7 of w = w64^t,
+// 6 flops / 4 instructions each) and S_T (one complex multiply per element).
 static double chunks_2d_bf(int S) { return 3072.0 + 16.0 * S; }
 static double tw_chunks_2d_bf(int S) { return 1536.0 + 8.0 * S; }
-static double flops_pair_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 42.0 * tw_chunks_2d_bf(S) + 6.0 * 4096.0; }
-static double alu_ops_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 28.0 * tw_chunks_2d_bf(S) + 4.0 * 4096.0; }
+static double flops_pair_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 78.0 * tw_chunks_2d_bf(S) + 6.0 * 4096.0; }
+static double alu_ops_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 52.0 * tw_chunks_2d_bf(S) + 4.0 * 4096.0; }
 static double model_flops_2d_bf(int S, int T) { return flops_pair_2d_bf(S) / (2.0 * S * (double)S * T); }
 static constexpr double kEff2dBf = 0.35;   // flops per FP64-pipe slot-flop x pipe efficiency (assumed)
 
