@@ -13,14 +13,12 @@
 //   P1 forward axis 2 | P2 forward axis 1 | P3 forward axis 0, * S_T, inverse axis 0 (writes
 //   only the S output planes) | P4 inverse axis 1 on those planes (writes only the S output
 //   rows) | P5 inverse axis 2 on the S x S output rows -> store the S^3 window.
-// Shared layout = the TMA SWIZZLE_128B image of a dense 16^3 box: element (l0, l1, l2) at
-// word 256 l0 + 16 l1 + (l2 ^ 2 (l1 & 7)) (the 16-byte chunk index XOR row mod 8).  Bank
-// check (8-byte words, a half-warp per wavefront; 16-byte words, a quarter-warp):
-//   P1/P5 (thread = (l0, l1), 16-byte loads of chunk c): lanes l1 = 0..7 -> chunks c ^ l1
-//         distinct.  P2/P4 (thread = (l0, l2), element l1 = p): lanes l2 = 0..15 -> words
-//         l2 ^ 2 (p & 7) distinct.  P3 (thread = (l1, l2), element l0 = p): lanes l2 = 0..15
-//         distinct.  All conflict-free except P5's ragged quarter-warps.
-// The spectrum S_T is in natural [k0][k1][k2] order (read coalesced across lanes in P3).
+// Shared layout: the tiles land as the TMA SWIZZLE_128B image of two dense 16^3 boxes (Re and
+// Im planes; element (l0, l1, l2) at word 256 l0 + 16 l1 + (l2 ^ 2 (l1 & 7))); P1 reads each
+// row from both planes (16-byte words, lanes l1 = 0..7 per quarter-warp: conflict-free) and
+// rewrites it in place in an interleaved complex layout (cofs below) that every later pass
+// reads and writes as one 16-byte word per element.  S_T is staged once per launch in shared
+// memory, interleaved, natural [k0][k1][k2] order.
 #include "fft_radix.cuh"
 #include "kernels.cuh"
 #include "tma.cuh"
@@ -53,15 +51,17 @@ __device__ __forceinline__ void load_row(const double* sR, const double* sI, int
     xi[2 * c] = i.x; xi[2 * c + 1] = i.y;
   }
 }
-__device__ __forceinline__ void store_row(double* sR, double* sI, int l0, int l1, const double (&xr)[16],
-                                          const double (&xi)[16]) {
-  const int base = (l0 << 8) | (l1 << 4), s = l1 & 7;
-#pragma unroll
-  for (int c = 0; c < 8; ++c) {
-    const int o = base + ((c ^ s) << 1);
-    *reinterpret_cast<double2*>(sR + o) = make_double2(xr[2 * c], xr[2 * c + 1]);
-    *reinterpret_cast<double2*>(sI + o) = make_double2(xi[2 * c], xi[2 * c + 1]);
-  }
+// Interleaved complex layout used after P1 (double2 (re, im) per element, one 16-byte word):
+// element (l0, l1, l2) of a group buffer sits in region l2 >> 3 (the bytes of the Re / Im
+// plane's row (l0, l1)), 16-byte chunk (l2 & 7) ^ (l1 & 7) of that row.  P1 converts each row
+// in place (a thread owns both planes' 128-byte rows of its row); every later access is one
+// 16-byte word per element, conflict-free per quarter-warp (lanes = 8 consecutive l2 or l1).
+__device__ __forceinline__ int cofs(int l0, int l1, int l2) {
+  return ((l2 >> 3) << 12) | (l0 << 8) | (l1 << 4) | (((l2 & 7) ^ (l1 & 7)) << 1);
+}
+__device__ __forceinline__ double2 ldc(const double* b, int o) { return *reinterpret_cast<const double2*>(b + o); }
+__device__ __forceinline__ void stc(double* b, int o, double re, double im) {
+  *reinterpret_cast<double2*>(b + o) = make_double2(re, im);
 }
 
 // Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
@@ -72,13 +72,14 @@ struct PairGeom {
   bool has_b;
 };
 __device__ __forceinline__ PairGeom pair_geom(const Fft3dArgs& a, int64_t p) {
-  const int S = a.S;
-  const int64_t line = p / a.npr, pj = p - line * a.npr;
-  const int64_t t0 = line / a.nt1, t1 = line - t0 * a.nt1;
+  // pair / tile indices fit 32 bits (the plan's pair count is far below 2^31)
+  const int S = a.S, npr = (int)a.npr, nt1 = (int)a.nt1, pi = (int)p;
+  const int line = pi / npr, pj = pi - line * npr;
+  const int t0 = line / nt1, t1 = line - t0 * nt1;
   PairGeom g;
-  g.o0 = t0 * S + a.bd.shift;
-  g.o1 = t1 * S + a.bd.shift;
-  g.oa2 = 2 * pj * S + a.bd.shift;
+  g.o0 = (int64_t)t0 * S + a.bd.shift;
+  g.o1 = (int64_t)t1 * S + a.bd.shift;
+  g.oa2 = (int64_t)2 * pj * S + a.bd.shift;
   g.ob2 = g.oa2 + S;
   g.has_b = 2 * pj + 1 < a.nt2;
   return g;
@@ -95,9 +96,8 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
   extern __shared__ unsigned char smem_raw[];
   const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
   double* base = reinterpret_cast<double*>(smem_raw + (mis ? kAlign - mis : 0));   // stays in the shared window
-  const double* sSr = base + 4 * PLANE;
-  const double* sSi = sSr + PLANE;
-  __shared__ __align__(8) uint64_t bar[3];
+  double* sS = base + 4 * PLANE;   // S_T interleaved (re, im), natural [k0][k1][k2]
+  __shared__ __align__(8) uint64_t bar[2];
   const int grp = threadIdx.x >> 8, tid = threadIdx.x & (NT - 1);
   const int hi = tid >> 4, lo = tid & 15;
   const int S = a.S, h = a.h;
@@ -106,14 +106,9 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
   if (threadIdx.x == 0) {
     tma::mbar_init(&bar[0], 1);
     tma::mbar_init(&bar[1], 1);
-    tma::mbar_init(&bar[2], 1);
   }
+  for (int e = threadIdx.x; e < PLANE; e += 2 * NT) stc(sS, 2 * e, __ldg(a.Sre + e), __ldg(a.Sim + e));   // once per launch
   __syncthreads();
-  if (threadIdx.x == 0) {   // S_T once per launch (planes are 4096 doubles each, contiguous re | im)
-    tma::mbar_expect_tx(&bar[2], 2u * PLANE * 8u);
-    tma::load_bulk(base + 4 * PLANE, a.Sre, PLANE * 8u, &bar[2]);
-    tma::load_bulk(base + 5 * PLANE, a.Sim, PLANE * 8u, &bar[2]);
-  }
   const int64_t stride = 2 * (int64_t)gridDim.x;
   const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
   auto issue = [&](int64_t p) {
@@ -123,7 +118,6 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     if (g.has_b) tma::load_3d(sI, &tm, (int)g.ob2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
   };
   if (TMA && tid == 0 && p0 < a.win.p_end) issue(p0);
-  tma::mbar_wait(&bar[2], 0);
 
   uint32_t parity = 0;
   for (int64_t p = p0; p < a.win.p_end; p += stride) {
@@ -150,71 +144,68 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
       group_sync(grp);
     }
     double xr[16], xi[16];
-    // ---- P1: forward axis 2 (thread = row (l0, l1) = (hi, lo)) ----
+    // ---- P1: forward axis 2 (thread = row (l0, l1) = (hi, lo)); TMA planes -> interleaved ----
     load_row(sR, sI, hi, lo, xr, xi);
     radix::fft16<false>(xr, xi);
-    store_row(sR, sI, hi, lo, xr, xi);
+#pragma unroll
+    for (int l2 = 0; l2 < 16; ++l2) stc(sR, cofs(hi, lo, l2), xr[l2], xi[l2]);
     __syncwarp();
     // ---- P2: forward axis 1 (thread = (l0, l2) = (hi, lo)); same planes as the warp's P1 rows ----
-    {
-      const int b = hi << 8;
 #pragma unroll
-      for (int l1 = 0; l1 < 16; ++l1) {
-        const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
-        xr[l1] = sR[o];
-        xi[l1] = sI[o];
-      }
-      radix::fft16<false>(xr, xi);
-#pragma unroll
-      for (int l1 = 0; l1 < 16; ++l1) {
-        const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
-        sR[o] = xr[l1];
-        sI[o] = xi[l1];
-      }
+    for (int l1 = 0; l1 < 16; ++l1) {
+      const double2 v = ldc(sR, cofs(hi, l1, lo));
+      xr[l1] = v.x;
+      xi[l1] = v.y;
     }
+    radix::fft16<false>(xr, xi);
+#pragma unroll
+    for (int l1 = 0; l1 < 16; ++l1) stc(sR, cofs(hi, l1, lo), xr[l1], xi[l1]);
     group_sync(grp);
     // ---- P3: forward axis 0, * S_T, inverse axis 0 (thread = (k1, k2) = (hi, lo)) ----
     {
-      const int b = wofs(0, hi, lo);
+      const int b = cofs(0, hi, lo);
 #pragma unroll
       for (int l0 = 0; l0 < 16; ++l0) {
-        xr[l0] = sR[b + (l0 << 8)];
-        xi[l0] = sI[b + (l0 << 8)];
+        const double2 v = ldc(sR, b + (l0 << 8));
+        xr[l0] = v.x;
+        xi[l0] = v.y;
       }
       radix::fft16<false>(xr, xi);
 #pragma unroll
-      for (int k0 = 0; k0 < 16; ++k0) radix::cmul(xr[k0], xi[k0], sSr[(k0 << 8) + tid], sSi[(k0 << 8) + tid]);
+      for (int k0 = 0; k0 < 16; ++k0) {
+        const double2 sv = ldc(sS, ((k0 << 8) + tid) << 1);
+        radix::cmul(xr[k0], xi[k0], sv.x, sv.y);
+      }
       radix::fft16<true>(xr, xi);
 #pragma unroll
       for (int l0 = 0; l0 < 16; ++l0)
-        if (l0 >= h && l0 < h + S) {
-          sR[b + (l0 << 8)] = xr[l0];
-          sI[b + (l0 << 8)] = xi[l0];
-        }
+        if (l0 >= h && l0 < h + S) stc(sR, b + (l0 << 8), xr[l0], xi[l0]);
     }
     group_sync(grp);
     // ---- P4: inverse axis 1 on the S output planes (thread = (l0 - h, l2)) ----
     if (hi < S) {
-      const int b = (h + hi) << 8;
 #pragma unroll
       for (int l1 = 0; l1 < 16; ++l1) {
-        const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
-        xr[l1] = sR[o];
-        xi[l1] = sI[o];
+        const double2 v = ldc(sR, cofs(h + hi, l1, lo));
+        xr[l1] = v.x;
+        xi[l1] = v.y;
       }
       radix::fft16<true>(xr, xi);
 #pragma unroll
       for (int l1 = 0; l1 < 16; ++l1)
-        if (l1 >= h && l1 < h + S) {
-          const int o = b | (l1 << 4) | (lo ^ ((l1 & 7) << 1));
-          sR[o] = xr[l1];
-          sI[o] = xi[l1];
-        }
+        if (l1 >= h && l1 < h + S) stc(sR, cofs(h + hi, l1, lo), xr[l1], xi[l1]);
     }
     __syncwarp();
     // ---- P5: inverse axis 2 on the output rows (thread = (l0 - h, l1 - h)), same planes as P4 ----
     const bool p5 = hi < S && lo < S;
-    if (p5) load_row(sR, sI, h + hi, h + lo, xr, xi);
+    if (p5) {
+#pragma unroll
+      for (int l2 = 0; l2 < 16; ++l2) {
+        const double2 v = ldc(sR, cofs(h + hi, h + lo, l2));
+        xr[l2] = v.x;
+        xi[l2] = v.y;
+      }
+    }
     // the buffer is free: order this thread's shared accesses before the next TMA write, then
     // refill it while the last transform and the stores run
     if (TMA) tma::fence_proxy_async();
