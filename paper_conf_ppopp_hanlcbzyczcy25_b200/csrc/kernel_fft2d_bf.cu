@@ -1,38 +1,39 @@
-// Fused 2D FFT-stencil tile kernel with register-resident radix-8 FFTs on the FP64 ALU
+// Fused 2D FFT-stencil tile kernel with register-resident butterflies on the FP64 ALU
 // (sm_100a): the default 2D engine.
 //
 // Same fused pass and tile geometry as kernel_fft2d_ct.cu (Algorithm 1 L252-L258 on
 // 64 x 64 overlap-save tiles, Double-layer Filling Eq. 9, temporal fusion Eq. 10, Stitching
-// Eq. 7), with every length-64 axis DFT evaluated as the Cooley-Tukey 64 = 8 x 8 factorisation
-// (§3.2.1's reshaping, L208-L218):
-//   X[k1 + 8 k2] = sum_n2 w8^(n2 k2) w64^(n2 k1) sum_n1 w8^(n1 k1) x[8 n1 + n2]
-// where each DFT-8 is a 56-instruction butterfly (fft_radix.cuh) held by one thread ("chunk" =
-// 8 complex values), instead of 8x8 complex GEMMs on DMMA (3-6x more FP64 pipe slots on B200,
-// whose DMMA and DFMA peaks are equal and shared, profiles/r01_fp64_shared.txt).
+// Eq. 7).  Each length-64 axis DFT is the Cooley-Tukey factorisation 64 = 4 x 16 (§3.2.1's
+// reshaping, L208-L218), n = 16 n2 + m, k = k0 + 4 k':
+//   X[k0 + 4 k'] = sum_m w16^(m k') w64^(m k0) sum_n2 w4^(n2 k0) x[16 n2 + m]
+// evaluated with butterflies in registers (fft_radix.cuh) instead of DFT GEMMs on DMMA (B200's
+// DMMA and DFMA peaks are equal and shared, profiles/r01_fp64_shared.txt, Q20).
 //
-// Stages per tile pair (each a shared-memory read -> registers -> write of 512 chunks, in place):
-//   R1 rows, stage a  (chunk (r, n2), n2 pairs as 16-byte words): DFT-8 over n1, * w64^(n2 k1)
-//   R2 rows, stage b  (chunk (r, k1), 4 x 16-byte words):          DFT-8 over n2 -> X[k1 + 8 k2]
-//                                                                     at column 8 k1 + k2
-//   C1 cols, stage a  (chunk (c, n2)):                               DFT-8 over n1, * w64^(n2 k1)
-//   C2 cols, stage b, * S_T, inverse stage b (chunk (c, k1)):       DFT-8 over n2, * S, IDFT-8
-//                                                                     over k2, * conj w64^(n2 k1)
-//   C3 cols, inverse stage a (chunk (c, n2)):                        IDFT-8 over k1 -> rows
-//                                                                     8 n1 + n2, S output rows kept
-//   R3 S output rows, inverse stage b (chunk (r, k1)):               IDFT-8 over k2, * conj twiddle
-//   R4 S output rows, inverse stage a (chunk (r, n2 pair)):          IDFT-8 over k1 -> store window
-// Shared layout: four 16-column blocks, each the TMA SWIZZLE_128B image of a 64 x 16 box:
+// Five in-place shared-memory passes per tile pair; a thread owns 16 complex values per pass:
+//   P1 (thread = row class rr, column class cc; the 4 x 4 block rows 16 i + rr, columns
+//      16 j + cc): DFT-4 over i and over j, * w64^(rr k0r) w64^(cc k0c)   [both axes, stage 1]
+//   P2 (thread = row r, column block b): DFT-16 over the 16 columns 16 b + m   [axis 1, stage 2]
+//   P3 (thread = column c, row block b): DFT-16 over the rows 16 b + m, * S_T, inverse DFT-16
+//                                                                           [axis 0, stage 2]
+//   P4 (thread = row r, column block b): inverse DFT-16                      [axis 1, stage 2]
+//   P5 (as P1): * conj twiddles, inverse DFT-4 over j and i -> store the S x S window.
+// After P2/P3 position 16 k0 + k' of an axis holds frequency k0 + 4 k' (S_T is stored in that
+// position order by the plan).  Doing stage 1 of both axes in one pass (4 x 4 register blocks)
+// needs 5 passes where a thread-per-chunk radix-8 design needs 7: shared-memory traffic, which
+// binds this kernel, drops by ~25%.
+// Shared layout: four 64 x 16 column blocks, each the TMA SWIZZLE_128B image of one box:
 //   word(r, c) = 1024 (c >> 4) + 16 r + ((c & 15) ^ 2 (r & 7)).
-// Bank check (8-byte words: a half-warp per wavefront; 16-byte: a quarter-warp): column stages
-// (lanes = 16 consecutive c, rows 8 m + n2) hit banks (c & 15) ^ 2 n2 -- distinct; row stages
-// use 16-byte words at 16-byte chunk ((c & 15) >> 1) ^ (r & 7) with lanes = 8 consecutive r --
-// distinct.  Twiddle indices (n2 or k1 of a chunk) are warp-uniform, so w64^m comes from a
-// 1 KB shared table by broadcast.  S_T sits in shared memory in position order (dense [64][64],
-// position 8a + b <-> frequency a + 8b on each axis; plan.cpp).
+// Bank check (8-byte words: a half-warp per wavefront; 16-byte: a quarter-warp): P1/P5/P3 give
+// a half-warp 16 consecutive columns of one block and one row -> words (c & 15) ^ 2 (r & 7)
+// distinct; P2/P4 read a row block as 16-byte words, chunk ((c & 15) >> 1) ^ (r & 7), with 8
+// consecutive rows per quarter-warp -> distinct.  S_T (interleaved re/im, 16-byte words,
+// consecutive columns per lane) and the w64 table sit in shared memory, staged once per launch.
 //
-// TMA path: one persistent CTA (8 warps) per SM holding two pair buffers (the next pair's
-// eight 64 x 16 boxes land while the current pair is transformed) and S_T, 194 KB; the
-// cp.async path (periodic wrap-around, or a pitch TMA cannot describe) uses one buffer.
+// One CTA per SM = two independent 256-thread groups, each transforming its own sequence of
+// tile pairs in its own 64 KB buffer (named barriers); a group releases its buffer after P5's
+// reads and its next pair's eight TMA boxes (64 x 16, SWIZZLE_128B, OOB -> 0) land while it
+// finishes the inverse and the stores.  The cp.async path (periodic wrap-around, or a pitch TMA
+// cannot describe) loads the same layout synchronously.
 #include "fft_radix.cuh"
 #include "kernels.cuh"
 #include "tma.cuh"
@@ -54,47 +55,8 @@ __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool v
 }
 
 using radix::cmul;
-using radix::fft8;
-
-// Tuning switches (ablation builds via FFTSTENCIL_NVCC_DEFS): BF_TW_POW = 0 twiddles from the
-// shared table, 1 the lane-varying R1 twiddles as powers of w64^n2 in registers, 2 every twiddle
-// as powers (default: +6% on B200, fewer shared-memory wavefronts and no spills,
-// profiles/r01_s2_ab2d.txt); BF_UNROLL = chunks per thread in flight in the column/row-b stages.
-#ifndef BF_TW_POW
-#define BF_TW_POW 2
-#endif
-#ifndef BF_UNROLL
-#define BF_UNROLL 1
-#endif
-constexpr int kUnroll = BF_UNROLL;
-
-// x[j] *= w^(+-j) for j = 1..7 with w = (wr, wi) = w64^t: powers by repeated multiplication
-// (6 complex multiplies; error ~ j ulp).
-template <bool INV>
-__device__ __forceinline__ void twiddle_pow(double (&xr)[8], double (&xi)[8], double wr, double wi) {
-  if (INV) wi = -wi;
-  double pr = wr, pi = wi;
-#pragma unroll
-  for (int j = 1; j < 8; ++j) {
-    cmul(xr[j], xi[j], pr, pi);
-    if (j < 7) {
-      const double t = pr * wr - pi * wi;
-      pi = fma(pr, wi, pi * wr);
-      pr = t;
-    }
-  }
-}
-
-// twiddle x[j] *= w64^(+-t j), j = 1..7; tw[8 j + t] = w64^(j t) (shared, 1 KB): a warp-uniform
-// t is a broadcast, t = lane & 7 hits 8 distinct 16-byte chunks per quarter-warp.
-template <bool INV>
-__device__ __forceinline__ void twiddle_chunk(double (&xr)[8], double (&xi)[8], const double2* tw, int t) {
-#pragma unroll
-  for (int j = 1; j < 8; ++j) {
-    const double2 w = tw[8 * j + t];
-    cmul(xr[j], xi[j], w.x, INV ? -w.y : w.y);
-  }
-}
+using radix::dft4;
+using radix::fft16;
 
 struct Geom {
   int64_t o0, oa1, ob1;
@@ -112,13 +74,7 @@ __device__ __forceinline__ Geom geom(const Fft2dArgs& a, int64_t p) {
   return g;
 }
 
-// Row of chunk u in the row stages R1/R4 (n2 = lane & 7): bits 0-1 <- warp & 3, bit 2 <- lane
-// bit 3, bit 3 <- lane bit 4, bits 4-5 <- (warp >> 2) + 2 u.
-__device__ __forceinline__ int row_of(int warp, int lane, int u) {
-  return (warp & 3) | (((lane >> 3) & 1) << 2) | (((lane >> 4) & 1) << 3) | (((warp >> 2) + 2 * u) << 4);
-}
-
-// TMA refill of a group buffer with pair p: eight 64 x 16 boxes (OOB -> 0).
+// TMA refill of a group buffer with one pair: eight 64 x 16 boxes (OOB -> 0).
 __device__ __forceinline__ void issue_pair(const Fft2dArgs& a, const CUtensorMap* tm, const Geom& g, double* dR,
                                            uint64_t* bar) {
   const int y = (int)(g.o0 - a.win.g0);
@@ -133,206 +89,149 @@ __device__ __forceinline__ void issue_pair(const Fft2dArgs& a, const CUtensorMap
 // Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
 __device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
 
-// The seven stages over the pair in (sR, sI) by group `grp`; returns after R4's shared reads
-// (the buffer may be refilled) with the TMA refill of `next` issued, then stores the window.
+// The 4 x 4 block of P1/P5: element [i][j] at row 16 i + rr, column 16 j + cc.
+__device__ __forceinline__ void load_block(const double* sR, const double* sI, int rr, int cc, double (&xr)[4][4],
+                                           double (&xi)[4][4]) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int o = wd(16 * i + rr, 16 * j + cc);
+      xr[i][j] = sR[o];
+      xi[i][j] = sI[o];
+    }
+}
+
+// DFT-4 over i (axis 0) for every j and over j (axis 1) for every i.
+template <bool INV>
+__device__ __forceinline__ void dft4x4(double (&xr)[4][4], double (&xi)[4][4]) {
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    dft4<INV>(xr[0][j], xi[0][j], xr[1][j], xi[1][j], xr[2][j], xi[2][j], xr[3][j], xi[3][j]);
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+    dft4<INV>(xr[i][0], xi[i][0], xr[i][1], xi[i][1], xr[i][2], xi[i][2], xr[i][3], xi[i][3]);
+}
+
+// element [i][j] *= w64^(+-(rr i + cc j)) (conjugate if INV); tw = shared w64^m table.
+template <bool INV>
+__device__ __forceinline__ void twiddle4x4(double (&xr)[4][4], double (&xi)[4][4], const double2* tw, int rr,
+                                           int cc) {
+#pragma unroll
+  for (int i = 1; i < 4; ++i) {
+    const double2 w = tw[(rr * i) & 63];
+    const double wi = INV ? -w.y : w.y;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) cmul(xr[i][j], xi[i][j], w.x, wi);
+  }
+#pragma unroll
+  for (int j = 1; j < 4; ++j) {
+    const double2 w = tw[(cc * j) & 63];
+    const double wi = INV ? -w.y : w.y;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) cmul(xr[i][j], xi[i][j], w.x, wi);
+  }
+}
+
+// P2/P4: the 16 columns 16 b + m of row r as 16-byte words (chunk (m >> 1) ^ (r & 7)).
+template <bool INV>
+__device__ __forceinline__ void row_pass(double* sR, double* sI, int r, int b) {
+  const int base = (b << 10) | (r << 4), s = r & 7;
+  double xr[16], xi[16];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    const int o = base + ((c ^ s) << 1);
+    const double2 vr = *reinterpret_cast<const double2*>(sR + o);
+    const double2 vi = *reinterpret_cast<const double2*>(sI + o);
+    xr[2 * c] = vr.x; xr[2 * c + 1] = vr.y;
+    xi[2 * c] = vi.x; xi[2 * c + 1] = vi.y;
+  }
+  fft16<INV>(xr, xi);
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    const int o = base + ((c ^ s) << 1);
+    *reinterpret_cast<double2*>(sR + o) = make_double2(xr[2 * c], xr[2 * c + 1]);
+    *reinterpret_cast<double2*>(sI + o) = make_double2(xi[2 * c], xi[2 * c + 1]);
+  }
+}
+
+// The five passes over the pair in (sR, sI) by group `grp`; releases the buffer (TMA refill
+// of the group's next pair `gn`) after P5's reads, then stores the window.
 template <bool TMA>
-__device__ __forceinline__ void tile_stages(double* sR, double* sI, const double* sSr, const double* sSi,
-                                            const double2* tw, const Fft2dArgs& a, const Geom& g, int warp,
-                                            int lane, int grp, const CUtensorMap* tm, uint64_t* bar, bool has_next,
-                                            const Geom& gn) {
+__device__ __forceinline__ void tile_passes(double* sR, double* sI, const double* sS, const double2* tw,
+                                            const Fft2dArgs& a, const Geom& g, int warp, int lane, int grp,
+                                            const CUtensorMap* tm, uint64_t* bar, bool has_next, const Geom& gn) {
   const int S = a.S, h = a.h;
-  // ---- R1: rows, stage a; chunk (r, n2), n2 = lane & 7; a half-warp covers rows r0, r0 + 4
-  // (8-byte words ((8 n1 + n2) & 15) ^ 2 (r & 7): the two rows land in opposite bank halves) ----
-#pragma unroll kUnroll
-  for (int u = 0; u < 2; ++u) {
-    const int r = row_of(warp, lane, u), n2 = lane & 7;
-    double xr[8], xi[8];
+  const int rr = (warp << 1) | (lane >> 4), cc = lane & 15;     // P1/P5 block classes
+  const int rc = lane + ((warp & 1) << 5), blk = warp >> 1;      // P2/P3/P4 row or column, block
+  // ---- P1: stage 1 of both axes ----
+  {
+    double xr[4][4], xi[4][4];
+    load_block(sR, sI, rr, cc, xr, xi);
+    dft4x4<false>(xr, xi);
+    twiddle4x4<false>(xr, xi, tw, rr, cc);
 #pragma unroll
-    for (int n1 = 0; n1 < 8; ++n1) {
-      const int o = wd(r, 8 * n1 + n2);
-      xr[n1] = sR[o];
-      xi[n1] = sI[o];
-    }
-    fft8<false>(xr, xi);
-    if (BF_TW_POW >= 1) {
-      const double2 w = tw[8 + n2];   // w64^n2
-      twiddle_pow<false>(xr, xi, w.x, w.y);
-    } else {
-      twiddle_chunk<false>(xr, xi, tw, n2);
-    }
-#pragma unroll
-    for (int k1 = 0; k1 < 8; ++k1) {
-      const int o = wd(r, 8 * k1 + n2);
-      sR[o] = xr[k1];
-      sI[o] = xi[k1];
-    }
-  }
-  group_sync(grp);
-  // ---- R2: rows, stage b; chunk (r, k1): columns 8 k1 + n2 (4 x 16-byte words) ----
-#pragma unroll kUnroll
-  for (int u = 0; u < 2; ++u) {
-    const int task = warp + NW * u, r = lane + 32 * (task & 1), k1 = task >> 1;
-    double xr[8], xi[8];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int o = wd(r, 8 * k1 + 2 * j);
-      const double2 vr = *reinterpret_cast<const double2*>(sR + o);
-      const double2 vi = *reinterpret_cast<const double2*>(sI + o);
-      xr[2 * j] = vr.x; xr[2 * j + 1] = vr.y; xi[2 * j] = vi.x; xi[2 * j + 1] = vi.y;
-    }
-    fft8<false>(xr, xi);
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int o = wd(r, 8 * k1 + 2 * j);
-      *reinterpret_cast<double2*>(sR + o) = make_double2(xr[2 * j], xr[2 * j + 1]);
-      *reinterpret_cast<double2*>(sI + o) = make_double2(xi[2 * j], xi[2 * j + 1]);
-    }
-  }
-  group_sync(grp);
-  // ---- C1: columns, stage a; chunk (c, n2): rows 8 n1 + n2 ----
-#pragma unroll kUnroll
-  for (int u = 0; u < 2; ++u) {
-    const int task = warp + NW * u, c = lane + 32 * (task & 1), n2 = task >> 1;
-    double xr[8], xi[8];
-#pragma unroll
-    for (int n1 = 0; n1 < 8; ++n1) {
-      const int o = wd(8 * n1 + n2, c);
-      xr[n1] = sR[o];
-      xi[n1] = sI[o];
-    }
-    fft8<false>(xr, xi);
-    if (BF_TW_POW >= 2) {
-      const double2 w = tw[8 + n2];
-      twiddle_pow<false>(xr, xi, w.x, w.y);
-    } else {
-      twiddle_chunk<false>(xr, xi, tw, n2);
-    }
-#pragma unroll
-    for (int k1 = 0; k1 < 8; ++k1) {
-      const int o = wd(8 * k1 + n2, c);
-      sR[o] = xr[k1];
-      sI[o] = xi[k1];
-    }
-  }
-  group_sync(grp);
-  // ---- C2: columns, stage b, * S_T, inverse stage b; chunk (c, k1): rows 8 k1 + n2 ----
-#pragma unroll kUnroll
-  for (int u = 0; u < 2; ++u) {
-    const int task = warp + NW * u, c = lane + 32 * (task & 1), k1 = task >> 1;
-    double xr[8], xi[8];
-#pragma unroll
-    for (int n2 = 0; n2 < 8; ++n2) {
-      const int o = wd(8 * k1 + n2, c);
-      xr[n2] = sR[o];
-      xi[n2] = sI[o];
-    }
-    fft8<false>(xr, xi);   // slot k2: frequency k1 + 8 k2 at position 8 k1 + k2
-#pragma unroll
-    for (int k2 = 0; k2 < 8; ++k2) {
-      const int so = (8 * k1 + k2) * L + c;
-      cmul(xr[k2], xi[k2], sSr[so], sSi[so]);
-    }
-    fft8<true>(xr, xi);    // slot n2
-    if (BF_TW_POW >= 2) {
-      const double2 w = tw[8 + k1];
-      twiddle_pow<true>(xr, xi, w.x, w.y);
-    } else {
-      twiddle_chunk<true>(xr, xi, tw, k1);
-    }
-#pragma unroll
-    for (int n2 = 0; n2 < 8; ++n2) {
-      const int o = wd(8 * k1 + n2, c);
-      sR[o] = xr[n2];
-      sI[o] = xi[n2];
-    }
-  }
-  group_sync(grp);
-  // ---- C3: columns, inverse stage a; chunk (c, n2): rows 8 k1 + n2 -> rows 8 n1 + n2 (S kept) ----
-#pragma unroll kUnroll
-  for (int u = 0; u < 2; ++u) {
-    const int task = warp + NW * u, c = lane + 32 * (task & 1), n2 = task >> 1;
-    double xr[8], xi[8];
-#pragma unroll
-    for (int k1 = 0; k1 < 8; ++k1) {
-      const int o = wd(8 * k1 + n2, c);
-      xr[k1] = sR[o];
-      xi[k1] = sI[o];
-    }
-    fft8<true>(xr, xi);
-#pragma unroll
-    for (int n1 = 0; n1 < 8; ++n1) {
-      const int rr = 8 * n1 + n2;
-      if (rr >= h && rr < h + S) {
-        const int o = wd(rr, c);
-        sR[o] = xr[n1];
-        sI[o] = xi[n1];
-      }
-    }
-  }
-  group_sync(grp);
-  const int nrb = (S + 31) >> 5;   // blocks of 32 output rows
-  // ---- R3: the S output rows, inverse stage b; chunk (r, k1) ----
-  for (int task = warp; task < 8 * nrb; task += NW) {
-    const int i = 32 * (task % nrb) + lane, k1 = task / nrb;
-    if (i < S) {
-      const int r = h + i;
-      double xr[8], xi[8];
+    for (int i = 0; i < 4; ++i)
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
-        const int o = wd(r, 8 * k1 + 2 * j);
-        const double2 vr = *reinterpret_cast<const double2*>(sR + o);
-        const double2 vi = *reinterpret_cast<const double2*>(sI + o);
-        xr[2 * j] = vr.x; xr[2 * j + 1] = vr.y; xi[2 * j] = vi.x; xi[2 * j + 1] = vi.y;
+        const int o = wd(16 * i + rr, 16 * j + cc);
+        sR[o] = xr[i][j];
+        sI[o] = xi[i][j];
       }
-      fft8<true>(xr, xi);
-      if (BF_TW_POW >= 2) {
-        const double2 w = tw[8 + k1];
-        twiddle_pow<true>(xr, xi, w.x, w.y);
-      } else {
-        twiddle_chunk<true>(xr, xi, tw, k1);
-      }
+  }
+  group_sync(grp);
+  // ---- P2: axis 1, DFT-16 along row rc in column block blk ----
+  row_pass<false>(sR, sI, rc, blk);
+  group_sync(grp);
+  // ---- P3: axis 0, DFT-16 down column rc in row block blk, * S_T, inverse DFT-16 ----
+  {
+    double xr[16], xi[16];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int o = wd(r, 8 * k1 + 2 * j);
-        *reinterpret_cast<double2*>(sR + o) = make_double2(xr[2 * j], xr[2 * j + 1]);
-        *reinterpret_cast<double2*>(sI + o) = make_double2(xi[2 * j], xi[2 * j + 1]);
-      }
+    for (int m = 0; m < 16; ++m) {
+      const int o = wd(16 * blk + m, rc);
+      xr[m] = sR[o];
+      xi[m] = sI[o];
+    }
+    fft16<false>(xr, xi);   // slot k': position 16 blk + k' <-> frequency blk + 4 k'
+#pragma unroll
+    for (int k = 0; k < 16; ++k) {
+      const double2 sv = *reinterpret_cast<const double2*>(sS + ((((16 * blk + k) << 6) + rc) << 1));
+      cmul(xr[k], xi[k], sv.x, sv.y);
+    }
+    fft16<true>(xr, xi);
+#pragma unroll
+    for (int m = 0; m < 16; ++m) {
+      const int o = wd(16 * blk + m, rc);
+      sR[o] = xr[m];
+      sI[o] = xi[m];
     }
   }
   group_sync(grp);
-  // ---- R4: the S output rows, inverse stage a; chunk (h + i, n2), the R1 lane map over i ->
-  // store the window; both chunks are read before the buffer is released for the refill ----
-  double yr[2][8], yi[2][8];
-#pragma unroll
-  for (int u = 0; u < 2; ++u) {
-    const int i = row_of(warp, lane, u), n2 = lane & 7;
-    if (i < S) {
-#pragma unroll
-      for (int k1 = 0; k1 < 8; ++k1) {
-        const int o = wd(h + i, 8 * k1 + n2);
-        yr[u][k1] = sR[o];
-        yi[u][k1] = sI[o];
-      }
-    }
-  }
+  // ---- P4: axis 1 inverse DFT-16 ----
+  row_pass<true>(sR, sI, rc, blk);
+  group_sync(grp);
+  // ---- P5: conj twiddles, inverse stage 1 of both axes, store (read, release, compute) ----
+  double xr[4][4], xi[4][4];
+  load_block(sR, sI, rr, cc, xr, xi);
   if (TMA) tma::fence_proxy_async();   // the buffer is refilled by TMA after the barrier
   group_sync(grp);
   if (TMA && warp == 0 && lane == 0 && has_next) issue_pair(a, tm, gn, sR, bar);
+  twiddle4x4<true>(xr, xi, tw, rr, cc);
+  dft4x4<true>(xr, xi);
 #pragma unroll
-  for (int u = 0; u < 2; ++u) {
-    const int i = row_of(warp, lane, u), n2 = lane & 7;
-    const int64_t c0 = g.o0 + h + i;
-    if (i >= S || c0 >= a.bd.lim0 || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
-    fft8<true>(yr[u], yi[u]);
+  for (int i = 0; i < 4; ++i) {
+    const int r = 16 * i + rr;
+    const int64_t c0 = g.o0 + r;
+    if (r < h || r >= h + S || c0 >= a.bd.lim0 || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
     double* drow = a.dst + (c0 - a.win.g0) * a.n1;
 #pragma unroll
-    for (int n1 = 0; n1 < 8; ++n1) {
-      const int cc = 8 * n1 + n2;
-      if (cc >= h && cc < h + S) {
-        int64_t c1 = g.oa1 + cc;
-        if (c1 < a.bd.lim1) drow[c1] = yr[u][n1];
-        c1 = g.ob1 + cc;
-        if (g.has_b && c1 < a.bd.lim1) drow[c1] = yi[u][n1];
+    for (int j = 0; j < 4; ++j) {
+      const int c = 16 * j + cc;
+      if (c >= h && c < h + S) {
+        int64_t c1 = g.oa1 + c;
+        if (c1 < a.bd.lim1) drow[c1] = xr[i][j];
+        c1 = g.ob1 + c;
+        if (g.has_b && c1 < a.bd.lim1) drow[c1] = xi[i][j];
       }
     }
   }
@@ -343,32 +242,23 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
   extern __shared__ unsigned char smem_raw[];
   const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
   double* base = reinterpret_cast<double*>(smem_raw + (mis ? kAlign - mis : 0));   // stays in the shared window
-  const double* sSr = base + 4 * PLANE;
-  const double* sSi = sSr + PLANE;
-  double2* tw = reinterpret_cast<double2*>(base + 6 * PLANE);
-  __shared__ __align__(8) uint64_t bar[3];
+  double* sS = base + 4 * PLANE;                                  // S_T interleaved (re, im), position order
+  double2* tw = reinterpret_cast<double2*>(base + 6 * PLANE);    // w64^m
+  __shared__ __align__(8) uint64_t bar[2];
   const int grp = threadIdx.x >> 8, tid = threadIdx.x & (NT - 1), warp = tid >> 5, lane = tid & 31;
   double* sR = base + grp * 2 * PLANE;
   double* sI = sR + PLANE;
   if (threadIdx.x == 0) {
     tma::mbar_init(&bar[0], 1);
     tma::mbar_init(&bar[1], 1);
-    tma::mbar_init(&bar[2], 1);
   }
-  if (threadIdx.x < L) {   // tw[8 j + t] = w64^(j t) from the plan's w64^m table
-    const int m = ((threadIdx.x >> 3) * (threadIdx.x & 7)) & 63;
-    tw[threadIdx.x] = make_double2(a.Fre[m], a.Fim[m]);
-  }
+  if (threadIdx.x < L) tw[threadIdx.x] = make_double2(a.Fre[threadIdx.x], a.Fim[threadIdx.x]);
+  for (int e = threadIdx.x; e < PLANE; e += 2 * NT)   // once per launch
+    *reinterpret_cast<double2*>(sS + 2 * e) = make_double2(__ldg(a.Sre + e), __ldg(a.Sim + e));
   __syncthreads();
-  if (threadIdx.x == 0) {   // S_T once per launch (position order, re | im planes contiguous)
-    tma::mbar_expect_tx(&bar[2], 2u * PLANE * 8u);
-    tma::load_bulk(base + 4 * PLANE, a.Sre, PLANE * 8u, &bar[2]);
-    tma::load_bulk(base + 5 * PLANE, a.Sim, PLANE * 8u, &bar[2]);
-  }
   const int64_t stride = 2 * (int64_t)gridDim.x;
   const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
   if (TMA && tid == 0 && p0 < a.win.p_end) issue_pair(a, &tm, geom(a, p0), sR, &bar[grp]);
-  tma::mbar_wait(&bar[2], 0);
 
   uint32_t parity = 0;
   for (int64_t p = p0; p < a.win.p_end; p += stride) {
@@ -395,7 +285,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
     }
     const bool has_next = p + stride < a.win.p_end;
     const Geom gn = geom(a, has_next ? p + stride : p);
-    tile_stages<TMA>(sR, sI, sSr, sSi, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn);
+    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn);
   }
 }
 

@@ -74,14 +74,12 @@ double model_flops_2d_ct(int S, int T) {
 
 static constexpr double kEffCt = 0.70;   // assumed until measured (profiles/)
 
-// Radix-8 ALU engine (kernel_fft2d_bf.cu), per pair: DFT-8 chunks of 56 instructions/flops --
-// 512 in each of R1, R2, C1, C3, 1024 in C2, 8 S in each of R3, R4 -- twiddled chunks (R1, C1,
-// C2, R3: 7 complex multiplies by w^j plus the 6 that form the powers w^2..w^7 of w = w64^t,
-// 6 flops / 4 instructions each) and S_T (one complex multiply per element).
-static double chunks_2d_bf(int S) { return 3072.0 + 16.0 * S; }
-static double tw_chunks_2d_bf(int S) { return 1536.0 + 8.0 * S; }
-static double flops_pair_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 78.0 * tw_chunks_2d_bf(S) + 6.0 * 4096.0; }
-static double alu_ops_2d_bf(int S) { return 56.0 * chunks_2d_bf(S) + 52.0 * tw_chunks_2d_bf(S) + 4.0 * 4096.0; }
+// Butterfly ALU engine (kernel_fft2d_bf.cu, 64 = 4 x 16 per axis), per pair and per thread of
+// the 256 that transform it: P1 and P5 eight DFT-4 (128 adds) + 24 complex twiddle multiplies
+// (96 instr., 144 flops); P2 and P4 one DFT-16 (160 instr., 168 flops); P3 two DFT-16 + 16
+// spectrum multiplies (384 instr., 432 flops) -- independent of S (no crop before the stores).
+static double flops_pair_2d_bf(int) { return 256.0 * (2 * 272 + 2 * 168 + 432); }
+static double alu_ops_2d_bf(int) { return 256.0 * (2 * 224 + 2 * 160 + 384); }
 static double model_flops_2d_bf(int S, int T) { return flops_pair_2d_bf(S) / (2.0 * S * (double)S * T); }
 static constexpr double kEff2dBf = 0.35;   // flops per FP64-pipe slot-flop x pipe efficiency (assumed)
 
@@ -495,9 +493,9 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
           const int64_t L = p.L[0], k0 = i / (L * L), k12 = i % (L * L);
           dst = k12 * L + k0;
         } else if (p.algo == 1 && p.engine == 1) {
-          // radix-8 ALU engine: position order on both axes, position 8a + b <-> frequency a + 8b
+          // butterfly ALU engine: position order on both axes, position 16 a + b <-> frequency a + 4 b
           const int64_t k0 = i / 64, k1 = i % 64;
-          dst = (8 * (k0 % 8) + k0 / 8) * 64 + 8 * (k1 % 8) + k1 / 8;
+          dst = (16 * (k0 % 4) + k0 / 4) * 64 + 16 * (k1 % 4) + k1 / 4;
         } else if (p.algo == 1) {
           // factored 2D: [k1][8 g + c] holds k0 = g + 8 c (digit order of the CT output)
           const int64_t k0 = i / 64, k1 = i % 64;

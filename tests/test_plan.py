@@ -424,8 +424,8 @@ def test_alu_w64_table_vs_numpy(alu):
 
 
 def _pos(m):
-    """Position of frequency m on an axis of the radix-8 engine: p = 8 (m % 8) + m // 8."""
-    return 8 * (m % 8) + m // 8
+    """Position of frequency m = k0 + 4 k' on an axis of the 2D ALU engine: p = 16 k0 + k'."""
+    return 16 * (m % 4) + m // 4
 
 
 @pytest.mark.parametrize("shape,r,T", [("box", 1, 8), ("star", 3, 4)])
@@ -447,34 +447,31 @@ def test_alu_3d_spectrum_natural_order(alu):
     np.testing.assert_allclose(G, spectrum.powered_spectrum(w, 1, (16, 16, 16), 2), atol=1e-15)
 
 
-def _dft8(x, axis, inverse=False):
-    """DFT-8 along `axis` (numpy's definition; conj kernel unnormalised for the inverse)."""
-    return np.fft.ifft(x, axis=axis) * 8 if inverse else np.fft.fft(x, axis=axis)
+def _dft(x, axis, inverse=False):
+    """DFT along `axis` (numpy's definition; conj kernel unnormalised for the inverse)."""
+    return np.fft.ifft(x, axis=axis) * x.shape[axis] if inverse else np.fft.fft(x, axis=axis)
 
 
 def _alu_2d_tile(Z, tw, Sp, h, S):
-    """The radix-8 engine's seven stages on one complex 64 x 64 tile, index for index
-    (kernel_fft2d_bf.cu): positions 8 a + b, twiddles from the exported w64 table."""
+    """The 2D ALU engine's five passes on one complex 64 x 64 tile, index for index
+    (kernel_fft2d_bf.cu): element (16 i + rr, 16 j + cc) of the tile is X[i][rr][j][cc];
+    twiddles from the exported w64 table, S_T in its exported position order."""
     W = lambda e: tw[np.mod(e, 64)]
-    j = np.arange(8)
-    X = Z.reshape(64, 8, 8).copy()                              # [r][n1][n2]: column 8 n1 + n2
-    # R1: DFT-8 over n1, * w64^(n2 k1)                           -> [r][k1][n2]
-    X = _dft8(X, 1) * W(np.outer(j, j))[None]
-    # R2: DFT-8 over n2 -> column 8 k1 + k2 holds frequency k1 + 8 k2
-    X = _dft8(X, 2).reshape(64, 64)
-    Y = X.reshape(8, 8, 64)                                      # [n1][n2][c]: row 8 n1 + n2
-    # C1: DFT-8 over n1, * w64^(n2 k1)                           -> [k1][n2][c]
-    Y = _dft8(Y, 0) * W(np.outer(j, j))[:, :, None]
-    # C2: DFT-8 over n2 (-> k2), * S at position (8 k1 + k2, c), IDFT-8 over k2, * conj w64^(n2 k1)
-    Y = _dft8(Y, 1) * Sp.reshape(8, 8, 64)
-    Y = _dft8(Y, 1, inverse=True) * np.conj(W(np.outer(j, j)))[:, :, None]
-    # C3: IDFT-8 over k1 -> rows 8 n1 + n2
-    Y = _dft8(Y, 0, inverse=True).reshape(64, 64)[h:h + S]
-    # R3: IDFT-8 over k2 (columns 8 k1 + k2), * conj w64^(n2 k1); R4: IDFT-8 over k1
-    R = Y.reshape(S, 8, 8)                                       # [r][k1][k2]
-    R = _dft8(R, 2, inverse=True) * np.conj(W(np.outer(j, j)))[None]
-    R = _dft8(R, 1, inverse=True).reshape(S, 64)                 # column 8 n1 + n2
-    return R[:, h:h + S]
+    q = np.arange(4)[:, None, None, None], np.arange(16)[None, :, None, None]
+    qc = np.arange(4)[None, None, :, None], np.arange(16)[None, None, None, :]
+    X = Z.reshape(4, 16, 4, 16).copy()
+    # P1: DFT-4 over i and over j, * w64^(rr k0r) w64^(cc k0c)
+    X = _dft(_dft(X, 0), 2) * W(q[1] * q[0]) * W(qc[1] * qc[0])
+    # P2: DFT-16 over cc (axis 1); position 16 j + k' holds frequency j + 4 k'
+    X = _dft(X, 3)
+    # P3: DFT-16 over rr (axis 0), * S_T at the positions, inverse DFT-16
+    X = _dft(_dft(X, 1) * Sp.reshape(4, 16, 4, 16), 1, inverse=True)
+    # P4: inverse DFT-16 over cc
+    X = _dft(X, 3, inverse=True)
+    # P5: * conj twiddles, inverse DFT-4 over j and i
+    X = X * np.conj(W(q[1] * q[0]) * W(qc[1] * qc[0]))
+    X = _dft(_dft(X, 2, inverse=True), 0, inverse=True).reshape(64, 64)
+    return X[h:h + S, h:h + S]
 
 
 @pytest.mark.parametrize("shape,r,T", [("box", 1, 11), ("star", 3, 4), ("box", 2, 5)])
