@@ -116,10 +116,12 @@ def kernel_name(info) -> str:
     """The fused kernel this plan launches (csrc/kernel_*.cu)."""
     nd, algo, L = info["ndim"], info["algo"], info["tile"][0]
     if nd == 1:
+        if algo == "factored" and info.get("engine") == "alu":
+            return "fft1d_bf_kernel (4096 = 64 x 64 four-step, 64 = 4 x 16 butterflies, FP64 ALU)"
         return "fft1d_ct_kernel (4096 = 64 x 64)" if algo == "factored" else "fft1d_kernel (PFA 8 x 7)"
     if nd == 2:
         if algo == "factored" and info.get("engine") == "alu":
-            return "fft2d_bf_kernel (64 = 8 x 8 radix-8 FFT per axis, FP64 ALU)"
+            return "fft2d_bf_kernel (64 = 4 x 16 butterflies per axis, FP64 ALU)"
         return {"factored": "fft2d_ct_kernel (64 = 8 x 8 per axis)", "dense": f"fft2d_kernel<{L}>",
                 "unfused": f"fft2d_kernel<{L}> forward / spec_mul / inverse"}[algo]
     if algo == "factored":
@@ -225,11 +227,11 @@ def main():
     if world > 1:
         obj = [fs.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
-        plan = fs.Plan(gext, w, wk.radius, args.T, nranks=world, rank=rank, nccl_id=obj[0])
+        plan = fs.Plan(gext, w, wk.radius, args.T or wk.T, nranks=world, rank=rank, nccl_id=obj[0])
         # this rank's slab of a seeded synthetic global grid (generated per slab)
         u0 = wl.grid(plan.extents, wk.cfg_id * 1000 + rank)
     else:
-        plan = fs.Plan(gext, w, wk.radius, args.T)
+        plan = fs.Plan(gext, w, wk.radius, args.T or wk.T)
         u0 = wk.grid()
     info = plan.info()
     d_in = torch.from_numpy(u0).to(dev)

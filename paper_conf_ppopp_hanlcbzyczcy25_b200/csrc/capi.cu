@@ -298,7 +298,17 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Sim = Sim;
     a.crt = p->dCrt;
     a.tw = p->dF + 256;
-    if (hp.algo == 1) {
+    if (hp.algo == 1 && hp.engine == 1) {
+      // TMA staging when every tile starts on a 64-cell row of the (window) buffer
+      CUtensorMap tm;
+      const int64_t gn = hp.g1 - hp.g0;
+      const bool aligned = !hp.periodic && hp.ext[0] % 64 == 0 && hp.S[0] % 64 == 0 && hp.g0 % 64 == 0 &&
+                           gn % 64 == 0;
+      const uint64_t dims[2] = {64, (uint64_t)(gn / 64)};
+      const uint32_t box[2] = {16, 64};
+      const bool use_tma = p->use_tma && aligned && encode_tensor_map(&tm, src, 2, dims, box, true);
+      e = launch_fused1d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+    } else if (hp.algo == 1) {
       e = launch_fused1d_ct(a, (int)std::min<int64_t>(p->fused_grid, np), s);
     } else {
       const int64_t blocks = (np + kFft1dWarpsPerBlock - 1) / kFft1dWarpsPerBlock;
@@ -630,6 +640,10 @@ int setup_device(fftstencil_plan* p) {
   } else if (hp.ndim == 3) {
     e = fused3d_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "fused 3D kernel configuration");
+  } else if (hp.algo == 1 && hp.engine == 1) {
+    if (const char* v = std::getenv("FFTSTENCIL_TMA")) p->use_tma = std::atoi(v) != 0;
+    e = fused1d_bf_configure(&occ);
+    if (e != cudaSuccess) return cuda_fail(e, "factored 1D kernel configuration");
   } else if (hp.algo == 1) {
     e = fused1d_ct_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "factored 1D kernel configuration");
@@ -642,6 +656,10 @@ int setup_device(fftstencil_plan* p) {
     return FFTSTENCIL_EUNSUPPORTED;
   }
   p->fused_grid = (int)std::max<int64_t>(1, (int64_t)p->sm_count * occ);
+  // 1D: the band is two blocks of t (~1000) sequential direct steps, as long as the fused pass;
+  // the register-full ALU kernel (one CTA per SM) would serialise it, so leave it its SMs
+  if (hp.ndim == 1 && hp.algo == 1 && hp.engine == 1 && !hp.band_blocks.empty())
+    p->fused_grid = (int)std::max<int64_t>(1, p->fused_grid - (int64_t)(hp.band_blocks.size() / 8));
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
   if (const char* v = std::getenv("FFTSTENCIL_BAND_STREAM")) p->band_concurrent = std::atoi(v) != 0;
   if (hp.band_blocks.empty()) p->band_concurrent = false;
@@ -729,7 +747,15 @@ int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* we
   std::vector<double> v;
   if (which == 0) {
     int L, row0 = 0, ld;
-    if (hp.ndim == 1 && hp.algo == 1) {
+    if (hp.ndim == 1 && hp.algo == 1 && hp.engine == 1) {
+      // ALU engine: axis 0 = w64^m (m < 64), axis 2 = w4096^m (m < 256)
+      if (axis != 0 && axis != 2) { set_error("axis must be 0 (w64^m) or 2 (w4096^m) for the ALU engine"); return FFTSTENCIL_EINVAL; }
+      if (axis == 0)
+        for (int m = 0; m < 64; ++m) { v.push_back(hp.Fre[m]); v.push_back(hp.Fim[m]); }
+      else
+        v.assign(hp.tw.begin(), hp.tw.end());
+      L = 0;
+    } else if (hp.ndim == 1 && hp.algo == 1) {
       // factored 1D: axis 0 = F_8, 1 = twiddles w64^(ka lb) (8 x 8), 2 = w4096^(a c) (64 x 64)
       if (axis < 0 || axis > 2) { set_error("axis must be 0 (F_8), 1 (w64) or 2 (w4096)"); return FFTSTENCIL_EINVAL; }
       if (axis == 2) {

@@ -89,8 +89,11 @@ __global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
 // without per-cell divisions.  Same definition and result as band_kernel.
 constexpr int kMaxTaps = 512;
 
-// (256, 6): at most 40 registers, so one band CTA fits beside three fused CTAs on an SM
-__global__ void __launch_bounds__(kBandThreads, 6) band_cone_kernel(const BandArgs a) {
+// NTH = 256, (256, 6): at most 40 registers (one band CTA fits beside the DMMA engines' fused
+// CTAs); NTH = 1024 for the 1D band, whose two blocks run t (~1000) sequential steps on SMs
+// the fused kernel leaves free (capi.cu), so per-step latency is what counts.
+template <int NTH>
+__global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(const BandArgs a) {
   extern __shared__ double sb[];
   __shared__ int s_off[kMaxTaps];
   __shared__ double s_w[kMaxTaps];
@@ -134,7 +137,7 @@ __global__ void __launch_bounds__(kBandThreads, 6) band_cone_kernel(const BandAr
   double* b0 = sb;
   double* b1 = sb + vol;
   const int rows = D[0] * D[1];
-  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5, ny = kBandThreads / 32;
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5, ny = NTH / 32;
   for (int row = ty; row < rows; row += ny) {
     const int i0 = row / D[1], i1 = row - i0 * D[1];
     const double* src = a.src + ((rl[0] + i0 - off[0]) * a.n[1] + (rl[1] + i1 - off[1])) * a.n[2] + (rl[2] - off[2]);
@@ -161,9 +164,9 @@ __global__ void __launch_bounds__(kBandThreads, 6) band_cone_kernel(const BandAr
     const int W12 = W1 * W2, ncone = W0 * W12;
     int k0 = threadIdx.x / W12, k1 = (threadIdx.x - k0 * W12) / W2;
     int k2 = threadIdx.x - k0 * W12 - k1 * W2;
-    const int d0 = kBandThreads / W12, d1 = (kBandThreads - d0 * W12) / W2;
-    const int d2 = kBandThreads - d0 * W12 - d1 * W2;
-    for (int f = threadIdx.x; f < ncone; f += kBandThreads) {
+    const int d0 = NTH / W12, d1 = (NTH - d0 * W12) / W2;
+    const int d2 = NTH - d0 * W12 - d1 * W2;
+    for (int f = threadIdx.x; f < ncone; f += NTH) {
       const int i0 = clo[0] + k0, i1 = clo[1] + k1, i2 = clo[2] + k2;
       const int e = (i0 * D[1] + i1) * D[2] + i2;
       double v;
@@ -225,9 +228,12 @@ cudaError_t band_configure(size_t smem) {
   const size_t lim0 = (size_t)optin - fa.sharedSizeBytes;
   if ((e = cudaFuncSetAttribute(band_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim0)) != cudaSuccess)
     return e;
-  if ((e = cudaFuncGetAttributes(&fa, band_cone_kernel)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&fa, band_cone_kernel<256>)) != cudaSuccess) return e;
   const size_t lim1 = (size_t)optin - fa.sharedSizeBytes;
-  if ((e = cudaFuncSetAttribute(band_cone_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
+  if ((e = cudaFuncSetAttribute(band_cone_kernel<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
+      cudaSuccess)
+    return e;
+  if ((e = cudaFuncSetAttribute(band_cone_kernel<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
       cudaSuccess)
     return e;
   return smem <= lim0 && smem <= lim1 ? cudaSuccess : cudaErrorInvalidValue;
@@ -237,8 +243,11 @@ cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s) {
   if (a.nblocks <= 0) return cudaSuccess;
   int taps = 1;
   for (int q = 0; q < 3; ++q) taps *= a.active[q] ? 2 * a.r + 1 : 1;
-  if (taps <= kMaxTaps && !a.reference)
-    band_cone_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
+  const bool one_d = a.active[0] + a.active[1] + a.active[2] == 1;
+  if (taps <= kMaxTaps && !a.reference && one_d)
+    band_cone_kernel<1024><<<a.nblocks, 1024, smem, s>>>(a);
+  else if (taps <= kMaxTaps && !a.reference)
+    band_cone_kernel<256><<<a.nblocks, kBandThreads, smem, s>>>(a);
   else
     band_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
   return cudaGetLastError();

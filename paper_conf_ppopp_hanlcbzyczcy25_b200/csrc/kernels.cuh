@@ -139,6 +139,12 @@ constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused1d(const Fft1dArgs& a, int grid, cudaStream_t s);
 size_t fused1d_ct_smem();
+// Butterfly ALU engine of the factored 1D tile (kernel_fft1d_bf.cu): Fre/Fim[0..63] = w64^m,
+// tw = w4096^m (m < 256, interleaved); Sre/Sim = S_T at [column position][row position].
+// tm: the buffer as rows of 64 cells (dims {64, gn / 64}, box {16, 64}, SWIZZLE_128B) or null.
+size_t fused1d_bf_smem();
+cudaError_t fused1d_bf_configure(int* max_blocks_per_sm);
+cudaError_t launch_fused1d_bf(const Fft1dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
 cudaError_t fused1d_ct_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused1d_ct(const Fft1dArgs& a, int grid, cudaStream_t s);
 

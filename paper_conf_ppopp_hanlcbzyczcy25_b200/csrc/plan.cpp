@@ -145,6 +145,13 @@ static constexpr double kEff1d = 0.73;     // PFA 8x7: executed DMMA efficiency 
 static double flops_pair_1d_ct() { return kProdFlops * 512.0 + 6.0 * 7.0 * 4096.0; }
 static double model_flops_1d_ct(int S, int T) { return flops_pair_1d_ct() / (2.0 * S * (double)T); }
 static constexpr double kEff1dCt = 0.70;   // assumed until measured
+// Butterfly ALU engine (kernel_fft1d_bf.cu), per pair and per thread of 256: P1/P3/P5/P7 four
+// DFT-4 + 12 twiddle multiplies (112 instr., 136 flops), P2/P6 a DFT-16 + 31 complex multiplies
+// (w4096 powers: 284 instr., 354 flops), P4 two DFT-16 + 16 spectrum multiplies (384, 432).
+static double flops_pair_1d_bf() { return 256.0 * (4 * 136 + 2 * 354 + 432); }
+static double alu_ops_1d_bf() { return 256.0 * (4 * 112 + 2 * 284 + 384); }
+static double model_flops_1d_bf(int S, int T) { return flops_pair_1d_bf() / (2.0 * S * (double)T); }
+static constexpr double kEff1dBf = 0.35;
 
 static int env_engine();
 
@@ -180,11 +187,16 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   if (ndim == 1) {
     // candidates: the prime-factor 8 x 7 tile (the paper's, §3.2.1) and the factored
     // 4096 = 64 x 64 tile (long tiles for deep temporal fusion, kernel_fft1d_ct.cu)
+    const int engine1d = env_engine();
     double best = 1e300;
     int bT = 0, bA = 0;
     for (int al = 0; al < 2; ++al) {
       if (algo >= 0 && al != algo) continue;
       const int L = al ? kCt1dL : kPfaN1 * kPfaN2;
+      // the cost model is per cell-step; it ignores parallelism, so the long tile is chosen
+      // automatically only when it still yields >= 64 tiles (short grids such as BASELINE
+      // configs[0], 4096 cells, keep the paper's 8 x 7 prime-factor tile)
+      if (al && algo < 0 && extents[0] < 64 * (int64_t)(kCt1dL / 2)) continue;
       const int smin = al ? 64 : 8;
       const int hmax = std::min(hmax_grid, (L - smin) / 2);
       if (hmax < radius) continue;
@@ -192,7 +204,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       const int tlo = T == 0 ? 1 : std::min(T, tmax), thi = T == 0 ? (al ? tmax : std::min(tmax, 64)) : tlo;
       for (int t = tlo; t <= thi; ++t) {
         const int S = L - 2 * radius * t;
-        const double f = al ? model_flops_1d_ct(S, t) / kEff1dCt : model_flops_1d(S, t) / kEff1d;
+        // ALU engine: 64-aligned valid lengths keep the tile origins on 64-cell rows (TMA staging)
+        const double f = !al ? model_flops_1d(S, t) / kEff1d
+                         : engine1d ? model_flops_1d_bf(S, t) / kEff1dBf * (S % 64 ? 1.05 : 1.0)
+                                    : model_flops_1d_ct(S, t) / kEff1dCt;
         if (f < best * (1 - 1e-12)) { best = f; bT = t; bA = al; }
       }
     }
@@ -205,7 +220,13 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
     p.h = radius * p.T;
     p.L[0] = L;
     p.S[0] = L - 2 * p.h;
-    if (bA) {
+    if (bA && engine1d) {
+      p.engine = 1;
+      p.flops_per_cell_step = model_flops_1d_bf(p.S[0], p.T);
+      p.mma_flops_per_pair = 0;
+      p.alu_ops_per_pair = alu_ops_1d_bf();
+      p.fused_smem = (size_t)6 * kCt1dL * sizeof(double) + (64 + 256) * 16 + 1024;
+    } else if (bA) {
       p.flops_per_cell_step = model_flops_1d_ct(p.S[0], p.T);
       p.mma_flops_per_pair = kProdDmmaFlops * 512.0;
       p.fused_smem = (size_t)2 * kCt1dL * sizeof(double);
@@ -373,7 +394,22 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   }
 
   // ---- DFT matrices (forward; the kernel conjugates for the inverse, L258/L278) ----
-  if (ndim == 1 && p.algo == 1) {
+  if (ndim == 1 && p.algo == 1 && p.engine == 1) {
+    // butterfly ALU engine: w64^m (m < 64) and w4096^m (m < 256, interleaved re, im)
+    p.Fre.assign(128, 0.0);
+    p.Fim.assign(128, 0.0);
+    for (int m = 0; m < 64; ++m) {
+      const cplx v = root(m, 64);
+      p.Fre[m] = v.real();
+      p.Fim[m] = v.imag();
+    }
+    p.tw.assign(2 * 256, 0.0);
+    for (int m = 0; m < 256; ++m) {
+      const cplx v = root(m, kCt1dL);
+      p.tw[2 * m] = v.real();
+      p.tw[2 * m + 1] = v.imag();
+    }
+  } else if (ndim == 1 && p.algo == 1) {
     // [F8 | twiddles w64^(ka lb)] as in 2D, and the four-step twiddles w4096^(a c)
     p.Fre.assign(128, 0.0);
     p.Fim.assign(128, 0.0);
@@ -479,7 +515,12 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
         // 2D: natural [k0][k1].  3D: [k1][k2][k0] -- the 3D kernel multiplies in C fragments
         // whose two adjacent columns are consecutive k0 (kernel_fft3d.cu phase 2).
         int64_t dst = i;
-        if (ndim == 1) {
+        if (ndim == 1 && p.engine == 1) {
+          // ALU engine: k = c + 64 d at [column position q(d)][row position p(c)], position
+          // 16 a + b <-> frequency a + 4 b (kernel_fft1d_bf.cu)
+          const int64_t c = i % 64, d = i / 64;
+          dst = (16 * (d % 4) + d / 4) * 64 + 16 * (c % 4) + c / 4;
+        } else if (ndim == 1) {
           // factored 1D: k = c + 64 d at [c][8 (d % 8) + d / 8] (row c, CT digit order of d)
           const int64_t c = i % 64, d = i / 64;
           dst = c * 64 + 8 * (d % 8) + d / 8;

@@ -479,3 +479,23 @@ def test_parity_2d_engines(fs, monkeypatch, engine, tma, ext, shape, r, T, steps
     assert p.info()["engine"] == engine
     ref = oracle.stencil_run(u0, w, r, steps)
     assert rel_err(got, ref) <= TOL, (rel_err(got, ref), p.info())
+
+
+CASES_1D_LONG = [((20000,), 1, 1024, 2100), ((9000,), 3, 352, 800), ((70000,), 2, 512, 1100), ((12345,), 1, 300, 700),
+                 ((131072,), 1, 1024, 2100), ((40960,), 3, 352, 1000), ((65536,), 2, 512, 1200)]
+
+
+@pytest.mark.parametrize("engine,tma", [("dmma", "1"), ("alu", "1"), ("alu", "0")])
+@pytest.mark.parametrize("ext,r,T,steps", CASES_1D_LONG)
+def test_parity_1d_engines(fs, monkeypatch, engine, tma, ext, r, T, steps):
+    """Both line engines of the factored 1D tile (4096 = 64 x 64 four-step) against the oracle;
+    64-aligned grids with 64-aligned valid lengths take the TMA staging path."""
+    monkeypatch.setenv("FFTSTENCIL_ALGO", "factored")
+    monkeypatch.setenv("FFTSTENCIL_ENGINE", engine)
+    monkeypatch.setenv("FFTSTENCIL_TMA", tma)
+    w = wl.seeded_weights("star", 1, r)
+    u0 = wl.grid(ext, 14)
+    got, p = run_gpu(fs, u0, w, r, T, steps)
+    assert p.info()["engine"] == engine and p.info()["T"] == T
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(got, ref) <= TOL, (rel_err(got, ref), p.info())

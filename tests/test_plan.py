@@ -337,8 +337,10 @@ def test_periodic_tiles_cover_grid_exactly_once(ext, shape, r, T):
 
 
 # ---------------------------------------------------------------- factored 1D (4096 = 64 x 64)
-def test_factored_1d_is_default_for_long_grids():
-    """The cost model takes the long tile for deep fusion: T = L / (4r) maximises S T."""
+def test_factored_1d_is_default_for_long_grids(monkeypatch):
+    """The cost model takes the long tile for deep fusion: T = L / (4r) maximises S T
+    (DMMA line engine; the ALU engine's choice is pinned by test_alu_1d_default_...)."""
+    monkeypatch.setenv("FFTSTENCIL_ENGINE", "dmma")
     for r in (1, 2, 3):
         info = fs.describe((1 << 24,), wl.seeded_weights("star", 1, r), r, 0)
         assert info["algo"] == "factored" and info["tile"] == [4096] and info["pfa"] == [64, 64]
@@ -496,3 +498,75 @@ def test_alu_2d_stage_model_vs_overlap_save(alu, shape, r, T):
         # and the direct-stencil oracle on the tile (valid window = exact T-step result)
         direct = oracle.stencil_run(np.pad(x, 0), w, r, T, periodic=True)[h:h + S, h:h + S]
         np.testing.assert_allclose(part, direct, atol=1e-11)
+
+
+# ---------------------------------------------------------------- ALU engine, 1D (4096 = 64 x 64)
+def test_alu_1d_default_and_aligned_valid_length():
+    """The ALU engine is the 1D default for long grids; its cost model prefers T with S a
+    multiple of 64 (tile origins on 64-cell rows: TMA staging) at < 1% loss of S T."""
+    for r in (1, 2, 3):
+        info = fs.describe((1 << 24,), wl.seeded_weights("star", 1, r), r, 0)
+        assert info["algo"] == "factored" and info["engine"] == "alu" and info["tile"] == [4096]
+        S, T = info["valid"][0], info["T"]
+        assert S % 64 == 0 and S * T >= 0.99 * max((4096 - 2 * r * t) * t for t in range(1, 2048 // r))
+
+
+def _alu_1d_tables(n, w, r, T):
+    c = lambda v: v[0::2] + 1j * v[1::2]   # noqa: E731
+    return c(fs.export_aux((n,), w, r, T, which=0, axis=0)), c(fs.export_aux((n,), w, r, T, which=0, axis=2))
+
+
+def test_alu_1d_tables_vs_numpy(alu):
+    w64, w4k = _alu_1d_tables(20000, wl.seeded_weights("star", 1, 1), 1, 100)
+    np.testing.assert_allclose(w64, np.exp(-2j * np.pi * np.arange(64) / 64), atol=1e-15)
+    np.testing.assert_allclose(w4k, np.exp(-2j * np.pi * np.arange(256) / 4096), atol=1e-15)
+
+
+def _alu_1d_tile(x, w64, w4k, Sq):
+    """The 1D ALU engine's seven passes on one complex 4096-cell tile (kernel_fft1d_bf.cu):
+    plane[b][a] = x[a + 64 b] viewed as [i][rr][j][cc] with b = 16 i + rr, a = 16 j + cc;
+    S_T in its exported [column position][row position] order."""
+    W = lambda e: w64[np.mod(e, 64)]                                     # noqa: E731
+    i4, r16 = np.arange(4)[:, None, None, None], np.arange(16)[None, :, None, None]
+    j4, c16 = np.arange(4)[None, None, :, None], np.arange(16)[None, None, None, :]
+    a = 16 * j4 + c16                                                    # column (cell digit a)
+    X = x.reshape(4, 16, 4, 16).copy()
+    X = _dft(X, 0) * W(r16 * i4)                                         # P1: column stage 1
+    X = _dft(X, 1)                                                       # P2: column stage 2 -> c
+    c = i4 + 4 * r16                                                     # row position 16 i + rr <-> c
+    tw4096 = w4k[np.mod(a * i4, 4096)] * w4k[np.mod(4 * a, 4096)] ** r16   # base * step^c'
+    X = X * tw4096
+    X = _dft(X, 2) * W(c16 * j4)                                         # P3: row stage 1
+    F = _dft(X, 3)                                                       # P4: row stage 2 -> d
+    Sp = Sq.T.reshape(4, 16, 4, 16)                                      # [row pos][column pos]
+    X = _dft(F * Sp, 3, inverse=True)
+    X = _dft(X * np.conj(W(c16 * j4)), 2, inverse=True)                  # P5
+    X = _dft(X * np.conj(tw4096), 1, inverse=True)                       # P6
+    X = _dft(X * np.conj(W(r16 * i4)), 0, inverse=True)                  # P7
+    return F, X.reshape(-1)
+
+
+@pytest.mark.parametrize("r,T", [(1, 1024), (2, 512), (3, 352), (3, 17)])
+def test_alu_1d_pass_model_matches_fft_and_oracle(alu, r, T):
+    """Run through the seven passes, the exported tables give fft(x) at the frequency
+    positions (row 16 c0 + c' <-> c = c0 + 4 c', column 16 d0 + d' <-> d = d0 + 4 d',
+    k = c + 64 d), and one fused pass equals T direct steps (the oracle) on [h, 4096 - h)."""
+    n = 4096
+    w = wl.seeded_weights("star", 1, r)
+    info = fs.describe((n,), w, r, T)
+    assert info["engine"] == "alu" and info["T"] == T
+    h = info["halo"]
+    w64, w4k = _alu_1d_tables(n, w, r, T)
+    v = fs.export_aux((n,), w, r, T, which=1, t=T)
+    Sq = (v[0::2] + 1j * v[1::2]).reshape(64, 64)
+    u, u2 = wl.grid((n,), 7), wl.grid((n,), 8)
+    F, y = _alu_1d_tile(u + 1j * u2, w64, w4k, Sq)
+    ref = np.fft.fft(u + 1j * u2)
+    pos = lambda f: 16 * (f % 4) + f // 4                                 # noqa: E731
+    k = np.arange(n)
+    got = F.reshape(64, 64)[pos(k % 64), pos(k // 64)]
+    np.testing.assert_allclose(got, ref, atol=1e-10)
+    for part, src in ((y.real, u), (y.imag, u2)):
+        want = oracle.stencil_run(src, w, r, T)
+        err = np.abs(part[h:n - h] - want[h:n - h]).max()
+        assert err <= 1e-11 * np.abs(want).max(), err

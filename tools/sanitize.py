@@ -10,10 +10,16 @@ import paper_conf_ppopp_hanlcbzyczcy25_b200 as fs  # noqa: E402
 from synth import workloads as wl  # noqa: E402
 
 torch.cuda.set_device(0)
-cases = [((150, 140), "box", 1, 4, 9, {}), ((150, 140), "box", 1, 4, 9, {"FFTSTENCIL_ALGO": "dense"}),
+F, D = "FFTSTENCIL_ALGO", "FFTSTENCIL_ENGINE"
+cases = [((150, 140), "box", 1, 4, 9, {}), ((150, 140), "box", 1, 4, 9, {F: "dense"}),
+         ((150, 140), "box", 1, 4, 9, {F: "factored", D: "dmma"}),
          ((130, 98), "star", 2, 3, 7, {"FFTSTENCIL_TMA": "0"}),
-         ((40, 36, 34), "box", 1, 2, 5, {}), ((40, 36, 34), "box", 1, 2, 5, {"FFTSTENCIL_ALGO": "dense"}),
-         ((33, 35, 37), "star", 1, 2, 3, {}), ((900,), "star", 1, 8, 19, {})]
+         ((40, 36, 34), "box", 1, 2, 5, {}), ((40, 36, 34), "box", 1, 2, 5, {F: "dense"}),
+         ((40, 36, 34), "box", 1, 2, 5, {F: "factored", D: "dmma"}),
+         ((33, 35, 37), "star", 1, 2, 3, {"FFTSTENCIL_TMA": "0"}), ((900,), "star", 1, 8, 19, {}),
+         ((16384,), "star", 1, 1024, 1030, {F: "factored"}),                      # 1D ALU, TMA rows
+         ((9000,), "star", 3, 352, 400, {F: "factored"}),                         # 1D ALU, cp.async
+         ((9000,), "star", 3, 352, 400, {F: "factored", D: "dmma"})]
 for ext, shape, r, T, steps, env in cases:
     for k, v in env.items():
         os.environ[k] = v
@@ -24,7 +30,7 @@ for ext, shape, r, T, steps, env in cases:
     p.run(u, o, steps)
     torch.cuda.synchronize()
     assert np.isfinite(o.cpu().numpy()).all()
-    print("ok", ext, env, p.info()["algo"])
+    print("ok", ext, env, p.info()["algo"], p.info()["engine"])
     for k in env:
         del os.environ[k]
 # loopback decomposition
