@@ -7,9 +7,12 @@
  *   - the grid is split into overlap-save tiles, halo h = radius*T  (§3.1 Splitting,
  *     Eq. 3, Eq. 4; Stitching Eq. 7);
  *   - each pair of real tiles is packed as one complex tile (Double-layer Filling,
- *     §3.2.3 Eq. 9), transformed by dense DFT-matrix GEMMs on the FP64
- *     tensor cores (Algorithm 1; 1D via the prime-factor map §3.2.1
- *     Eq. 8), multiplied by the stencil spectrum raised to the power T
+ *     §3.2.3 Eq. 9), transformed axis by axis (Algorithm 1) with
+ *     each length-L DFT reshaped into small DFTs (§3.2.1: Cooley-Tukey per
+ *     axis; 1D prime-factor map Eq. 8 L214-L218 for short grids) that run either as
+ *     butterflies on the FP64 ALU (default: on B200 the FP64 tensor path equals and
+ *     shares the DFMA budget, reading Q20) or as DFT GEMMs on the FP64
+ *     tensor cores (DMMA; FFTSTENCIL_ENGINE=dmma), multiplied by the stencil spectrum raised to the power T
  *     (temporal fusion §4 Eq. 10), inverse-transformed, cropped and stored,
  *     all inside one fused kernel (Kernel Tailoring, §3.1 Fusing L190-L198);
  *   - cells within h of the fixed ring are recomputed by T direct steps (the paper is
@@ -90,9 +93,9 @@ typedef struct {
                                    (FFTSTENCIL_ALGO=unfused: forward / multiply / inverse as
                                    three kernels with the spectrum in HBM)                  */
   int periodic;                 /* 1 for a FFTSTENCIL_PERIODIC plan                      */
-  int engine;                   /* line-DFT engine of the factored 3D tile: 0 DFT-8 GEMMs on
-                                   the FP64 tensor pipe (DMMA), 1 radix-4 FFTs in registers on
-                                   the FP64 ALU (default; FFTSTENCIL_ENGINE=dmma|alu)         */
+  int engine;                   /* line-DFT engine of the factored tile (algo 1): 0 DFT GEMMs
+                                   on the FP64 tensor pipe (DMMA), 1 butterflies in registers
+                                   on the FP64 ALU (default; FFTSTENCIL_ENGINE=dmma|alu)      */
   double alu_ops_per_pass;      /* engine 1: FP64 ALU instructions one fused launch executes
                                    (adds, multiplies and FMAs, each one)                    */
 } fftstencil_info;

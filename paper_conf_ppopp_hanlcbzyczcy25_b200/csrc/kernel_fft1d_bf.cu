@@ -250,16 +250,20 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
   group_sync(grp);
   if (TMA && warp == 0 && lane == 0 && has_next) issue_pair(a, tm, gn, sR, bar);
   col_stage1<true>(br, bi, tw64, rr);
+  // tile offsets l = a + 64 b stored: [h, h + S) within the grid limit and the rank's window
+  const int64_t hi_c = min(a.bd.lim0, a.win.w_hi);
+  const int la0 = (int)max((int64_t)h, a.win.w_lo - g.oa), la1 = (int)min((int64_t)(h + S), hi_c - g.oa);
+  const int lb0 = (int)max((int64_t)h, a.win.w_lo - g.ob);
+  const int lb1 = g.has_b ? (int)min((int64_t)(h + S), hi_c - g.ob) : 0;
+  double* da = a.dst + (g.oa - a.win.g0);
+  double* db = a.dst + (g.ob - a.win.g0);
 #pragma unroll
   for (int i = 0; i < 4; ++i)
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       const int l = 16 * j + cc + 64 * (16 * i + rr);   // cell offset a + 64 b within the tile
-      if (l < h || l >= h + S) continue;
-      int64_t c = g.oa + l;
-      if (c < a.bd.lim0 && c >= a.win.w_lo && c < a.win.w_hi) a.dst[c - a.win.g0] = br[i][j];
-      c = g.ob + l;
-      if (g.has_b && c < a.bd.lim0 && c >= a.win.w_lo && c < a.win.w_hi) a.dst[c - a.win.g0] = bi[i][j];
+      if (l >= la0 && l < la1) da[l] = br[i][j];
+      if (l >= lb0 && l < lb1) db[l] = bi[i][j];
     }
 }
 

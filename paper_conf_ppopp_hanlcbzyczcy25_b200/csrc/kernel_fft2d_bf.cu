@@ -218,21 +218,28 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
   if (TMA && warp == 0 && lane == 0 && has_next) issue_pair(a, tm, gn, sR, bar);
   twiddle4x4<true>(xr, xi, tw, rr, cc);
   dft4x4<true>(xr, xi);
+  // column predicates once per pass (valid window [h, h + S), grid limit, tile b present)
+  const int64_t ca = g.oa1 + cc, cb = g.ob1 + cc;
+  bool va[4], vb[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int c = 16 * j + cc;
+    const bool in = c >= h && c < h + S;
+    va[j] = in && ca + 16 * j < a.bd.lim1;
+    vb[j] = in && g.has_b && cb + 16 * j < a.bd.lim1;
+  }
+  const int64_t r_lo = max((int64_t)h, max(a.win.w_lo, (int64_t)0) - g.o0);    // rows [r_lo, r_hi) of the tile
+  const int64_t r_hi = min((int64_t)(h + S), min(a.bd.lim0, a.win.w_hi) - g.o0);
+  double* dbase = a.dst + (g.o0 - a.win.g0) * a.n1;
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     const int r = 16 * i + rr;
-    const int64_t c0 = g.o0 + r;
-    if (r < h || r >= h + S || c0 >= a.bd.lim0 || c0 < a.win.w_lo || c0 >= a.win.w_hi) continue;
-    double* drow = a.dst + (c0 - a.win.g0) * a.n1;
+    if (r < r_lo || r >= r_hi) continue;
+    double* drow = dbase + (int64_t)r * a.n1;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      const int c = 16 * j + cc;
-      if (c >= h && c < h + S) {
-        int64_t c1 = g.oa1 + c;
-        if (c1 < a.bd.lim1) drow[c1] = xr[i][j];
-        c1 = g.ob1 + c;
-        if (g.has_b && c1 < a.bd.lim1) drow[c1] = xi[i][j];
-      }
+      if (va[j]) drow[ca + 16 * j] = xr[i][j];
+      if (vb[j]) drow[cb + 16 * j] = xi[i][j];
     }
   }
 }
