@@ -58,6 +58,33 @@ using radix::cmul;
 using radix::dft4;
 using radix::fft16;
 
+// BF_TMEM_S = 1: S_T lives in tensor memory instead of shared memory (P3 reads it with
+// tcgen05.ld, a data path of its own, taking 512 wavefronts per pair off shared memory).
+// Per TMEM lane 32 (w & 3) + lane of a group-local warp w: the S values of P3 column
+// rc = lane + 32 (w & 1), row block (w >> 1), set s = w >> 2 -> columns 64 s + 4 k + {re lo,
+// re hi, im lo, im hi}, k = 0..15; both groups share them (128 columns).
+#ifndef BF_TMEM_S
+#define BF_TMEM_S 0
+#endif
+
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8]) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+               : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+}
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
+          taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
+}
+__device__ __forceinline__ double u2d(uint32_t lo, uint32_t hi) {
+  return __hiloint2double((int)hi, (int)lo);
+}
+
 struct Geom {
   int64_t o0, oa1, ob1;
   bool has_b;
@@ -160,7 +187,8 @@ __device__ __forceinline__ void row_pass(double* sR, double* sI, int r, int b) {
 template <bool TMA>
 __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double* sS, const double2* tw,
                                             const Fft2dArgs& a, const Geom& g, int warp, int lane, int grp,
-                                            const CUtensorMap* tm, uint64_t* bar, bool has_next, const Geom& gn) {
+                                            const CUtensorMap* tm, uint64_t* bar, bool has_next, const Geom& gn,
+                                            uint32_t tmem_s) {
   const int S = a.S, h = a.h;
   const int rr = (warp << 1) | (lane >> 4), cc = lane & 15;     // P1/P5 block classes
   const int rc = lane + ((warp & 1) << 5), blk = warp >> 1;      // P2/P3/P4 row or column, block
@@ -193,10 +221,21 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
       xi[m] = sI[o];
     }
     fft16<false>(xr, xi);   // slot k': position 16 blk + k' <-> frequency blk + 4 k'
+    if (BF_TMEM_S) {
 #pragma unroll
-    for (int k = 0; k < 16; ++k) {
-      const double2 sv = *reinterpret_cast<const double2*>(sS + ((((16 * blk + k) << 6) + rc) << 1));
-      cmul(xr[k], xi[k], sv.x, sv.y);
+      for (int q = 0; q < 8; ++q) {   // 2 complex values per 8-column load
+        uint32_t v[8];
+        tmem_ld8(tmem_s + 8 * q, v);
+#pragma unroll
+        for (int e = 0; e < 2; ++e)
+          cmul(xr[2 * q + e], xi[2 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < 16; ++k) {
+        const double2 sv = *reinterpret_cast<const double2*>(sS + ((((16 * blk + k) << 6) + rc) << 1));
+        cmul(xr[k], xi[k], sv.x, sv.y);
+      }
     }
     fft16<true>(xr, xi);
 #pragma unroll
@@ -260,9 +299,43 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
     tma::mbar_init(&bar[1], 1);
   }
   if (threadIdx.x < L) tw[threadIdx.x] = make_double2(a.Fre[threadIdx.x], a.Fim[threadIdx.x]);
-  for (int e = threadIdx.x; e < PLANE; e += 2 * NT)   // once per launch
-    *reinterpret_cast<double2*>(sS + 2 * e) = make_double2(__ldg(a.Sre + e), __ldg(a.Sim + e));
+  __shared__ uint32_t tmem_base;
+  uint32_t tmem_s = 0;
+  if (BF_TMEM_S) {
+    if (threadIdx.x < 32) {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;\n" ::"r"(tma::smem_addr(&tmem_base)));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;\n");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;\n");
+    // this thread's lane quadrant and column set (see BF_TMEM_S)
+    tmem_s = tmem_base + ((uint32_t)(32 * (warp & 3)) << 16) + 64 * (warp >> 2);
+    if (grp == 0) {   // group 0 fills the (shared) S values of its P3 lines
+      const int rc = lane + ((warp & 1) << 5), blk = warp >> 1;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint32_t v[16];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int idx = ((16 * blk + 4 * q + e) << 6) + rc;
+          const double re = __ldg(a.Sre + idx), im = __ldg(a.Sim + idx);
+          v[4 * e] = (uint32_t)__double2loint(re);
+          v[4 * e + 1] = (uint32_t)__double2hiint(re);
+          v[4 * e + 2] = (uint32_t)__double2loint(im);
+          v[4 * e + 3] = (uint32_t)__double2hiint(im);
+        }
+        tmem_st16(tmem_s + 16 * q, v);
+      }
+      asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;\n");
+  } else {
+    for (int e = threadIdx.x; e < PLANE; e += 2 * NT)   // once per launch
+      *reinterpret_cast<double2*>(sS + 2 * e) = make_double2(__ldg(a.Sre + e), __ldg(a.Sim + e));
+  }
   __syncthreads();
+  if (BF_TMEM_S) asm volatile("tcgen05.fence::after_thread_sync;\n");
   const int64_t stride = 2 * (int64_t)gridDim.x;
   const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
   if (TMA && tid == 0 && p0 < a.win.p_end) issue_pair(a, &tm, geom(a, p0), sR, &bar[grp]);
@@ -292,7 +365,13 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
     }
     const bool has_next = p + stride < a.win.p_end;
     const Geom gn = geom(a, has_next ? p + stride : p);
-    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn);
+    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn, tmem_s);
+  }
+  if (BF_TMEM_S) {
+    asm volatile("tcgen05.fence::before_thread_sync;\n");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;\n");
+    if (threadIdx.x < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;\n" ::"r"(tmem_base));
   }
 }
 
