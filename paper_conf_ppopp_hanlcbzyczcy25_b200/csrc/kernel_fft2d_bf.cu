@@ -49,6 +49,19 @@ constexpr int kAlign = 1024;
 
 __device__ __forceinline__ int wd(int r, int c) { return ((c >> 4) << 10) | (r << 4) | ((c & 15) ^ ((r & 7) << 1)); }
 
+// BF_WARP_LOCAL = 1: P1 rewrites its rows in the layout wn (row swizzle gn below instead of the
+// TMA's r & 7), and P2 / P4 give warp w exactly the eight rows 16 i + 2 w + e (i = 0..3,
+// e = 0..1) its P1 / P5 blocks cover (lane = 8 b + 2 i + e, b = column block).  P1 -> P2 and
+// P4 -> P5 then exchange data only inside a warp (__syncwarp instead of a group barrier: three
+// group barriers per pair instead of five).  gn = i | e << 2 is distinct over a warp's eight
+// rows, so a quarter-warp's eight 16-byte row-pass words stay conflict-free; the row and
+// column segments of P1 / P3 / P5 are conflict-free under any row swizzle.
+#ifndef BF_WARP_LOCAL
+#define BF_WARP_LOCAL 0
+#endif
+__device__ __forceinline__ int gn(int r) { return BF_WARP_LOCAL ? (((r >> 4) & 3) | ((r & 1) << 2)) : (r & 7); }
+__device__ __forceinline__ int wn(int r, int c) { return ((c >> 4) << 10) | (r << 4) | ((c & 15) ^ (gn(r) << 1)); }
+
 __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
@@ -73,6 +86,16 @@ __device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8]) {
                : "r"(taddr));
   asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
 }
+// 16 columns (4 complex S values) in one load, one wait (BF_TMEM_S = 2).
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),
+        "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+}
+
 __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
   asm volatile(
       "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
@@ -117,13 +140,14 @@ __device__ __forceinline__ void issue_pair(const Fft2dArgs& a, const CUtensorMap
 __device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
 
 // The 4 x 4 block of P1/P5: element [i][j] at row 16 i + rr, column 16 j + cc.
+template <bool TMA_LAYOUT>
 __device__ __forceinline__ void load_block(const double* sR, const double* sI, int rr, int cc, double (&xr)[4][4],
                                            double (&xi)[4][4]) {
 #pragma unroll
   for (int i = 0; i < 4; ++i)
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      const int o = wd(16 * i + rr, 16 * j + cc);
+      const int o = TMA_LAYOUT ? wd(16 * i + rr, 16 * j + cc) : wn(16 * i + rr, 16 * j + cc);
       xr[i][j] = sR[o];
       xi[i][j] = sI[o];
     }
@@ -140,30 +164,68 @@ __device__ __forceinline__ void dft4x4(double (&xr)[4][4], double (&xi)[4][4]) {
     dft4<INV>(xr[i][0], xi[i][0], xr[i][1], xi[i][1], xr[i][2], xi[i][2], xr[i][3], xi[i][3]);
 }
 
-// element [i][j] *= w64^(+-(rr i + cc j)) (conjugate if INV); tw = shared w64^m table.
+// element [i][j] *= w64^(+-(rr i + cc j)) (conjugate if INV).  BF_TW_REG = 1: two table loads
+// (w64^rr, one address per half-warp; w64^cc, 16 consecutive words) and their squares and cubes
+// formed in registers (16 FP64 instructions instead of four more lane-varying shared-memory
+// loads, which conflict for j = 2); BF_TW_REG = 0: all six powers from the shared w64^m table.
+#ifndef BF_TW_REG
+#define BF_TW_REG 0
+#endif
+// BF_TW_COMB = 1: one multiply by the combined w64^(rr i + cc j) per element (15 complex
+// multiplies, 15 table loads) instead of a row and a column twiddle (24 multiplies, 6 loads).
+#ifndef BF_TW_COMB
+#define BF_TW_COMB 0
+#endif
+
+__device__ __forceinline__ void powers3(double2 w, double2 (&p)[4]) {
+  p[1] = w;
+  p[2] = make_double2(fma(w.x, w.x, -w.y * w.y), 2.0 * (w.x * w.y));
+  p[3] = make_double2(fma(w.x, p[2].x, -w.y * p[2].y), fma(w.x, p[2].y, w.y * p[2].x));
+}
+
 template <bool INV>
 __device__ __forceinline__ void twiddle4x4(double (&xr)[4][4], double (&xi)[4][4], const double2* tw, int rr,
                                            int cc) {
+  if (BF_TW_COMB) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (i | j) {
+          const double2 w = tw[(rr * i + cc * j) & 63];
+          cmul(xr[i][j], xi[i][j], w.x, INV ? -w.y : w.y);
+        }
+    return;
+  }
+  double2 pr[4], pc[4];
+  if (BF_TW_REG) {
+    powers3(tw[rr], pr);
+    powers3(tw[cc], pc);
+  } else {
+#pragma unroll
+    for (int i = 1; i < 4; ++i) {
+      pr[i] = tw[(rr * i) & 63];
+      pc[i] = tw[(cc * i) & 63];
+    }
+  }
 #pragma unroll
   for (int i = 1; i < 4; ++i) {
-    const double2 w = tw[(rr * i) & 63];
-    const double wi = INV ? -w.y : w.y;
+    const double wi = INV ? -pr[i].y : pr[i].y;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) cmul(xr[i][j], xi[i][j], w.x, wi);
+    for (int j = 0; j < 4; ++j) cmul(xr[i][j], xi[i][j], pr[i].x, wi);
   }
 #pragma unroll
   for (int j = 1; j < 4; ++j) {
-    const double2 w = tw[(cc * j) & 63];
-    const double wi = INV ? -w.y : w.y;
+    const double wi = INV ? -pc[j].y : pc[j].y;
 #pragma unroll
-    for (int i = 0; i < 4; ++i) cmul(xr[i][j], xi[i][j], w.x, wi);
+    for (int i = 0; i < 4; ++i) cmul(xr[i][j], xi[i][j], pc[j].x, wi);
   }
 }
 
-// P2/P4: the 16 columns 16 b + m of row r as 16-byte words (chunk (m >> 1) ^ (r & 7)).
+// P2/P4: the 16 columns 16 b + m of row r as 16-byte words (chunk (m >> 1) ^ gn(r)).
 template <bool INV>
 __device__ __forceinline__ void row_pass(double* sR, double* sI, int r, int b) {
-  const int base = (b << 10) | (r << 4), s = r & 7;
+  const int base = (b << 10) | (r << 4), s = gn(r);
   double xr[16], xi[16];
 #pragma unroll
   for (int c = 0; c < 8; ++c) {
@@ -191,37 +253,50 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
                                             uint32_t tmem_s) {
   const int S = a.S, h = a.h;
   const int rr = (warp << 1) | (lane >> 4), cc = lane & 15;     // P1/P5 block classes
-  const int rc = lane + ((warp & 1) << 5), blk = warp >> 1;      // P2/P3/P4 row or column, block
+  const int rc = lane + ((warp & 1) << 5), blk = warp >> 1;      // P3 column, row block
+  // P2/P4 row and column block (BF_WARP_LOCAL: the warp's P1/P5 rows)
+  const int r2 = BF_WARP_LOCAL ? ((((lane & 7) >> 1) << 4) | (warp << 1) | (lane & 1)) : rc;
+  const int b2 = BF_WARP_LOCAL ? (lane >> 3) : blk;
   // ---- P1: stage 1 of both axes ----
   {
     double xr[4][4], xi[4][4];
-    load_block(sR, sI, rr, cc, xr, xi);
+    load_block<true>(sR, sI, rr, cc, xr, xi);
     dft4x4<false>(xr, xi);
     twiddle4x4<false>(xr, xi, tw, rr, cc);
+    if (BF_WARP_LOCAL) __syncwarp();   // the warp's rows are rewritten in layout wn
 #pragma unroll
     for (int i = 0; i < 4; ++i)
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
-        const int o = wd(16 * i + rr, 16 * j + cc);
+        const int o = wn(16 * i + rr, 16 * j + cc);
         sR[o] = xr[i][j];
         sI[o] = xi[i][j];
       }
   }
-  group_sync(grp);
-  // ---- P2: axis 1, DFT-16 along row rc in column block blk ----
-  row_pass<false>(sR, sI, rc, blk);
+  if (BF_WARP_LOCAL) __syncwarp(); else group_sync(grp);
+  // ---- P2: axis 1, DFT-16 along row r2 in column block b2 ----
+  row_pass<false>(sR, sI, r2, b2);
   group_sync(grp);
   // ---- P3: axis 0, DFT-16 down column rc in row block blk, * S_T, inverse DFT-16 ----
   {
     double xr[16], xi[16];
 #pragma unroll
     for (int m = 0; m < 16; ++m) {
-      const int o = wd(16 * blk + m, rc);
+      const int o = wn(16 * blk + m, rc);
       xr[m] = sR[o];
       xi[m] = sI[o];
     }
     fft16<false>(xr, xi);   // slot k': position 16 blk + k' <-> frequency blk + 4 k'
-    if (BF_TMEM_S) {
+    if (BF_TMEM_S == 2) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {   // 4 complex values per 16-column load
+        uint32_t v[16];
+        tmem_ld16(tmem_s + 16 * q, v);
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          cmul(xr[4 * q + e], xi[4 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
+      }
+    } else if (BF_TMEM_S) {
 #pragma unroll
       for (int q = 0; q < 8; ++q) {   // 2 complex values per 8-column load
         uint32_t v[8];
@@ -240,18 +315,18 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
     fft16<true>(xr, xi);
 #pragma unroll
     for (int m = 0; m < 16; ++m) {
-      const int o = wd(16 * blk + m, rc);
+      const int o = wn(16 * blk + m, rc);
       sR[o] = xr[m];
       sI[o] = xi[m];
     }
   }
   group_sync(grp);
   // ---- P4: axis 1 inverse DFT-16 ----
-  row_pass<true>(sR, sI, rc, blk);
-  group_sync(grp);
+  row_pass<true>(sR, sI, r2, b2);
+  if (BF_WARP_LOCAL) __syncwarp(); else group_sync(grp);
   // ---- P5: conj twiddles, inverse stage 1 of both axes, store (read, release, compute) ----
   double xr[4][4], xi[4][4];
-  load_block(sR, sI, rr, cc, xr, xi);
+  load_block<false>(sR, sI, rr, cc, xr, xi);
   if (TMA) tma::fence_proxy_async();   // the buffer is refilled by TMA after the barrier
   group_sync(grp);
   if (TMA && warp == 0 && lane == 0 && has_next) issue_pair(a, tm, gn, sR, bar);
