@@ -139,6 +139,30 @@ __device__ __forceinline__ void issue_pair(const Fft2dArgs& a, const CUtensorMap
 // Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
 __device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
 
+// BF_PINGPONG = 1: the two groups take turns at shared memory (the FA3 "ping-pong" schedule).
+// Each pass of a group is a memory phase M (the previous pass's shared stores, the group
+// barrier, this pass's shared loads) followed by a compute phase C (butterflies in registers);
+// group g starts an M phase with bar.sync on barrier 3 + g and ends it -- once its loads have
+// returned -- with bar.arrive on the other group's barrier, so one group's butterflies run
+// while the other group moves data.  Group 0 skips the wait of its very first phase and group 1
+// the arrive of its very last one (group 1, which may own one pair fewer, pads with turns that
+// do no work), so the two barriers see matched sync / arrive counts.
+#ifndef BF_PINGPONG
+#define BF_PINGPONG 0
+#endif
+__device__ __forceinline__ void pp_begin(int grp, bool first_phase) {
+  if (BF_PINGPONG && !(grp == 0 && first_phase))
+    asm volatile("bar.sync %0, %1;\n" ::"r"(3 + grp), "r"(2 * NT) : "memory");
+}
+// a0..a3: loaded values, so the arrive waits for the phase's loads to return
+// (BF_PINGPONG = 2: arrive as soon as the loads are issued)
+__device__ __forceinline__ void pp_end(int grp, bool last_phase, double a0, double a1, double a2, double a3) {
+  if (BF_PINGPONG == 1 && !(grp == 1 && last_phase))
+    asm volatile("bar.arrive %0, %1;\n" ::"r"(4 - grp), "r"(2 * NT), "d"(a0), "d"(a1), "d"(a2), "d"(a3) : "memory");
+  if (BF_PINGPONG == 2 && !(grp == 1 && last_phase))
+    asm volatile("bar.arrive %0, %1;\n" ::"r"(4 - grp), "r"(2 * NT) : "memory");
+}
+
 // The 4 x 4 block of P1/P5: element [i][j] at row 16 i + rr, column 16 j + cc.
 template <bool TMA_LAYOUT>
 __device__ __forceinline__ void load_block(const double* sR, const double* sI, int rr, int cc, double (&xr)[4][4],
@@ -223,10 +247,9 @@ __device__ __forceinline__ void twiddle4x4(double (&xr)[4][4], double (&xi)[4][4
 }
 
 // P2/P4: the 16 columns 16 b + m of row r as 16-byte words (chunk (m >> 1) ^ gn(r)).
-template <bool INV>
-__device__ __forceinline__ void row_pass(double* sR, double* sI, int r, int b) {
+__device__ __forceinline__ void row_load(const double* sR, const double* sI, int r, int b, double (&xr)[16],
+                                         double (&xi)[16]) {
   const int base = (b << 10) | (r << 4), s = gn(r);
-  double xr[16], xi[16];
 #pragma unroll
   for (int c = 0; c < 8; ++c) {
     const int o = base + ((c ^ s) << 1);
@@ -235,7 +258,10 @@ __device__ __forceinline__ void row_pass(double* sR, double* sI, int r, int b) {
     xr[2 * c] = vr.x; xr[2 * c + 1] = vr.y;
     xi[2 * c] = vi.x; xi[2 * c + 1] = vi.y;
   }
-  fft16<INV>(xr, xi);
+}
+__device__ __forceinline__ void row_store(double* sR, double* sI, int r, int b, const double (&xr)[16],
+                                          const double (&xi)[16]) {
+  const int base = (b << 10) | (r << 4), s = gn(r);
 #pragma unroll
   for (int c = 0; c < 8; ++c) {
     const int o = base + ((c ^ s) << 1);
@@ -243,95 +269,123 @@ __device__ __forceinline__ void row_pass(double* sR, double* sI, int r, int b) {
     *reinterpret_cast<double2*>(sI + o) = make_double2(xi[2 * c], xi[2 * c + 1]);
   }
 }
+// P3: the 16 rows 16 blk + m of column rc (8-byte words).
+__device__ __forceinline__ void col_load(const double* sR, const double* sI, int rc, int blk, double (&xr)[16],
+                                         double (&xi)[16]) {
+#pragma unroll
+  for (int m = 0; m < 16; ++m) {
+    const int o = wn(16 * blk + m, rc);
+    xr[m] = sR[o];
+    xi[m] = sI[o];
+  }
+}
+__device__ __forceinline__ void col_store(double* sR, double* sI, int rc, int blk, const double (&xr)[16],
+                                          const double (&xi)[16]) {
+#pragma unroll
+  for (int m = 0; m < 16; ++m) {
+    const int o = wn(16 * blk + m, rc);
+    sR[o] = xr[m];
+    sI[o] = xi[m];
+  }
+}
+__device__ __forceinline__ void block_store(double* sR, double* sI, int rr, int cc, const double (&xr)[4][4],
+                                            const double (&xi)[4][4]) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int o = wn(16 * i + rr, 16 * j + cc);
+      sR[o] = xr[i][j];
+      sI[o] = xi[i][j];
+    }
+}
 
-// The five passes over the pair in (sR, sI) by group `grp`; releases the buffer (TMA refill
-// of the group's next pair `gn`) after P5's reads, then stores the window.
+// The five passes over the pair in (sR, sI) by group `grp`, whose tile data are in place (the
+// caller waited for them in the first memory phase); releases the buffer (TMA refill of the
+// group's next pair `gn`) after P5's reads, then stores the window.  M / C mark the memory and
+// compute phases of the ping-pong schedule (BF_PINGPONG).
 template <bool TMA>
 __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double* sS, const double2* tw,
                                             const Fft2dArgs& a, const Geom& g, int warp, int lane, int grp,
                                             const CUtensorMap* tm, uint64_t* bar, bool has_next, const Geom& gn,
-                                            uint32_t tmem_s) {
+                                            uint32_t tmem_s, bool last) {
   const int S = a.S, h = a.h;
   const int rr = (warp << 1) | (lane >> 4), cc = lane & 15;     // P1/P5 block classes
   const int rc = lane + ((warp & 1) << 5), blk = warp >> 1;      // P3 column, row block
   // P2/P4 row and column block (BF_WARP_LOCAL: the warp's P1/P5 rows)
   const int r2 = BF_WARP_LOCAL ? ((((lane & 7) >> 1) << 4) | (warp << 1) | (lane & 1)) : rc;
   const int b2 = BF_WARP_LOCAL ? (lane >> 3) : blk;
-  // ---- P1: stage 1 of both axes ----
+  double xr[16], xi[16];
   {
-    double xr[4][4], xi[4][4];
-    load_block<true>(sR, sI, rr, cc, xr, xi);
-    dft4x4<false>(xr, xi);
-    twiddle4x4<false>(xr, xi, tw, rr, cc);
+    // ---- P1 (M: loads) (C: stage 1 of both axes) ----
+    double br[4][4], bi[4][4];
+    load_block<true>(sR, sI, rr, cc, br, bi);
+    pp_end(grp, false, br[0][0], bi[0][0], br[3][3], bi[3][3]);
+    dft4x4<false>(br, bi);
+    twiddle4x4<false>(br, bi, tw, rr, cc);
+    // ---- P2 (M: P1 stores, barrier, loads) (C: axis 1, DFT-16 along row r2, block b2) ----
+    pp_begin(grp, false);
     if (BF_WARP_LOCAL) __syncwarp();   // the warp's rows are rewritten in layout wn
-#pragma unroll
-    for (int i = 0; i < 4; ++i)
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int o = wn(16 * i + rr, 16 * j + cc);
-        sR[o] = xr[i][j];
-        sI[o] = xi[i][j];
-      }
+    block_store(sR, sI, rr, cc, br, bi);
   }
   if (BF_WARP_LOCAL) __syncwarp(); else group_sync(grp);
-  // ---- P2: axis 1, DFT-16 along row r2 in column block b2 ----
-  row_pass<false>(sR, sI, r2, b2);
+  row_load(sR, sI, r2, b2, xr, xi);
+  pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
+  fft16<false>(xr, xi);
+  // ---- P3 (M: P2 stores, barrier, loads) (C: axis 0 DFT-16 down column rc in row block blk,
+  //      * S_T, inverse DFT-16) ----
+  pp_begin(grp, false);
+  row_store(sR, sI, r2, b2, xr, xi);
   group_sync(grp);
-  // ---- P3: axis 0, DFT-16 down column rc in row block blk, * S_T, inverse DFT-16 ----
-  {
-    double xr[16], xi[16];
+  col_load(sR, sI, rc, blk, xr, xi);
+  pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
+  fft16<false>(xr, xi);   // slot k': position 16 blk + k' <-> frequency blk + 4 k'
+  if (BF_TMEM_S == 2) {
 #pragma unroll
-    for (int m = 0; m < 16; ++m) {
-      const int o = wn(16 * blk + m, rc);
-      xr[m] = sR[o];
-      xi[m] = sI[o];
+    for (int q = 0; q < 4; ++q) {   // 4 complex values per 16-column load
+      uint32_t v[16];
+      tmem_ld16(tmem_s + 16 * q, v);
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+        cmul(xr[4 * q + e], xi[4 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
     }
-    fft16<false>(xr, xi);   // slot k': position 16 blk + k' <-> frequency blk + 4 k'
-    if (BF_TMEM_S == 2) {
+  } else if (BF_TMEM_S) {
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {   // 4 complex values per 16-column load
-        uint32_t v[16];
-        tmem_ld16(tmem_s + 16 * q, v);
+    for (int q = 0; q < 8; ++q) {   // 2 complex values per 8-column load
+      uint32_t v[8];
+      tmem_ld8(tmem_s + 8 * q, v);
 #pragma unroll
-        for (int e = 0; e < 4; ++e)
-          cmul(xr[4 * q + e], xi[4 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
-      }
-    } else if (BF_TMEM_S) {
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {   // 2 complex values per 8-column load
-        uint32_t v[8];
-        tmem_ld8(tmem_s + 8 * q, v);
-#pragma unroll
-        for (int e = 0; e < 2; ++e)
-          cmul(xr[2 * q + e], xi[2 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
-      }
-    } else {
-#pragma unroll
-      for (int k = 0; k < 16; ++k) {
-        const double2 sv = *reinterpret_cast<const double2*>(sS + ((((16 * blk + k) << 6) + rc) << 1));
-        cmul(xr[k], xi[k], sv.x, sv.y);
-      }
+      for (int e = 0; e < 2; ++e)
+        cmul(xr[2 * q + e], xi[2 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
     }
-    fft16<true>(xr, xi);
+  } else {
 #pragma unroll
-    for (int m = 0; m < 16; ++m) {
-      const int o = wn(16 * blk + m, rc);
-      sR[o] = xr[m];
-      sI[o] = xi[m];
+    for (int k = 0; k < 16; ++k) {
+      const double2 sv = *reinterpret_cast<const double2*>(sS + ((((16 * blk + k) << 6) + rc) << 1));
+      cmul(xr[k], xi[k], sv.x, sv.y);
     }
   }
+  fft16<true>(xr, xi);
+  // ---- P4 (M: P3 stores, barrier, loads) (C: axis 1 inverse DFT-16) ----
+  pp_begin(grp, false);
+  col_store(sR, sI, rc, blk, xr, xi);
   group_sync(grp);
-  // ---- P4: axis 1 inverse DFT-16 ----
-  row_pass<true>(sR, sI, r2, b2);
+  row_load(sR, sI, r2, b2, xr, xi);
+  pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
+  fft16<true>(xr, xi);
+  // ---- P5 (M: P4 stores, barrier, loads, release) (C: conj twiddles, inverse stage 1 of both
+  //      axes, store the window) ----
+  pp_begin(grp, false);
+  row_store(sR, sI, r2, b2, xr, xi);
   if (BF_WARP_LOCAL) __syncwarp(); else group_sync(grp);
-  // ---- P5: conj twiddles, inverse stage 1 of both axes, store (read, release, compute) ----
-  double xr[4][4], xi[4][4];
-  load_block<false>(sR, sI, rr, cc, xr, xi);
+  double br[4][4], bi[4][4];
+  load_block<false>(sR, sI, rr, cc, br, bi);
   if (TMA) tma::fence_proxy_async();   // the buffer is refilled by TMA after the barrier
   group_sync(grp);
   if (TMA && warp == 0 && lane == 0 && has_next) issue_pair(a, tm, gn, sR, bar);
-  twiddle4x4<true>(xr, xi, tw, rr, cc);
-  dft4x4<true>(xr, xi);
+  pp_end(grp, last, br[0][0], bi[0][0], br[3][3], bi[3][3]);
+  twiddle4x4<true>(br, bi, tw, rr, cc);
+  dft4x4<true>(br, bi);
   // column predicates once per pass (valid window [h, h + S), grid limit, tile b present)
   const int64_t ca = g.oa1 + cc, cb = g.ob1 + cc;
   bool va[4], vb[4];
@@ -352,8 +406,8 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
     double* drow = dbase + (int64_t)r * a.n1;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      if (va[j]) drow[ca + 16 * j] = xr[i][j];
-      if (vb[j]) drow[cb + 16 * j] = xi[i][j];
+      if (va[j]) drow[ca + 16 * j] = br[i][j];
+      if (vb[j]) drow[cb + 16 * j] = bi[i][j];
     }
   }
 }
@@ -415,9 +469,25 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
   const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
   if (TMA && tid == 0 && p0 < a.win.p_end) issue_pair(a, &tm, geom(a, p0), sR, &bar[grp]);
 
+  // pairs of this group and of group 0 (which owns as many as group 1 or one more)
+  const int64_t pb0 = a.win.p_begin + 2 * (int64_t)blockIdx.x;
+  const int64_t n0 = pb0 < a.win.p_end ? (a.win.p_end - pb0 + stride - 1) / stride : 0;
+  const int64_t nmine = p0 < a.win.p_end ? (a.win.p_end - p0 + stride - 1) / stride : 0;
+  const int64_t niter = BF_PINGPONG ? n0 : nmine;
   uint32_t parity = 0;
-  for (int64_t p = p0; p < a.win.p_end; p += stride) {
+  for (int64_t it = 0; it < niter; ++it) {
+    const int64_t p = p0 + it * stride;
+    const bool last = it == niter - 1;
+    if (it >= nmine) {   // ping-pong turns without work (group 1)
+#pragma unroll 1
+      for (int k = 0; k < 5; ++k) {
+        pp_begin(grp, false);
+        pp_end(grp, last && k == 4, 0.0, 0.0, 0.0, 0.0);
+      }
+      continue;
+    }
     const Geom g = geom(a, p);
+    pp_begin(grp, it == 0);   // M of P1: the tile's arrival and P1's loads
     if (TMA) {
       tma::mbar_wait(&bar[grp], parity);
       parity ^= 1;
@@ -440,7 +510,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
     }
     const bool has_next = p + stride < a.win.p_end;
     const Geom gn = geom(a, has_next ? p + stride : p);
-    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn, tmem_s);
+    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn, tmem_s, last);
   }
   if (BF_TMEM_S) {
     asm volatile("tcgen05.fence::before_thread_sync;\n");

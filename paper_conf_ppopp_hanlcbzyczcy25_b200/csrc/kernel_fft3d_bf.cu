@@ -67,6 +67,22 @@ __device__ __forceinline__ void stc(double* b, int o, double re, double im) {
 // Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
 __device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
 
+// BF3_PINGPONG = 1: the two groups take turns at shared memory (ping-pong schedule, as
+// kernel_fft2d_bf.cu's BF_PINGPONG): each pass is a memory phase (previous pass's stores,
+// barrier, this pass's loads) then a compute phase; group g waits on barrier 3 + g before a
+// memory phase and arrives on the other group's barrier once its loads have returned.
+#ifndef BF3_PINGPONG
+#define BF3_PINGPONG 0
+#endif
+__device__ __forceinline__ void pp_begin(int grp, bool first_phase) {
+  if (BF3_PINGPONG && !(grp == 0 && first_phase))
+    asm volatile("bar.sync %0, %1;\n" ::"r"(3 + grp), "r"(2 * NT) : "memory");
+}
+__device__ __forceinline__ void pp_end(int grp, bool last_phase, double a0, double a1, double a2, double a3) {
+  if (BF3_PINGPONG && !(grp == 1 && last_phase))
+    asm volatile("bar.arrive %0, %1;\n" ::"r"(4 - grp), "r"(2 * NT), "d"(a0), "d"(a1), "d"(a2), "d"(a3) : "memory");
+}
+
 struct PairGeom {
   int64_t o0, o1, oa2, ob2;
   bool has_b;
@@ -119,9 +135,25 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
   };
   if (TMA && tid == 0 && p0 < a.win.p_end) issue(p0);
 
+  // pairs of this group and of group 0 (which owns as many as group 1 or one more)
+  const int64_t pb0 = a.win.p_begin + 2 * (int64_t)blockIdx.x;
+  const int64_t n0 = pb0 < a.win.p_end ? (a.win.p_end - pb0 + stride - 1) / stride : 0;
+  const int64_t nmine = p0 < a.win.p_end ? (a.win.p_end - p0 + stride - 1) / stride : 0;
+  const int64_t niter = BF3_PINGPONG ? n0 : nmine;
   uint32_t parity = 0;
-  for (int64_t p = p0; p < a.win.p_end; p += stride) {
+  for (int64_t it = 0; it < niter; ++it) {
+    const int64_t p = p0 + it * stride;
+    const bool last = it == niter - 1;
+    if (it >= nmine) {   // ping-pong turns without work (group 1)
+#pragma unroll 1
+      for (int k = 0; k < 5; ++k) {
+        pp_begin(grp, false);
+        pp_end(grp, last && k == 4, 0.0, 0.0, 0.0, 0.0);
+      }
+      continue;
+    }
     const PairGeom g = pair_geom(a, p);
+    pp_begin(grp, it == 0);   // M of P1: the tile's arrival and P1's loads
     if (TMA) {
       tma::mbar_wait(&bar[grp], parity);
       parity ^= 1;
@@ -146,7 +178,9 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     double xr[16], xi[16];
     // ---- P1: forward axis 2 (thread = row (l0, l1) = (hi, lo)); TMA planes -> interleaved ----
     load_row(sR, sI, hi, lo, xr, xi);
+    pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
     radix::fft16<false>(xr, xi);
+    pp_begin(grp, false);   // M of P2: P1's stores and P2's loads
 #pragma unroll
     for (int l2 = 0; l2 < 16; ++l2) stc(sR, cofs(hi, lo, l2), xr[l2], xi[l2]);
     __syncwarp();
@@ -157,7 +191,9 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
       xr[l1] = v.x;
       xi[l1] = v.y;
     }
+    pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
     radix::fft16<false>(xr, xi);
+    pp_begin(grp, false);   // M of P3
 #pragma unroll
     for (int l1 = 0; l1 < 16; ++l1) stc(sR, cofs(hi, l1, lo), xr[l1], xi[l1]);
     group_sync(grp);
@@ -170,6 +206,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
         xr[l0] = v.x;
         xi[l0] = v.y;
       }
+      pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
       radix::fft16<false>(xr, xi);
 #pragma unroll
       for (int k0 = 0; k0 < 16; ++k0) {
@@ -177,6 +214,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
         radix::cmul(xr[k0], xi[k0], sv.x, sv.y);
       }
       radix::fft16<true>(xr, xi);
+      pp_begin(grp, false);   // M of P4
 #pragma unroll
       for (int l0 = 0; l0 < 16; ++l0)
         if (l0 >= h && l0 < h + S) stc(sR, b + (l0 << 8), xr[l0], xi[l0]);
@@ -190,7 +228,11 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
         xr[l1] = v.x;
         xi[l1] = v.y;
       }
-      radix::fft16<true>(xr, xi);
+    }
+    pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
+    if (hi < S) radix::fft16<true>(xr, xi);
+    pp_begin(grp, false);   // M of P5
+    if (hi < S) {
 #pragma unroll
       for (int l1 = 0; l1 < 16; ++l1)
         if (l1 >= h && l1 < h + S) stc(sR, cofs(h + hi, l1, lo), xr[l1], xi[l1]);
@@ -211,6 +253,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     if (TMA) tma::fence_proxy_async();
     group_sync(grp);
     if (TMA && tid == 0 && p + stride < a.win.p_end) issue(p + stride);
+    pp_end(grp, last, xr[0], xi[0], xr[15], xi[15]);
     if (p5) {
       const int l0 = h + hi, l1 = h + lo;
       radix::fft16<true>(xr, xi);
