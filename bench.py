@@ -35,6 +35,25 @@ FP64_PEAK_TFLOPS = 37.18   # measured DMMA.8x8x4 peak on this pool's B200 (profi
 FP64_ALU_PEAK_TOPS = 34.13 / 2   # measured DFMA 34.13 TF/s = 17.07 T FP64 instructions/s
 FP64_ALU_PEAK_SOURCE = ("measured: tools/fp64_peak.cu DFMA microbenchmark 34.13 TFLOP/s / 2 flops per DFMA "
                         "(profiles/r01_fp64_peak.txt); one DADD/DMUL/DFMA = one FP64 pipe slot")
+# Shared memory: 128 B per clock per SM (crossbar, /opt/skills/guides/B300_MICROARCH.md "LDS/STS"),
+# 148 SMs at the 1.965 GHz max SM clock.
+SMEM_PEAK_TBPS = 128 * 148 * 1.965e9 / 1e12
+
+
+def smem_wavefronts_per_pair(info) -> float:
+    """Designed shared-memory wavefronts (128 B each) per tile pair of the ALU kernels
+    (DESIGN.md §5): every pass reads and writes the 64 KB complex pair (512 wavefronts each way)
+    except where it is cropped, plus one read of S_T (512).  Twiddle-table loads and the TMA
+    writes (async proxy) are not counted."""
+    nd = info["ndim"]
+    if nd == 2:       # P1..P4 read + write, P5 read, S_T
+        return 9 * 512 + 512
+    if nd == 3:       # P1, P2 full; P3 reads all, writes S planes; P4 on S planes; P5 on S^2 rows
+        S = info["valid"][0]
+        return 4 * 512 + 512 + 512 * S / 16 + 512 * S / 16 + 2 * 512 * S * S / 256 + 512
+    return 13 * 512 + 512   # 1D: P1..P6 read + write, P7 read, S_T
+
+
 FP64_PEAK_SOURCE = ("measured: tools/fp64_peak.cu DMMA m8n8k4 microbenchmark, 148 SMs x 64 FMA/clk x 1.965 GHz "
                     "(profiles/r01_fp64_peak.txt); MEASURED_PEAKS.json carries no FP64 figure")
 
@@ -305,6 +324,14 @@ def main():
                          "frac": ops / FP64_ALU_PEAK_TOPS, "dtype": "f64 (DADD/DMUL/DFMA)",
                          "peak_source": FP64_ALU_PEAK_SOURCE, "alu_ops_per_launch": info["alu_ops_per_pass"],
                          "alg_tflops": achieved})
+        # the other unit the ALU kernels lean on (ncu: both below saturation)
+        pairs = info["pair_end"] - info["pair_begin"]
+        wf = smem_wavefronts_per_pair(info)
+        smem_tbps = pairs * wf * 128 / fused_avg_s / 1e12
+        roofline["smem"] = {"achieved": smem_tbps, "peak": SMEM_PEAK_TBPS, "unit": "TB/s",
+                            "frac": smem_tbps / SMEM_PEAK_TBPS, "wavefronts_per_pair": wf,
+                            "note": "designed LSU shared-memory traffic (no twiddle loads, no TMA writes) / "
+                                    "fused-kernel time vs 128 B/clk/SM x 148 SMs x 1.965 GHz"}
 
     # ---- end to end through the host-buffer C-ABI entry point ----
     e2e = None

@@ -26,3 +26,12 @@ def test_weak_scaling_counts_each_slab_once():
             cells *= e
         # perfect weak scaling (same time per rank) reports exactly world x the 1-GPU value
         assert abs(bench.gstencils(cells, 1000, 50.0) / one - world) < 1e-12
+
+
+def test_smem_wavefront_model():
+    # 2D five passes (4 read + write, 1 read) + S_T; 3D cropped inverse passes
+    assert bench.smem_wavefronts_per_pair({"ndim": 2}) == 10 * 512
+    assert bench.smem_wavefronts_per_pair({"ndim": 3, "valid": [12, 12, 12]}) == 4416
+    assert bench.smem_wavefronts_per_pair({"ndim": 3, "valid": [16, 16, 16]}) == 10 * 512
+    assert bench.smem_wavefronts_per_pair({"ndim": 1}) == 14 * 512
+    assert abs(bench.SMEM_PEAK_TBPS - 37.22496) < 1e-9
