@@ -171,6 +171,17 @@ def gstencils(global_cells: int, time_steps: int, ms: float) -> float:
     return global_cells * time_steps / (ms / 1e3) / 1e9
 
 
+def cpu_model() -> str:
+    """The host CPU's model name (/proc/cpuinfo), reported beside the oracle's core count."""
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def cpu_oracle_sample(wk, w, budget_s: float = 12.0):
     """Time the oracle as it stands on the host cores on a bounded sample."""
     import oracle
@@ -187,6 +198,7 @@ def cpu_oracle_sample(wk, w, budget_s: float = 12.0):
         t1 = time.perf_counter() - t0
     cells = int(np.prod(wk.extents))
     return {"value": cells * steps / t1 / 1e9, "unit": "GStencils/s", "cores": threads, "kind": "oracle",
+            "cpu_model": cpu_model(),
             "sample": f"full {wk.name} grid {'x'.join(map(str, wk.extents))}, {steps} direct time step(s), "
                       f"{t1:.1f} s wall, OMP threads={threads}"}
 
@@ -215,10 +227,12 @@ def run_reference(args):
         "impl": "reference", "metric": "GStencils/s FP64", "value": value, "unit": "GStencils/s",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"{wk.name} {'x'.join(map(str, wk.extents))} (BASELINE configs[1])",
+        "config": {"workload": f"{wk.name} {'x'.join(map(str, wk.extents))}"
+                               + (" (BASELINE configs[1])" if args.workload in ("heat2d", "box2d9p") else ""),
                    "stencil": f"{wk.points}-point {wk.shape} r={wk.radius}, {args.weights} weights",
                    "time_steps_per_step": s_ref, "sample": "full grid, 1 direct time step per bench step"},
         "cpu_baseline": {"value": value, "unit": "GStencils/s", "cores": threads, "kind": "oracle",
+                         "cpu_model": cpu_model(),
                          "sample": f"full grid, {s_ref} direct time step per bench step, {args.steps} timed"},
         "e2e": {"value": value, "unit": "GStencils/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
