@@ -32,9 +32,29 @@ sys.path.insert(0, ROOT)
 from synth import workloads as wl  # noqa: E402
 
 FP64_PEAK_TFLOPS = 37.18   # measured DMMA.8x8x4 peak on this pool's B200 (profiles/r01_fp64_peak.txt)
-FP64_ALU_PEAK_TOPS = 34.13 / 2   # measured DFMA 34.13 TF/s = 17.07 T FP64 instructions/s
-FP64_ALU_PEAK_SOURCE = ("measured: tools/fp64_peak.cu DFMA microbenchmark 34.13 TFLOP/s / 2 flops per DFMA "
-                        "(profiles/r01_fp64_peak.txt); one DADD/DMUL/DFMA = one FP64 pipe slot")
+# Measured FP64 instruction rates on this pool's B200 (tools/fp64_peak.cu, 8 independent chains
+# per thread, 296 x 1024 threads; profiles/r01_s3_fp64_peak.txt), T instructions/s: DADD and
+# DMUL issue at 64 per clock per SM, DFMA slightly slower.
+FP64_RATES_TOPS = {"DADD": 18.51, "DMUL": 18.50, "DFMA": 17.05}
+# FP64 instruction mix (DADD, DMUL, DFMA) of each default ALU kernel: static SASS counts of
+# its TMA instantiation (cuobjdump -sass; the passes are straight-line code, so static =
+# dynamic per thread and pair).  tests/test_bench.py re-counts them from the built objects.
+ALU_KERNEL_MIX = {
+    "kernel_fft2d_bf": (752, 168, 208),
+    "kernel_fft3d_bf": (744, 92, 152),
+    "kernel_fft1d_bf": (752, 292, 332),
+}
+
+
+def alu_peak_tops(mix) -> float:
+    """Peak FP64 instruction rate for a kernel's mix: the time-weighted harmonic mean of the
+    measured per-opcode rates (every DADD / DMUL / DFMA takes one FP64 pipe issue slot)."""
+    n = sum(mix)
+    return n / sum(k / FP64_RATES_TOPS[op] for k, op in zip(mix, ("DADD", "DMUL", "DFMA")))
+
+
+FP64_ALU_PEAK_SOURCE = ("measured: tools/fp64_peak.cu per-opcode rates DADD 18.51 / DMUL 18.50 / DFMA 17.05 T "
+                        "instructions/s (profiles/r01_s3_fp64_peak.txt), weighted by the kernel's SASS FP64 mix")
 # Shared memory: 128 B per clock per SM (crossbar, /opt/skills/guides/B300_MICROARCH.md "LDS/STS"),
 # 148 SMs at the 1.965 GHz max SM clock.
 SMEM_PEAK_TBPS = 128 * 148 * 1.965e9 / 1e12
@@ -334,8 +354,10 @@ def main():
         # FP64 ALU engine: the binding unit is the FP64 pipe's issue rate (adds, multiplies and
         # FMAs each take one slot); peak = the measured DFMA rate / 2 (profiles/r01_fp64_peak.txt)
         ops = info["alu_ops_per_pass"] / fused_avg_s / 1e12
-        roofline.update({"bound": "alu", "achieved": ops, "peak": FP64_ALU_PEAK_TOPS, "unit": "Top/s",
-                         "frac": ops / FP64_ALU_PEAK_TOPS, "dtype": "f64 (DADD/DMUL/DFMA)",
+        mix = ALU_KERNEL_MIX[("kernel_fft1d_bf", "kernel_fft2d_bf", "kernel_fft3d_bf")[info["ndim"] - 1]]
+        peak = alu_peak_tops(mix)
+        roofline.update({"bound": "alu", "achieved": ops, "peak": peak, "unit": "Top/s",
+                         "frac": ops / peak, "dtype": "f64 (DADD/DMUL/DFMA)", "fp64_mix": list(mix),
                          "peak_source": FP64_ALU_PEAK_SOURCE, "alu_ops_per_launch": info["alu_ops_per_pass"],
                          "alg_tflops": achieved})
         # the other unit the ALU kernels lean on (ncu: both below saturation)

@@ -35,3 +35,43 @@ def test_smem_wavefront_model():
     assert bench.smem_wavefronts_per_pair({"ndim": 3, "valid": [16, 16, 16]}) == 10 * 512
     assert bench.smem_wavefronts_per_pair({"ndim": 1}) == 14 * 512
     assert abs(bench.SMEM_PEAK_TBPS - 37.22496) < 1e-9
+
+
+def _sass_mix(obj):
+    """(DADD, DMUL, DFMA) static counts of the TMA instantiation (<true, false>) in `obj`."""
+    import re
+    import subprocess
+    out = subprocess.run(["cuobjdump", "-sass", obj], capture_output=True, text=True).stdout
+    counts = {"DADD": 0, "DMUL": 0, "DFMA": 0}
+    inside = False
+    for ln in out.splitlines():
+        if "Function" in ln:
+            inside = "ILb1ELb0E" in ln
+            continue
+        if inside:
+            for m in re.finditer(r"\b(DADD|DMUL|DFMA)\b", ln):
+                counts[m.group(1)] += 1
+    return counts["DADD"], counts["DMUL"], counts["DFMA"]
+
+
+def test_alu_kernel_mix_matches_build():
+    """bench.py's FP64 mixes (the weights of the ALU peak) are those of the built kernels."""
+    import os
+    import shutil
+
+    import pytest
+    build = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                         "paper_conf_ppopp_hanlcbzyczcy25_b200", "_build")
+    if shutil.which("cuobjdump") is None or not os.path.isdir(build):
+        pytest.skip("needs cuobjdump and a built tree")
+    for name, mix in bench.ALU_KERNEL_MIX.items():
+        obj = os.path.join(build, name + ".cu.o")
+        if not os.path.exists(obj):
+            pytest.skip(f"{obj} not built")
+        assert _sass_mix(obj) == mix, name
+
+
+def test_alu_peak_between_opcode_rates():
+    for mix in bench.ALU_KERNEL_MIX.values():
+        p = bench.alu_peak_tops(mix)
+        assert min(bench.FP64_RATES_TOPS.values()) < p < max(bench.FP64_RATES_TOPS.values())

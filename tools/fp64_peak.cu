@@ -41,6 +41,34 @@ __global__ void dfma_loop(double* out, int iters, double a0, double b0) {
   out[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
 
+// Per-instruction FP64 rate of DADD / DMUL / an FFT-like mix (2 DADD : 1 DMUL : 1 DFMA): does
+// every FP64 instruction take one pipe slot (the ALU roofline of bench.py assumes so)?
+// OP 0 = DADD, 1 = DMUL, 2 = mix.  CH independent chains per thread.
+template <int CH, int OP>
+__global__ void op_loop(double* out, int iters, double a0, double b0) {
+  double c[CH];
+#pragma unroll
+  for (int i = 0; i < CH; ++i) c[i] = threadIdx.x * 1e-3 + i;
+  const double a = a0, b = b0;
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int i = 0; i < CH; ++i) {
+      if (OP == 0) c[i] = c[i] + b;
+      else if (OP == 1) c[i] = c[i] * a;
+      else {   // 4 instructions per chain step
+        c[i] = __dadd_rn(c[i], b);   // _rn intrinsics: no FMA contraction
+        c[i] = __dmul_rn(c[i], a);
+        c[i] = __dsub_rn(c[i], b);
+        c[i] = fma(c[i], a, b);
+      }
+    }
+  }
+  double s = 0;
+#pragma unroll
+  for (int i = 0; i < CH; ++i) s += c[i];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
 // DMMA and DFMA interleaved in one warp stream (independent accumulators): tells whether
 // the tensor DMMA path and the FP64 FMA units share throughput on this GPU.
 template <int CH, int NF>
@@ -107,6 +135,24 @@ int main() {
       if (rep) printf("DFMA: warps/block %d blocks %d -> %.2f TFLOP/s (%.3f ms)\n", wpb, blocks, flops / ms / 1e9, ms);
     }
   }
+  {
+    const int wpb = 32, blocks = sms * 2;
+    auto run_op = [&](auto kern, const char* name, double instr_per_iter) {
+      for (int rep = 0; rep < 2; ++rep) {
+        cudaEventRecord(e0);
+        kern<<<blocks, wpb * 32>>>(out, iters, 1.0000001, 1e-9);
+        cudaEventRecord(e1); cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        const double ins = instr_per_iter * (double)iters * blocks * wpb * 32;
+        if (rep) printf("%s: %.3f ms  %.2f T FP64 instructions/s (DFMA equivalent %.2f TF)\n", name, ms, ins / ms / 1e9,
+                        2 * ins / ms / 1e9);
+      }
+    };
+    run_op(op_loop<8, 0>, "DADD x8 chains       ", 8.0);
+    run_op(op_loop<8, 1>, "DMUL x8 chains       ", 8.0);
+    run_op(op_loop<8, 2>, "mix add/mul/sub/fma  ", 32.0);
+    run_op(dfma_loop<8>, "DFMA x8 chains       ", 8.0);
+  }
   // shared or separate FP64 throughput: CH DMMA + NF DFMA per iteration and warp
   {
     const int wpb = 16, blocks = sms * 2;
@@ -122,7 +168,6 @@ int main() {
       }
     };
     run(mix_loop<8, 0>, "mix DMMA x8 only      ", 2.0 * 256 * 8, 0.0);
-    run(mix_loop<8, 64>, "mix DMMA x8 + DFMA x64", 2.0 * 256 * 8, 2.0 * 32 * 64);
     run(mix_loop<8, 32>, "mix DMMA x8 + DFMA x32", 2.0 * 256 * 8, 2.0 * 32 * 32);
     run(mix_loop<8, 16>, "mix DMMA x8 + DFMA x16", 2.0 * 256 * 8, 2.0 * 32 * 16);
   }
