@@ -62,6 +62,31 @@ __device__ __forceinline__ int wd(int r, int c) { return ((c >> 4) << 10) | (r <
 __device__ __forceinline__ int gn(int r) { return BF_WARP_LOCAL ? (((r >> 4) & 3) | ((r & 1) << 2)) : (r & 7); }
 __device__ __forceinline__ int wn(int r, int c) { return ((c >> 4) << 10) | (r << 4) | ((c & 15) ^ (gn(r) << 1)); }
 
+// BF_CPLX = 1: after P1 every element is one 16-byte (re, im) word.  Row r's 64 complex values
+// occupy exactly the bytes row r had in the two TMA planes (1 KB: four 128-byte segments per
+// plane): columns 16 b + 0..7 in the Re plane's segment b, 16 b + 8..15 in the Im plane's, as
+// 16-byte chunk (c & 7) ^ (r & 7).  A half-warp of P1 owns four whole rows, so it converts them
+// in place after a __syncwarp.  Every later access moves one complex value per instruction
+// (LDS.128 / STS.128): 176 shared-memory instructions per thread and pair instead of 240, the
+// same wavefronts (a quarter-warp covers 8 chunks of one segment: 8 consecutive columns of a row
+// in P1 / P3 / P5, 8 consecutive rows of a column chunk in P2 / P4 -> distinct banks).
+#ifndef BF_CPLX
+#define BF_CPLX 0
+#endif
+static_assert(!(BF_CPLX && BF_WARP_LOCAL), "BF_CPLX and BF_WARP_LOCAL are exclusive");
+// double offset of element (r, c)'s (re, im) word from the group buffer base sR
+__device__ __forceinline__ int wc(int r, int c) {
+  return (((c >> 3) & 1) << 12) | ((c >> 4) << 10) | (r << 4) | (((c & 7) ^ (r & 7)) << 1);
+}
+__device__ __forceinline__ void ldc2(const double* b, int o, double& re, double& im) {
+  const double2 v = *reinterpret_cast<const double2*>(b + o);
+  re = v.x;
+  im = v.y;
+}
+__device__ __forceinline__ void stc2(double* b, int o, double re, double im) {
+  *reinterpret_cast<double2*>(b + o) = make_double2(re, im);
+}
+
 __device__ __forceinline__ void cp_async8(double* dst, const double* src, bool valid) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 8 : 0));
@@ -171,6 +196,10 @@ __device__ __forceinline__ void load_block(const double* sR, const double* sI, i
   for (int i = 0; i < 4; ++i)
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
+      if (BF_CPLX && !TMA_LAYOUT) {
+        ldc2(sR, wc(16 * i + rr, 16 * j + cc), xr[i][j], xi[i][j]);
+        continue;
+      }
       const int o = TMA_LAYOUT ? wd(16 * i + rr, 16 * j + cc) : wn(16 * i + rr, 16 * j + cc);
       xr[i][j] = sR[o];
       xi[i][j] = sI[o];
@@ -249,6 +278,11 @@ __device__ __forceinline__ void twiddle4x4(double (&xr)[4][4], double (&xi)[4][4
 // P2/P4: the 16 columns 16 b + m of row r as 16-byte words (chunk (m >> 1) ^ gn(r)).
 __device__ __forceinline__ void row_load(const double* sR, const double* sI, int r, int b, double (&xr)[16],
                                          double (&xi)[16]) {
+  if (BF_CPLX) {
+#pragma unroll
+    for (int m = 0; m < 16; ++m) ldc2(sR, wc(r, 16 * b + m), xr[m], xi[m]);
+    return;
+  }
   const int base = (b << 10) | (r << 4), s = gn(r);
 #pragma unroll
   for (int c = 0; c < 8; ++c) {
@@ -261,6 +295,11 @@ __device__ __forceinline__ void row_load(const double* sR, const double* sI, int
 }
 __device__ __forceinline__ void row_store(double* sR, double* sI, int r, int b, const double (&xr)[16],
                                           const double (&xi)[16]) {
+  if (BF_CPLX) {
+#pragma unroll
+    for (int m = 0; m < 16; ++m) stc2(sR, wc(r, 16 * b + m), xr[m], xi[m]);
+    return;
+  }
   const int base = (b << 10) | (r << 4), s = gn(r);
 #pragma unroll
   for (int c = 0; c < 8; ++c) {
@@ -274,6 +313,10 @@ __device__ __forceinline__ void col_load(const double* sR, const double* sI, int
                                          double (&xi)[16]) {
 #pragma unroll
   for (int m = 0; m < 16; ++m) {
+    if (BF_CPLX) {
+      ldc2(sR, wc(16 * blk + m, rc), xr[m], xi[m]);
+      continue;
+    }
     const int o = wn(16 * blk + m, rc);
     xr[m] = sR[o];
     xi[m] = sI[o];
@@ -283,6 +326,10 @@ __device__ __forceinline__ void col_store(double* sR, double* sI, int rc, int bl
                                           const double (&xi)[16]) {
 #pragma unroll
   for (int m = 0; m < 16; ++m) {
+    if (BF_CPLX) {
+      stc2(sR, wc(16 * blk + m, rc), xr[m], xi[m]);
+      continue;
+    }
     const int o = wn(16 * blk + m, rc);
     sR[o] = xr[m];
     sI[o] = xi[m];
@@ -294,6 +341,10 @@ __device__ __forceinline__ void block_store(double* sR, double* sI, int rr, int 
   for (int i = 0; i < 4; ++i)
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
+      if (BF_CPLX) {
+        stc2(sR, wc(16 * i + rr, 16 * j + cc), xr[i][j], xi[i][j]);
+        continue;
+      }
       const int o = wn(16 * i + rr, 16 * j + cc);
       sR[o] = xr[i][j];
       sI[o] = xi[i][j];
@@ -325,7 +376,7 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
     twiddle4x4<false>(br, bi, tw, rr, cc);
     // ---- P2 (M: P1 stores, barrier, loads) (C: axis 1, DFT-16 along row r2, block b2) ----
     pp_begin(grp, false);
-    if (BF_WARP_LOCAL) __syncwarp();   // the warp's rows are rewritten in layout wn
+    if (BF_WARP_LOCAL || BF_CPLX) __syncwarp();   // the warp's rows are rewritten in layout wn / wc
     block_store(sR, sI, rr, cc, br, bi);
   }
   if (BF_WARP_LOCAL) __syncwarp(); else group_sync(grp);
