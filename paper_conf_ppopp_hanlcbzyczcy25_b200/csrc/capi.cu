@@ -372,6 +372,7 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
   b.g0 = hp.g0;
   b.gn = hp.g1 - hp.g0;
   b.reference = p->band_reference;
+  b.region_cells = hp.band_region_cells;
   cudaStream_t bs = s;
   if (p->band_concurrent) {
     cudaError_t e = cudaEventRecord(p->ev_fork, s);

@@ -236,6 +236,9 @@ cudaError_t band_configure(size_t smem) {
   if ((e = cudaFuncSetAttribute(band_cone_kernel<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
       cudaSuccess)
     return e;
+  if ((e = cudaFuncSetAttribute(band_cone_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
+      cudaSuccess)
+    return e;
   return smem <= lim0 && smem <= lim1 ? cudaSuccess : cudaErrorInvalidValue;
 }
 
@@ -244,8 +247,13 @@ cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s) {
   int taps = 1;
   for (int q = 0; q < 3; ++q) taps *= a.active[q] ? 2 * a.r + 1 : 1;
   const bool one_d = a.active[0] + a.active[1] + a.active[2] == 1;
-  if (taps <= kMaxTaps && !a.reference && one_d)
+  // 1D: 1024 threads for the long bands of deep-fusion plans (t ~ 1000 sequential steps over
+  // thousands of cells); a 64-thread CTA when the region is small (e.g. configs[0]: 23 cells,
+  // where 32 mostly idle warps spent ~150 issue slots each per step: 15 us vs ~3 us)
+  if (taps <= kMaxTaps && !a.reference && one_d && a.region_cells > 512)
     band_cone_kernel<1024><<<a.nblocks, 1024, smem, s>>>(a);
+  else if (taps <= kMaxTaps && !a.reference && one_d)
+    band_cone_kernel<64><<<a.nblocks, 64, smem, s>>>(a);
   else if (taps <= kMaxTaps && !a.reference)
     band_cone_kernel<256><<<a.nblocks, kBandThreads, smem, s>>>(a);
   else
