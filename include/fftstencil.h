@@ -118,7 +118,11 @@ fftstencil_plan* fftstencil_plan_create_ex(int ndim, const int64_t* extents, con
  * legacy default stream).  `in` and `out` are device pointers to prod(extents) FP64
  * values on the plan's device; the caller owns them.  `in` is read only unless it
  * aliases `out` (allowed).  total_steps == 0 copies in to out.  Asynchronous: no host
- * synchronisation.  Returns FFTSTENCIL_OK or a negative code. */
+ * synchronisation.  Returns FFTSTENCIL_OK or a negative code.
+ * Launches: per fused pass the tile kernel (+ the band kernel on a side stream, joined
+ * before the next pass); a small non-periodic 1D grid (PFA tile, <= 8192 cells) runs the
+ * whole call as ONE launch of an 8-CTA cluster with the grid in shared memory
+ * (kernel_small1d.cu; FFTSTENCIL_SMALL1D=0 disables). */
 int fftstencil_run(fftstencil_plan* plan, const double* in, double* out, int64_t total_steps,
                    void* stream);
 

@@ -80,6 +80,7 @@ struct fftstencil_plan {
   // ---- the band kernel runs on a side stream, concurrent with the fused kernel (it reads
   // the same source and writes disjoint cells); FFTSTENCIL_BAND_STREAM=0 serialises it ----
   bool band_concurrent = true;
+  bool small1d = false;       // whole run in one on-chip launch (small 1D PFA plans, kernel_small1d.cu)
   cudaStream_t band_stream = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_band = nullptr;
   bool band_pending = false;
@@ -433,6 +434,36 @@ int run_single(fftstencil_plan* p, const double* in, double* out, int64_t total_
   const int64_t nfull = total_steps / T;
   const int rem = (int)(total_steps % T);
   const int64_t passes = nfull + (rem ? 1 : 0);
+  if (p->small1d) {
+    const HostPlan& hp = p->hp;
+    Small1dArgs a;
+    a.in = in;
+    a.out = out;
+    a.n = hp.ext[0];
+    a.h = hp.h;
+    a.S = hp.S[0];
+    a.L = hp.L[0];
+    a.r = hp.radius;
+    a.T = T;
+    a.rem = rem;
+    a.rmax = (int)std::min<int64_t>(hp.h + (int64_t)hp.radius * T, hp.ext[0]);
+    a.ntiles = hp.tiles;
+    a.passes = passes;
+    a.Fre = p->dF;
+    a.Fim = p->dF + 128;
+    a.crt = p->dCrt;
+    a.Sre_T = p->dS + (size_t)(T - 1) * 2 * p->spec_vol;
+    a.Sim_T = a.Sre_T + p->spec_vol;
+    a.Sre_rem = p->dS + (size_t)((rem ? rem : T) - 1) * 2 * p->spec_vol;
+    a.Sim_rem = a.Sre_rem + p->spec_vol;
+    a.w = p->dW;
+    const long pb = prof_begin(p, 0, s);
+    cudaError_t e = launch_small1d(a, s);
+    prof_end(p, pb, s);
+    if (e != cudaSuccess) return cuda_fail(e, "small 1D launch");
+    ++p->last_launches;
+    return FFTSTENCIL_OK;
+  }
   // destination sequence: alternate out / scratch so the last pass writes `out`;
   // with in == out the first destination must be scratch (a final copy if needed).
   const bool alias = in == out;
@@ -670,6 +701,12 @@ int setup_device(fftstencil_plan* p) {
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->ev_band, cudaEventDisableTiming);
     if (e != cudaSuccess) return cuda_fail(e, "band stream/events");
   }
+  // small non-periodic 1D grids: the whole run in one launch, the grid in shared memory
+  // (FFTSTENCIL_SMALL1D=0 keeps the per-pass driver)
+  p->small1d = hp.ndim == 1 && hp.algo == 0 && !hp.periodic && !p->dist && hp.ext[0] <= kSmall1dMaxCells &&
+               hp.ext[0] >= 4 * (int64_t)hp.h + 2 * hp.radius && std::min<int64_t>(2 * hp.h, hp.ext[0]) <= kSmall1dMaxBand;
+  if (const char* v = std::getenv("FFTSTENCIL_SMALL1D")) p->small1d = p->small1d && std::atoi(v) != 0;
+  if (p->small1d && (e = small1d_configure()) != cudaSuccess) return cuda_fail(e, "small 1D kernel configuration");
   p->band_smem = (size_t)2 * hp.band_region_cells * sizeof(double);
   if (p->band_smem > 0) {
     e = band_configure(p->band_smem);

@@ -25,6 +25,28 @@ __device__ __forceinline__ void dmma(double (&c)[2], double a, double b) {
       : "d"(a), "d"(b));
 }
 
+// Complex 8x8x8 product C = A . B on DMMA, A given as per-thread A fragments (two k-chunks),
+// B as B fragments; CONJ multiplies by conj(A).  4 DMMA per k-chunk (4M form).
+template <bool CONJ>
+__device__ __forceinline__ void cgemm8(const double (&ar)[2], const double (&ai)[2], const double (&br)[2],
+                                       const double (&bi)[2], double (&cr)[2], double (&ci)[2]) {
+  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    if (CONJ) {
+      dmma(cr, ar[j], br[j]);
+      dmma(cr, ai[j], bi[j]);
+      dmma(ci, ar[j], bi[j]);
+      dmma(ci, -ai[j], br[j]);
+    } else {
+      dmma(cr, ar[j], br[j]);
+      dmma(cr, -ai[j], bi[j]);
+      dmma(ci, ar[j], bi[j]);
+      dmma(ci, ai[j], br[j]);
+    }
+  }
+}
+
 // Physical column of logical column c inside its group of 8: even columns first.
 __host__ __device__ __forceinline__ int perm8(int c) {
   return (c & ~7) | ((c & 1) << 2) | ((c & 7) >> 1);

@@ -19,26 +19,7 @@ namespace {
 
 using dev::dmma;
 
-// complex 8x8x8 product C = A . B with A given as per-thread fragments (conj optional)
-template <bool CONJ>
-__device__ __forceinline__ void cgemm8(const double (&ar)[2], const double (&ai)[2], const double (&br)[2],
-                                       const double (&bi)[2], double (&cr)[2], double (&ci)[2]) {
-  cr[0] = cr[1] = ci[0] = ci[1] = 0.0;
-#pragma unroll
-  for (int j = 0; j < 2; ++j) {
-    if (CONJ) {
-      dmma(cr, ar[j], br[j]);
-      dmma(cr, ai[j], bi[j]);
-      dmma(ci, ar[j], bi[j]);
-      dmma(ci, -ai[j], br[j]);
-    } else {
-      dmma(cr, ar[j], br[j]);
-      dmma(cr, -ai[j], bi[j]);
-      dmma(ci, ar[j], bi[j]);
-      dmma(ci, ai[j], br[j]);
-    }
-  }
-}
+using dev::cgemm8;
 
 template <bool WRAP>   // periodic boundary: a separate instantiation (no wrap arithmetic otherwise)
 __global__ void __launch_bounds__(kFft1dWarpsPerBlock * 32) fft1d_kernel(const Fft1dArgs a) {

@@ -139,6 +139,30 @@ cudaError_t launch_fused2d_ct(int cfg, const Fft2dArgs& a, const CUtensorMap* tm
 constexpr int kFft1dWarpsPerBlock = 8;
 cudaError_t fused1d_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused1d(const Fft1dArgs& a, int grid, cudaStream_t s);
+
+// A whole fftstencil_run of a small non-periodic 1D PFA plan in one launch of one CTA, the grid
+// resident in shared memory (kernel_small1d.cu).
+constexpr int64_t kSmall1dMaxCells = 8192;   // 2 buffers = 128 KB of shared memory
+constexpr int kSmall1dMaxBand = 64;          // cells of one band cone region, h + r t <= 2h < 56
+constexpr int kSmall1dMaxR = 8;              // radius limit of the C ABI
+struct Small1dArgs {
+  const double* in;      // global grid (read once)
+  double* out;           // global grid (written once; may alias in)
+  int64_t n;
+  int h, S, L, r, T, rem, rmax;   // rem = steps mod T (0: none); rmax = min(h + r T, n)
+  int64_t ntiles, passes;
+  const double* Fre;     // as Fft1dArgs
+  const double* Fim;
+  const int* crt;
+  const double* Sre_T;   // powered spectra S_T and S_rem (Ruritanian 8 x 8)
+  const double* Sim_T;
+  const double* Sre_rem;
+  const double* Sim_rem;
+  const double* w;       // 2r + 1 weights
+};
+size_t small1d_smem(int64_t n, int rmax);
+cudaError_t small1d_configure();
+cudaError_t launch_small1d(const Small1dArgs& a, cudaStream_t s);
 size_t fused1d_ct_smem();
 // Butterfly ALU engine of the factored 1D tile (kernel_fft1d_bf.cu): Fre/Fim[0..63] = w64^m,
 // tw = w4096^m (m < 256, interleaved); Sre/Sim = S_T at [column position][row position].

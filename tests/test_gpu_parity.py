@@ -499,3 +499,38 @@ def test_parity_1d_engines(fs, monkeypatch, engine, tma, ext, r, T, steps):
     assert p.info()["engine"] == engine and p.info()["T"] == T
     ref = oracle.stencil_run(u0, w, r, steps)
     assert rel_err(got, ref) <= TOL, (rel_err(got, ref), p.info())
+
+
+# ---------------------------------------------------------------- small 1D grids: one launch per run
+SMALL1D_CASES = [c for c in CASES if len(c[0]) == 1] + [((8192,), "star", 3, 4, 41, "seeded"),
+                                                       ((5000,), "star", 2, 6, 6, "classic")]
+
+
+@pytest.mark.parametrize("small", ["1", "0"])
+@pytest.mark.parametrize("ext,shape,r,T,steps,kind", SMALL1D_CASES)
+def test_small1d_whole_run_parity(fs, monkeypatch, small, ext, shape, r, T, steps, kind):
+    """The on-chip whole-run kernel (kernel_small1d.cu) and the per-pass driver both match the
+    oracle; the whole-run path is one launch per fftstencil_run."""
+    monkeypatch.setenv("FFTSTENCIL_SMALL1D", small)
+    w = wl.stencil_weights(shape, 1, r, kind)
+    u0 = wl.grid(ext, 13)
+    got, p = run_gpu(fs, u0, w, r, T, steps)
+    ref = oracle.stencil_run(u0, w, r, steps)
+    assert rel_err(got, ref) <= TOL, p.info()
+    if small == "1" and p.info()["algo"] == "pfa":
+        assert p.info()["last_run_launches"] == 1
+
+
+def test_small1d_in_place_and_zero_steps(fs):
+    ext, r, T = (4096,), 1, 8
+    w = wl.seeded_weights("star", 1, r)
+    u0 = wl.grid(ext, 17)
+    p = fs.Plan(ext, w, r, T)
+    a = torch.from_numpy(u0).cuda()
+    p.run(a, a, 64)   # in == out
+    torch.cuda.synchronize()
+    assert rel_err(a.cpu().numpy(), oracle.stencil_run(u0, w, r, 64)) <= TOL
+    b = torch.empty_like(a)
+    p.run(a, b, 0)
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
