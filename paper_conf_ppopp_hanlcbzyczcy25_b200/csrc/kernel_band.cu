@@ -152,15 +152,48 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
     rlo[q] = a.active[q] ? (int)(r - rl[q]) : -(1 << 30);
     rhi[q] = a.active[q] ? (int)(a.n[q] - r - rl[q]) : (1 << 30);
   }
+#ifndef BAND_ROWS
+#define BAND_ROWS 0   // 1: a warp per cone row for 2D / 3D wide rows (measured slower, ablation)
+#endif
+  const bool rows_ok = BAND_ROWS && a.active[1] && a.active[2];   // 2D and 3D (not 1D)
   for (int s = 1; s <= a.t; ++s) {
 #pragma unroll
     for (int q = 0; q < 3; ++q) {
       clo[q] = open_lo[q] ? r * s : 0;
       chi[q] = D[q] - (open_hi[q] ? r * s : 0);
     }
+    const int W0 = chi[0] - clo[0], W1 = chi[1] - clo[1], W2 = chi[2] - clo[2];
+    if (rows_ok && W2 >= 16) {
+      // 2D / 3D blocks whose cone rows (axis 2) are >= 16 cells: a warp per cone row, lanes
+      // along the row; the ring test is per row plus a column range, the cell index one add --
+      // the flattened form below spends ~50 integer instructions per FMA on index bookkeeping
+      // (ncu, profiles/r01_s3_band2d_ncu.txt), yet this form measured slower (band 95 -> 114 us
+      // per Heat-2D launch, profiles/r01_s3_ab_band.txt), so it is an ablation only.
+      for (int row = ty; row < W0 * W1; row += ny) {
+        const int k0 = row / W1, k1 = row - k0 * W1;
+        const int i0 = clo[0] + k0, i1 = clo[1] + k1;
+        const bool ring_row = i0 < rlo[0] || i0 >= rhi[0] || i1 < rlo[1] || i1 >= rhi[1];
+        const int c_lo = ring_row ? W2 : max(0, rlo[2] - clo[2]), c_hi = ring_row ? W2 : min(W2, rhi[2] - clo[2]);
+        const int rowbase = (i0 * D[1] + i1) * D[2] + clo[2];
+        for (int k2 = tx; k2 < W2; k2 += 32) {
+          const int e = rowbase + k2;
+          double v;
+          if (k2 < c_lo || k2 >= c_hi) {
+            v = b0[e];                                      // fixed ring
+          } else {
+            v = 0.0;
+#pragma unroll 4
+            for (int k = 0; k < ntaps; ++k) v = fma(s_w[k], b0[e + s_off[k]], v);
+          }
+          b1[e] = v;
+        }
+      }
+      __syncthreads();
+      double* t = b0; b0 = b1; b1 = t;
+      continue;
+    }
     // cone box of this step, flattened over all threads (no idle lanes on narrow faces);
     // the (k0, k1, k2) decomposition is advanced by carries, not recomputed by divisions
-    const int W0 = chi[0] - clo[0], W1 = chi[1] - clo[1], W2 = chi[2] - clo[2];
     const int W12 = W1 * W2, ncone = W0 * W12;
     int k0 = threadIdx.x / W12, k1 = (threadIdx.x - k0 * W12) / W2;
     int k2 = threadIdx.x - k0 * W12 - k1 * W2;
