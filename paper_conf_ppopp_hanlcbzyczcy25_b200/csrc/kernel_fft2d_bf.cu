@@ -34,6 +34,12 @@
 // reads and its next pair's eight TMA boxes (64 x 16, SWIZZLE_128B, OOB -> 0) land while it
 // finishes the inverse and the stores.  The cp.async path (periodic wrap-around, or a pitch TMA
 // cannot describe) loads the same layout synchronously.
+//
+// Compile-time ablations (all 0 by default; each measured slower on B200, DESIGN.md §13,
+// profiles/r01_s3_ab2d.txt): BF_TW_REG (twiddle powers in registers), BF_TW_COMB (combined
+// twiddles), BF_WARP_LOCAL (warp-local row passes), BF_TMEM_S (S_T in tensor memory),
+// BF_PINGPONG (the two groups alternate memory and compute phases), BF_CPLX (interleaved
+// complex words after P1).  Build one with FFTSTENCIL_NVCC_DEFS="-DBF_...=1".
 #include "fft_radix.cuh"
 #include "kernels.cuh"
 #include "tma.cuh"
