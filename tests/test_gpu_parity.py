@@ -534,3 +534,65 @@ def test_small1d_in_place_and_zero_steps(fs):
     p.run(a, b, 0)
     torch.cuda.synchronize()
     assert torch.equal(a, b)
+
+
+# ---------------------------------------------------------------- beyond 2^31 cells (int32 indices)
+def _window_ref(u_dev, w, r, steps, cell, ext):
+    """Oracle value at `cell` from the dependency cone only: the sub-box of radius
+    r*steps + 2r around it (clipped to the grid, whose faces keep the true fixed ring); a
+    window face inside the grid is treated as fixed by the oracle, and its error front moves r
+    cells per step, so it stops 2r cells short of `cell`."""
+    R = r * steps + 2 * r
+    lo = [max(0, c - R) for c in cell]
+    hi = [min(e, c + R + 1) for c, e in zip(cell, ext)]
+    sl = tuple(slice(a, b) for a, b in zip(lo, hi))
+    sub = u_dev[sl].cpu().numpy()
+    loc = np.array([[c - a for c, a in zip(cell, lo)]], dtype=np.int64)
+    # a window face that is not a grid face must not be the oracle's ring at distance < R
+    return float(oracle.stencil_point(sub, w, r, steps, loc)[0])
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("ext,shape,r", [((2 ** 31 - 4103,), "star", 1), ((2 ** 31 - 6400,), "star", 1),
+                                         ((46341, 46341), "star", 1), ((46400, 46400), "box", 1),
+                                         ((1296, 1296, 1296), "star", 1),
+                                         ((1291, 1291, 1291), "box", 1)])
+def test_beyond_int32_cells_sampled(fs, ext, shape, r):
+    """The maximum-size edge case: 1D at the per-axis limit (extents < 2^31; unaligned ->
+    cp.async loads, 64-aligned -> TMA), 2D and 3D grids of more than 2^31 cells (every cell
+    offset needs 64 bits; odd row pitch -> cp.async, 16-byte pitch -> TMA); automatic T, two or more passes plus a remainder, sampled against the
+    oracle on the cells' dependency cones (interior, flat offset 2^31, band, ring)."""
+    w = wl.seeded_weights(shape, len(ext), r)
+    g = torch.Generator(device="cuda")
+    g.manual_seed(2 ** 31 + len(ext))
+    u = torch.rand(ext, dtype=torch.float64, device="cuda", generator=g)
+    p = fs.Plan(ext, w, r, 0)
+    T = p.info()["T"]
+    steps = 2 * T + 3 if len(ext) > 1 else T + 5
+    out = torch.empty_like(u)
+    p.run(u, out, steps)
+    torch.cuda.synchronize()
+    h = p.info()["halo"]
+    total = int(np.prod(ext))
+    flat = [f for f in (2 ** 31 - 1, 2 ** 31, 2 ** 31 + 1, total - 1) if f < total]
+    cells = []
+    for f in flat:   # cells around flat offset 2^31
+        c, idx = int(f), []
+        for e in reversed(ext):
+            idx.append(c % e)
+            c //= e
+        cells.append(tuple(reversed(idx)))
+    rng = np.random.default_rng(7)
+    for _ in range(12):
+        cells.append(tuple(int(rng.integers(0, e)) for e in ext))
+    for d in (0, r - 1, r, h - 1, h, h + 1):
+        cells.append(tuple(min(d, e - 1) for e in ext))
+        cells.append(tuple(max(0, e - 1 - d) for e in ext))
+    scale = float(u.abs().max())
+    for cell in cells:
+        ref = _window_ref(u, w, r, steps, cell, ext)
+        got = float(out[cell].item())
+        assert abs(got - ref) <= TOL * scale, (cell, got, ref, p.info())
+    del u, out
+    p.close()
+    torch.cuda.empty_cache()
