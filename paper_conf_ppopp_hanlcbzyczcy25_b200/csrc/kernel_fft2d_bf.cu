@@ -443,18 +443,20 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
   pp_end(grp, last, br[0][0], bi[0][0], br[3][3], bi[3][3]);
   twiddle4x4<true>(br, bi, tw, rr, cc);
   dft4x4<true>(br, bi);
-  // column predicates once per pass (valid window [h, h + S), grid limit, tile b present)
-  const int64_t ca = g.oa1 + cc, cb = g.ob1 + cc;
+  // column predicates once per pass (valid window [h, h + S), grid limit, tile b present), in
+  // 32-bit arithmetic: every column coordinate and limit is < 2^31 (plan: extents < 2^31)
+  const int ca = (int)g.oa1 + cc, cb = (int)g.ob1 + cc, lim1 = (int)a.bd.lim1;
   bool va[4], vb[4];
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
     const int c = 16 * j + cc;
     const bool in = c >= h && c < h + S;
-    va[j] = in && ca + 16 * j < a.bd.lim1;
-    vb[j] = in && g.has_b && cb + 16 * j < a.bd.lim1;
+    va[j] = in && ca + 16 * j < lim1;
+    vb[j] = in && g.has_b && cb + 16 * j < lim1;
   }
-  const int64_t r_lo = max((int64_t)h, max(a.win.w_lo, (int64_t)0) - g.o0);    // rows [r_lo, r_hi) of the tile
-  const int64_t r_hi = min((int64_t)(h + S), min(a.bd.lim0, a.win.w_hi) - g.o0);
+  // rows [r_lo, r_hi) of the tile (clamped into [h, h + S] before narrowing)
+  const int r_lo = (int)min((int64_t)(h + S), max((int64_t)h, max(a.win.w_lo, (int64_t)0) - g.o0));
+  const int r_hi = (int)max((int64_t)h, min((int64_t)(h + S), min(a.bd.lim0, a.win.w_hi) - g.o0));
   double* dbase = a.dst + (g.o0 - a.win.g0) * a.n1;
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
