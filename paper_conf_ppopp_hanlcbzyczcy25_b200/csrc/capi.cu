@@ -374,6 +374,8 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
   b.gn = hp.g1 - hp.g0;
   b.reference = p->band_reference;
   b.region_cells = hp.band_region_cells;
+  b.ntaps = 0;
+  for (double wv : hp.w) b.ntaps += wv != 0.0;
   cudaStream_t bs = s;
   if (p->band_concurrent) {
     cudaError_t e = cudaEventRecord(p->ev_fork, s);

@@ -15,6 +15,9 @@
 #ifndef BAND_LEAN
 #define BAND_LEAN 1   // 0: per-cell ring test and index recomputation (the session-2 loop)
 #endif
+#ifndef BAND_TAPREG
+#define BAND_TAPREG 1   // 0: taps always read from shared memory (ablation)
+#endif
 
 namespace fstencil {
 namespace {
@@ -96,7 +99,9 @@ constexpr int kMaxTaps = 512;
 // NTH = 256, (256, 6): at most 40 registers (one band CTA fits beside the DMMA engines' fused
 // CTAs); NTH = 1024 for the 1D band, whose two blocks run t (~1000) sequential steps on SMs
 // the fused kernel leaves free (capi.cu), so per-step latency is what counts.
-template <int NTH>
+// NTAPS > 0: the stencil has exactly NTAPS nonzero taps (host-counted); the lean cone loop then
+// keeps offsets and weights in registers, fully unrolled (no shared-memory tap loads, no loop).
+template <int NTH, int NTAPS = 0>
 __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(const BandArgs a) {
   extern __shared__ double sb[];
   __shared__ int s_off[kMaxTaps];
@@ -221,10 +226,23 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
         const int de = e2 + e1 * D[2] + e0 * D12;       // index step per NTH cells, before carries
         const int c2 = D[2] - w3[2], c1 = (D[1] - w3[1]) * D[2];
         int e = (lo3[0] + j0) * D12 + (lo3[1] + j1) * D[2] + lo3[2] + j2;
+        constexpr int NR = NTAPS > 0 ? NTAPS : 1;
+        double wr[NR];
+        int orr[NR];
+#pragma unroll
+        for (int k = 0; k < NR; ++k) {
+          wr[k] = NTAPS > 0 ? s_w[k] : 0.0;
+          orr[k] = NTAPS > 0 ? s_off[k] : 0;
+        }
         for (int f = threadIdx.x; f < nc; f += NTH) {
           double v = 0.0;
+          if (NTAPS > 0) {
+#pragma unroll
+            for (int k = 0; k < NR; ++k) v = fma(wr[k], b0[e + orr[k]], v);
+          } else {
 #pragma unroll 4
-          for (int k = 0; k < ntaps; ++k) v = fma(s_w[k], b0[e + s_off[k]], v);
+            for (int k = 0; k < ntaps; ++k) v = fma(s_w[k], b0[e + s_off[k]], v);
+          }
           b1[e] = v;
           j2 += e2;
           j1 += e1;
@@ -309,6 +327,11 @@ cudaError_t band_configure(size_t smem) {
     return e;
   if ((e = cudaFuncGetAttributes(&fa, band_cone_kernel<256>)) != cudaSuccess) return e;
   const size_t lim1 = (size_t)optin - fa.sharedSizeBytes;
+  if ((e = cudaFuncSetAttribute(band_cone_kernel<256, 5>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
+      cudaSuccess ||
+      (e = cudaFuncSetAttribute(band_cone_kernel<256, 7>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
+      cudaSuccess)
+    return e;
   if ((e = cudaFuncSetAttribute(band_cone_kernel<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
       cudaSuccess)
     return e;
@@ -334,7 +357,13 @@ cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s) {
   else if (taps <= kMaxTaps && !a.reference && one_d)
     band_cone_kernel<64><<<a.nblocks, 64, smem, s>>>(a);
   else if (taps <= kMaxTaps && !a.reference)
-    band_cone_kernel<256><<<a.nblocks, kBandThreads, smem, s>>>(a);
+    // register-resident taps for 5- and 7-point stars (9 taps spill at the 40-register budget
+    // and measured 0.4% slower, profiles/r01_s3_ab_band_tapreg.txt)
+    switch (BAND_LEAN && BAND_TAPREG ? a.ntaps : 0) {
+      case 5: band_cone_kernel<256, 5><<<a.nblocks, kBandThreads, smem, s>>>(a); break;
+      case 7: band_cone_kernel<256, 7><<<a.nblocks, kBandThreads, smem, s>>>(a); break;
+      default: band_cone_kernel<256><<<a.nblocks, kBandThreads, smem, s>>>(a);
+    }
   else
     band_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
   return cudaGetLastError();

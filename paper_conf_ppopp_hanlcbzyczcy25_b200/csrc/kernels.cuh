@@ -104,6 +104,7 @@ struct BandArgs {
   int64_t g0, gn;        // buffers hold global outer-axis rows [g0, g0 + gn)
   int reference;         // 1: the first (unoptimised) band kernel, for ablation/tests
   int region_cells;      // host hint: largest block region (cells) at t = T -- sizes the 1D CTA
+  int ntaps;             // host hint: nonzero weights (selects a register-tap specialisation)
 };
 
 // Copy a box (embedded coordinates) from src to dst0 and dst1 (either may be null).
