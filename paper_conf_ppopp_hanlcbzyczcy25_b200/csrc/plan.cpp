@@ -603,8 +603,13 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   // Split each band box into CTA blocks whose input region (block + r*T on every
   // active side) fits the band kernel's shared-memory budget (2 buffers of FP64).
   // 24 KB of FP64 pairs: small enough to co-reside with three 64 KB fused CTAs per SM (the
-  // band runs concurrently on its own stream, capi.cu)
-  const int budget_cells = 1536;
+  // band runs concurrently on its own stream, capi.cu).  The 2D ALU engine fills the register
+  // file, so its band never co-resides and runs between fused launches: blocks of 2240 cells
+  // per buffer (still 6 CTAs per SM, bound by registers) recompute less halo per band cell and
+  // fit the 10240^2 band into about one wave (Heat-2D +1.5%; 3D measured best at 1536,
+  // profiles/r01_s3_ab_band_budget.txt).  FFTSTENCIL_BAND_BUDGET overrides (cells per buffer).
+  int budget_cells = p.engine == 1 && p.ndim == 2 ? 2240 : 1536;
+  if (const char* v = std::getenv("FFTSTENCIL_BAND_BUDGET")) budget_cells = std::max(256, std::atoi(v));
   const int grow = 2 * r * p.T;
   for (const Box& b : p.band_boxes) {
     int64_t len[3], blk[3];
