@@ -391,7 +391,10 @@ def main():
         # whole job: every rank copies its slab in and its slab out each step
         e2e = {"value": gstencils(cells, steps_per_run * k_e, e_ms), "unit": "GStencils/s",
                "h2d_bytes_per_step": world * int(u0.nbytes), "d2h_bytes_per_step": world * int(u0.nbytes),
-               "steps": k_e, "ms_per_step": e_ms / k_e, "api": "fftstencil_run_host (pinned host buffers)"}
+               "steps": k_e, "ms_per_step": e_ms / k_e, "api": "fftstencil_run_host (pinned host buffers)",
+               "overlap": None if u0.ndim < 2 or world > 1 else ("copies overlapped with row-skewed passes: "
+                           f"K={os.environ.get('FFTSTENCIL_E2E_PIPE', '6')} row chunks, "
+                           f"Q={os.environ.get('FFTSTENCIL_E2E_DEPTH', '16')} skewed passes (DESIGN.md §6)")}
         if not np.isfinite(h_out.numpy()).all():
             raise RuntimeError("non-finite output")
 

@@ -135,7 +135,14 @@ int fftstencil_run_emit(fftstencil_plan* plan, const double* in, const int64_t* 
 
 /* End-to-end variant with HOST buffers: copies h_in (prod(extents) FP64, pageable or
  * pinned) to device, runs, copies the result to h_out, and synchronises `stream`
- * before returning.  Uses two device grids owned by the plan (allocated on first use). */
+ * before returning.  Uses two device grids owned by the plan (allocated on first use).
+ * Single-GPU 2D/3D fixed-boundary plans with >= 2K outer tile rows overlap the copies with
+ * the passes (DESIGN.md §6 "pipelined run_host"): the input arrives in K outer-row chunks
+ * while the first Q passes advance row-skewed behind it, and the last Q passes finish the
+ * result chunk by chunk while earlier chunks are copied out; results are bitwise equal to
+ * fftstencil_run.  The copies run on a plan-owned stream ordered after / before `stream`.
+ * Environment: FFTSTENCIL_E2E_PIPE=K (default 6, 0 = plain copy-run-copy),
+ * FFTSTENCIL_E2E_DEPTH=Q (default 16), FFTSTENCIL_E2E_BAND_SMS (SMs left to the band, 8). */
 int fftstencil_run_host(fftstencil_plan* plan, const double* h_in, double* h_out,
                         int64_t total_steps, void* stream);
 

@@ -14,6 +14,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <cstdint>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -84,6 +85,14 @@ struct fftstencil_plan {
   cudaStream_t band_stream = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_band = nullptr;
   bool band_pending = false;
+  int64_t band_clip_lo = 0, band_clip_hi = INT64_MAX;   // outer rows the band pass produces
+  // ---- pipelined run_host: chunked H2D / D2H on their own stream (FFTSTENCIL_E2E_PIPE) ----
+  cudaStream_t copy_stream = nullptr;
+  cudaStream_t pipe_stream = nullptr;   // greatest priority: fused CTAs dispatch before the band's
+  std::vector<cudaEvent_t> ev_copy;
+  std::vector<int64_t> blk_lo;   // outer-axis start of each band block (blocks sorted by it)
+  int64_t blk_hmax = 0;          // tallest band block along the outer axis
+  int grid_cap = 0;              // > 0: fused launches use at most this many CTAs
   double* dE[2] = {nullptr, nullptr};   // slab + halo buffers, rows [g0, g1)
   int ecur = 0;               // index of the buffer holding the current state
   // ---- profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run() ----
@@ -144,6 +153,9 @@ void free_plan(fftstencil_plan* p) {
   if (p->ev_ready) cudaEventDestroy(p->ev_ready);
   if (p->ev_xchg) cudaEventDestroy(p->ev_xchg);
   if (p->band_stream) cudaStreamDestroy(p->band_stream);
+  if (p->copy_stream) cudaStreamDestroy(p->copy_stream);
+  if (p->pipe_stream) cudaStreamDestroy(p->pipe_stream);
+  for (cudaEvent_t ev : p->ev_copy) cudaEventDestroy(ev);
   if (p->ev_fork) cudaEventDestroy(p->ev_fork);
   if (p->ev_band) cudaEventDestroy(p->ev_band);
   for (cudaEvent_t ev : p->ev_pool) cudaEventDestroy(ev);
@@ -232,6 +244,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
   win.p_begin = pb;
   win.p_end = pe;
   const int64_t np = pe - pb;
+  const int64_t fg = p->grid_cap > 0 ? std::min(p->grid_cap, p->fused_grid) : p->fused_grid;
   Bound bd;
   bd.wrap = hp.periodic;
   bd.shift = hp.periodic ? -hp.h : 0;
@@ -262,7 +275,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     if (hp.algo == 2) {
       // unfused ablation: forward -> HBM spectrum, multiply in HBM, inverse (3 launches)
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
-      const int grid = (int)std::min<int64_t>(p->fused_grid, np);
+      const int grid = (int)std::min<int64_t>(fg, np);
       e = launch_unfused2d(hp.L[0], 1, a, grid, s);
       if (e == cudaSuccess) e = launch_spec_mul(p->dSpec, hp.pairs, hp.L[0], Sre, Sim, s);
       if (e == cudaSuccess) e = launch_unfused2d(hp.L[0], 2, a, grid, s);
@@ -275,12 +288,12 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
       const bool bf = hp.engine == 1;
       const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 2, dims, bf ? box_bf : box, bf);
       if (bf)
-        e = launch_fused2d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+        e = launch_fused2d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
       else
-        e = launch_fused2d_ct(p->ct_cfg, a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+        e = launch_fused2d_ct(p->ct_cfg, a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
-      e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(p->fused_grid, np), s);
+      e = launch_fused2d(hp.L[0], p->variant, a, (int)std::min<int64_t>(fg, np), s);
     }
   } else if (hp.ndim == 1) {
     Fft1dArgs a;
@@ -308,12 +321,12 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
       const uint64_t dims[2] = {64, (uint64_t)(gn / 64)};
       const uint32_t box[2] = {16, 64};
       const bool use_tma = p->use_tma && aligned && encode_tensor_map(&tm, src, 2, dims, box, true);
-      e = launch_fused1d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+      e = launch_fused1d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
     } else if (hp.algo == 1) {
-      e = launch_fused1d_ct(a, (int)std::min<int64_t>(p->fused_grid, np), s);
+      e = launch_fused1d_ct(a, (int)std::min<int64_t>(fg, np), s);
     } else {
       const int64_t blocks = (np + kFft1dWarpsPerBlock - 1) / kFft1dWarpsPerBlock;
-      e = launch_fused1d(a, (int)std::max<int64_t>(1, std::min<int64_t>(p->fused_grid, blocks)), s);
+      e = launch_fused1d(a, (int)std::max<int64_t>(1, std::min<int64_t>(fg, blocks)), s);
     }
   } else {
     Fft3dArgs a;
@@ -339,12 +352,12 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
       const uint32_t box[3] = {16, 16, 16};
       const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 3, dims, box, hp.engine == 1);
       if (hp.engine == 1)
-        e = launch_fused3d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+        e = launch_fused3d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
       else
-        e = launch_fused3d_ct(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(p->fused_grid, np), s);
+        e = launch_fused3d_ct(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
     } else {
       a.Fim = p->dF + (size_t)hp.L[0] * hp.L[0];
-      e = launch_fused3d(a, (int)std::min<int64_t>(p->fused_grid, np), s);
+      e = launch_fused3d(a, (int)std::min<int64_t>(fg, np), s);
     }
   }
   prof_end(p, pe_, s);
@@ -356,9 +369,15 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
 // The band pass of one fused pass.  Concurrent mode: forked from `s` (after everything
 // already enqueued there, i.e. after the pass that produced `src`) onto the band stream;
 // band_join() makes `s` wait for it before the next pass touches either buffer.
-int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s) {
+int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s,
+                     bool forked = false) {
   const HostPlan& hp = p->hp;
-  const int nb = (int)(hp.band_blocks.size() / 8);
+  int64_t i0 = 0, i1 = (int64_t)(hp.band_blocks.size() / 8);
+  if (p->band_clip_lo > 0 || p->band_clip_hi < INT64_MAX) {   // blocks meeting the clip rows
+    i0 = std::upper_bound(p->blk_lo.begin(), p->blk_lo.end(), p->band_clip_lo - p->blk_hmax) - p->blk_lo.begin();
+    i1 = std::lower_bound(p->blk_lo.begin(), p->blk_lo.end(), p->band_clip_hi) - p->blk_lo.begin();
+  }
+  const int nb = (int)std::max<int64_t>(0, i1 - i0);
   if (nb == 0) return FFTSTENCIL_OK;
   BandArgs b;
   b.src = src;
@@ -367,7 +386,7 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
   b.r = hp.radius;
   b.t = t;
   b.w = p->dW;
-  b.blocks = p->dBlocks;
+  b.blocks = p->dBlocks + 8 * i0;
   b.nblocks = nb;
   b.oax = 3 - hp.ndim;
   b.g0 = hp.g0;
@@ -376,13 +395,15 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
   b.region_cells = hp.band_region_cells;
   b.ntaps = 0;
   for (double wv : hp.w) b.ntaps += wv != 0.0;
+  b.clip_lo = p->band_clip_lo;
+  b.clip_hi = p->band_clip_hi;
   cudaStream_t bs = s;
-  if (p->band_concurrent) {
+  if (p->band_concurrent && !forked) {
     cudaError_t e = cudaEventRecord(p->ev_fork, s);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(p->band_stream, p->ev_fork, 0);
     if (e != cudaSuccess) return cuda_fail(e, "band fork");
-    bs = p->band_stream;
   }
+  if (p->band_concurrent) bs = p->band_stream;
   const long pb = prof_begin(p, 1, bs);
   cudaError_t e = launch_band(b, p->band_smem, bs);
   prof_end(p, pb, bs);
@@ -620,10 +641,28 @@ int setup_device(fftstencil_plan* p) {
   p->row_cells = 1;
   for (int a = 1; a < hp.ndim; ++a) p->row_cells *= (size_t)hp.ext[a];
   p->grid_cells = p->row_cells * (size_t)(hp.row_hi - hp.row_lo);
+  // band blocks sorted by their outer-axis start (blocks are independent), so a row range of
+  // the pipelined run_host maps to one contiguous index range
+  std::vector<int32_t> blocks(hp.band_blocks);
+  {
+    const int oax = 3 - hp.ndim;
+    const size_t nb = blocks.size() / 8;
+    std::vector<size_t> order(nb);
+    for (size_t i = 0; i < nb; ++i) order[i] = i;
+    std::stable_sort(order.begin(), order.end(), [&](size_t x, size_t y) {
+      return hp.band_blocks[8 * x + oax] < hp.band_blocks[8 * y + oax];
+    });
+    p->blk_lo.resize(nb);
+    for (size_t i = 0; i < nb; ++i) {
+      for (int q = 0; q < 8; ++q) blocks[8 * i + q] = hp.band_blocks[8 * order[i] + q];
+      p->blk_lo[i] = blocks[8 * i + oax];
+      p->blk_hmax = std::max<int64_t>(p->blk_hmax, blocks[8 * i + 3 + oax] - blocks[8 * i + oax]);
+    }
+  }
   if ((e = upload(&p->dF, F.data(), F.size(), acc)) != cudaSuccess ||
       (e = upload(&p->dS, Sv.data(), Sv.size(), acc)) != cudaSuccess ||
       (e = upload(&p->dW, hp.w.data(), hp.w.size(), acc)) != cudaSuccess ||
-      (e = upload(&p->dBlocks, hp.band_blocks.data(), hp.band_blocks.size(), acc)) != cudaSuccess ||
+      (e = upload(&p->dBlocks, blocks.data(), blocks.size(), acc)) != cudaSuccess ||
       (hp.ndim == 1 && (e = upload(&p->dCrt, hp.crt.data(), hp.crt.size(), acc)) != cudaSuccess))
     return cuda_fail(e, "device upload");
   if (!p->dist) {
@@ -1031,6 +1070,169 @@ int fftstencil_run_emit(fftstencil_plan* p, const double* in, const int64_t* emi
   return FFTSTENCIL_OK;
 }
 
+// ---------------------------------------------------------------- pipelined run_host
+// The host->device copy of the input and the device->host copy of the result take ~30% of a
+// Heat-2D run_host call (2 x 839 MB over PCIe).  They overlap the passes here by
+// skewing the passes over outer tile rows ("units", the Eq. 3 tiles of one outer index):
+// pass k may produce unit u once pass k-1 holds units u-1..u+1 (a unit reads rows
+// [uS, uS+L) = its own output rows +- h, and h <= S), which is also the ping-pong
+// anti-dependency (pass k+1 overwrites pass k-1's buffer only where pass k is done with it).
+// Keeping f[k] (units of pass k produced, from the top) <= f[k-1] - 1 therefore makes any issue
+// order on one stream correct.  Head: the input arrives in K row chunks; after each chunk the
+// first Q passes advance.  Tail: the last Q passes advance in K steps whose pass-P frontier
+// reaches chunk j's last unit, and chunk j of the result is copied out while the next advances.
+// Band (boundary-strip) cells go with the unit whose row range R(u) holds them, the fixed
+// ring with the input chunk.  Same kernels, same per-cell arithmetic: bitwise equal to
+// fftstencil_run (tests/test_gpu_e2e_pipe.py).
+static int copy_ring_rows(fftstencil_plan* p, const double* src, double* d0, double* d1, int64_t y0, int64_t y1,
+                          cudaStream_t s) {
+  const int oax = 3 - p->hp.ndim;
+  for (const Box& b : p->hp.ring_boxes) {
+    BoxCopyArgs a;
+    a.src = src;
+    a.dst0 = d0;
+    a.dst1 = d1;
+    for (int q = 0; q < 3; ++q) { a.n[q] = p->hp.n[q]; a.lo[q] = b.lo[q]; a.hi[q] = b.hi[q]; }
+    a.lo[oax] = std::max<int64_t>(a.lo[oax], y0);
+    a.hi[oax] = std::min<int64_t>(a.hi[oax], y1);
+    if (a.hi[oax] <= a.lo[oax]) continue;
+    a.oax = oax;
+    a.src_off = 0;
+    a.dst_off = 0;
+    cudaError_t e = launch_box_copy(a, s);
+    if (e != cudaSuccess) return cuda_fail(e, "ring copy launch");
+    ++p->last_launches;
+  }
+  return FFTSTENCIL_OK;
+}
+
+static int env_int(const char* name, int dflt) {
+  const char* v = std::getenv(name);
+  return v && *v ? std::atoi(v) : dflt;
+}
+
+// 0: not eligible (the caller runs H2D, fftstencil_run, D2H back to back).
+static int pipe_chunks(const fftstencil_plan* p, int64_t total_steps) {
+  const HostPlan& hp = p->hp;
+  const int K = env_int("FFTSTENCIL_E2E_PIPE", 6);   // 0 disables; else the number of row chunks
+  if (K < 2 || p->dist || p->small1d || hp.ndim < 2 || hp.periodic || hp.algo == 2 || total_steps <= 0) return 0;
+  if (hp.h > hp.S[0] || hp.pair_lo != 0 || hp.pair_hi != hp.pairs || hp.nt[0] < 2 * (int64_t)K) return 0;
+  return K;
+}
+
+static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_out, int64_t total_steps, int K,
+                              cudaStream_t caller) {
+  const HostPlan& hp = p->hp;
+  const int64_t U = hp.nt[0], n0 = hp.ext[0], S = hp.S[0], h = hp.h, ppu = hp.pairs_per_unit;
+  const size_t rcells = p->row_cells;
+  const int Q = std::max(1, env_int("FFTSTENCIL_E2E_DEPTH", 16));
+  const int T = hp.T;
+  const int64_t nfull = total_steps / T;
+  const int rem = (int)(total_steps % T);
+  const int64_t P = nfull + (rem ? 1 : 0);
+  double* in = p->dHostIn;
+  double* out = p->dHostOut;
+  double* dsts[2] = {(P % 2) ? out : p->dScratch, (P % 2) ? p->dScratch : out};
+  auto row_of = [&](int64_t u) -> int64_t { return u <= 0 ? 0 : u >= U ? n0 : u * S + h; };
+  cudaError_t e = cudaSuccess;
+  if (!p->copy_stream && (e = cudaStreamCreateWithFlags(&p->copy_stream, cudaStreamNonBlocking)) != cudaSuccess)
+    return cuda_fail(e, "copy stream");
+  // The schedule runs on an internal greatest-priority stream: when an item's fused kernel and
+  // its band kernel (band stream, default priority) are both pending, the block scheduler places
+  // the fused CTAs first, so they take all but the reserved SMs and the band lands on those
+  // (placed first, the band's CTAs spread one per SM and hold back as many fused CTAs for their
+  // whole ~45 us latency: measured ~40 us per item).  FFTSTENCIL_E2E_PRIO=0 uses the caller's.
+  cudaStream_t s = caller;
+  if (env_int("FFTSTENCIL_E2E_PRIO", 1)) {
+    if (!p->pipe_stream) {
+      int least = 0, greatest = 0;
+      cudaDeviceGetStreamPriorityRange(&least, &greatest);
+      if ((e = cudaStreamCreateWithPriority(&p->pipe_stream, cudaStreamNonBlocking, greatest)) != cudaSuccess)
+        return cuda_fail(e, "pipeline stream");
+    }
+    s = p->pipe_stream;
+  }
+  while (p->ev_copy.size() < (size_t)(2 * K + 4)) {
+    cudaEvent_t ev;
+    if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) return cuda_fail(e, "copy event");
+    p->ev_copy.push_back(ev);
+  }
+  size_t evi = 0;
+  // s -> copy stream (the staging buffers are free once earlier work on s is done), and back
+  auto hand = [&](cudaStream_t from, cudaStream_t to) -> cudaError_t {
+    cudaEvent_t ev = p->ev_copy[evi++];
+    cudaError_t r = cudaEventRecord(ev, from);
+    return r == cudaSuccess ? cudaStreamWaitEvent(to, ev, 0) : r;
+  };
+  const int occ = std::max(1, p->fused_grid / std::max(1, p->sm_count));
+  const int reserve = std::max(0, env_int("FFTSTENCIL_E2E_BAND_SMS", 8));
+  const int grid_cap = std::max(1, p->fused_grid - reserve * occ);
+  std::vector<int64_t> f((size_t)P + 1, 0);
+  auto item = [&](int64_t k, int64_t a, int64_t b) -> int {
+    const int t = k <= nfull ? T : rem;
+    const double* src = k == 1 ? in : dsts[(k - 2) % 2];
+    double* dst = dsts[(k - 1) % 2];
+    // fork the band first (it needs only what `s` holds so far), launch the fused tiles on all
+    // but `reserve` SMs, then the band: its latency-bound CTAs (t sequential steps) run beside
+    // the fused CTAs on the reserved SMs instead of after them
+    if (p->band_concurrent) {
+      cudaError_t e2 = cudaEventRecord(p->ev_fork, s);
+      if (e2 == cudaSuccess) e2 = cudaStreamWaitEvent(p->band_stream, p->ev_fork, 0);
+      if (e2 != cudaSuccess) return cuda_fail(e2, "band fork");
+    }
+    p->grid_cap = p->band_concurrent && b - a < U ? grid_cap : 0;   // whole passes: every SM
+    int rc = launch_fused(p, src, dst, t, a * ppu, b * ppu, s);
+    p->grid_cap = 0;
+    if (rc) return rc;
+    p->band_clip_lo = row_of(a);
+    p->band_clip_hi = row_of(b);
+    rc = launch_band_pass(p, src, dst, t, s, p->band_concurrent);
+    p->band_clip_lo = 0;
+    p->band_clip_hi = INT64_MAX;
+    if (rc) return rc;
+    return band_join(p, s);
+  };
+  auto propagate = [&](auto cap) -> int {
+    for (int64_t k = 1; k <= P; ++k) {
+      int64_t want = f[k - 1] >= U ? U : std::max<int64_t>(0, f[k - 1] - 1);
+      want = std::min<int64_t>(want, cap(k));
+      if (want > f[k]) {
+        if (int rc = item(k, f[k], want)) return rc;
+        f[k] = want;
+      }
+    }
+    return FFTSTENCIL_OK;
+  };
+  if (s != caller && (e = hand(caller, s)) != cudaSuccess) return cuda_fail(e, "pipeline fork");
+  if ((e = hand(s, p->copy_stream)) != cudaSuccess) return cuda_fail(e, "copy fork");
+  int rc = FFTSTENCIL_OK;
+  // head: input chunk c (units [U(c-1)/K, Uc/K)) -> ring rows -> the first Q passes advance
+  for (int c = 1; c <= K; ++c) {
+    const int64_t y0 = row_of(U * (c - 1) / K), y1 = row_of(U * c / K);
+    const size_t off = (size_t)y0 * rcells, bytes = (size_t)(y1 - y0) * rcells * sizeof(double);
+    if ((e = cudaMemcpyAsync(in + off, h_in + off, bytes, cudaMemcpyHostToDevice, p->copy_stream)) != cudaSuccess)
+      return cuda_fail(e, "H2D chunk");
+    if ((e = hand(p->copy_stream, s)) != cudaSuccess) return cuda_fail(e, "H2D join");
+    if ((rc = copy_ring_rows(p, in, out, P > 1 ? p->dScratch : nullptr, y0, y1, s))) return rc;
+    f[0] = U * c / K;
+    if ((rc = propagate([&](int64_t k) { return k <= Q ? U : (int64_t)0; }))) return rc;
+  }
+  // tail: chunk j of the result is final once pass P holds units [0, Uj/K)
+  for (int j = 1; j <= K; ++j) {
+    const int64_t bj = U * j / K;
+    if ((rc = propagate([&](int64_t k) { return k <= P - Q ? U : std::min<int64_t>(U, bj + (P - k)); }))) return rc;
+    if (f[P] < bj) { set_error("pipelined run_host: schedule did not reach the chunk"); return FFTSTENCIL_EINVAL; }
+    const int64_t y0 = row_of(U * (j - 1) / K), y1 = row_of(bj);
+    const size_t off = (size_t)y0 * rcells, bytes = (size_t)(y1 - y0) * rcells * sizeof(double);
+    if ((e = hand(s, p->copy_stream)) != cudaSuccess) return cuda_fail(e, "D2H fork");
+    if ((e = cudaMemcpyAsync(h_out + off, out + off, bytes, cudaMemcpyDeviceToHost, p->copy_stream)) != cudaSuccess)
+      return cuda_fail(e, "D2H chunk");
+  }
+  if ((e = hand(p->copy_stream, s)) != cudaSuccess) return cuda_fail(e, "D2H join");
+  if (s != caller && (e = hand(s, caller)) != cudaSuccess) return cuda_fail(e, "pipeline join");
+  return FFTSTENCIL_OK;
+}
+
 int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, int64_t total_steps, void* stream) {
   if (!p || !h_in || !h_out) { set_error("plan, h_in and h_out must be non-NULL"); return FFTSTENCIL_EINVAL; }
   cudaStream_t s = (cudaStream_t)stream;
@@ -1048,7 +1250,13 @@ int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, i
     p->device_bytes += 2 * bytes;
   }
   int rc = FFTSTENCIL_OK;
-  if ((e = cudaMemcpyAsync(p->dHostIn, h_in, bytes, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
+  const int K = pipe_chunks(p, total_steps);
+  if (K) {
+    p->last_launches = 0;
+    if ((rc = run_host_pipelined(p, h_in, h_out, total_steps, K, (cudaStream_t)stream)) == FFTSTENCIL_OK &&
+        (e = cudaStreamSynchronize(s)) != cudaSuccess)
+      rc = cuda_fail(e, "stream synchronize");
+  } else if ((e = cudaMemcpyAsync(p->dHostIn, h_in, bytes, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
     rc = cuda_fail(e, "H2D copy");
   } else if ((rc = fftstencil_run(p, p->dHostIn, p->dHostOut, total_steps, stream)) == FFTSTENCIL_OK) {
     if ((e = cudaMemcpyAsync(h_out, p->dHostOut, bytes, cudaMemcpyDeviceToHost, s)) != cudaSuccess)

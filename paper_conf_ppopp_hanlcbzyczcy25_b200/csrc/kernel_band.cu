@@ -31,12 +31,14 @@ __global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
   for (int q = 0; q < 3; ++q) {
     lo[q] = blk[q];
     hi[q] = blk[3 + q];
+    if (q == a.oax) { lo[q] = max(lo[q], a.clip_lo); hi[q] = min(hi[q], a.clip_hi); }
     const int64_t gq = a.active[q] ? (int64_t)a.r * a.t : 0;
     int64_t l = max((int64_t)0, lo[q] - gq), u = min(a.n[q], hi[q] + gq);
     if (q == a.oax) { l = max(l, a.g0); u = min(u, a.g0 + a.gn); }
     rl[q] = l;
     D[q] = u - l;
   }
+  if (hi[a.oax] <= lo[a.oax]) return;   // block outside the clip rows (whole CTA)
   const int64_t vol = D[0] * D[1] * D[2];
   double* b0 = sb;
   double* b1 = sb + vol;
@@ -116,6 +118,7 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
   for (int q = 0; q < 3; ++q) {
     lo[q] = blk[q];
     hi[q] = blk[3 + q];
+    if (q == a.oax) { lo[q] = max(lo[q], a.clip_lo); hi[q] = min(hi[q], a.clip_hi); }
     const int64_t gq = a.active[q] ? (int64_t)a.r * a.t : 0;
     int64_t l = max((int64_t)0, lo[q] - gq), u = min(a.n[q], hi[q] + gq);
     if (q == a.oax) { l = max(l, a.g0); u = min(u, a.g0 + a.gn); }
@@ -124,6 +127,7 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
     open_lo[q] = a.active[q] && l > 0;               // cells below were not loaded
     open_hi[q] = a.active[q] && u < a.n[q];
   }
+  if (hi[a.oax] <= lo[a.oax]) return;   // block outside the clip rows (whole CTA)
   const int r = a.r, wd = 2 * r + 1;
   if (threadIdx.x == 0) {
     int n = 0;

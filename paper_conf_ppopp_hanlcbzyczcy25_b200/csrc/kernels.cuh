@@ -105,6 +105,7 @@ struct BandArgs {
   int reference;         // 1: the first (unoptimised) band kernel, for ablation/tests
   int region_cells;      // host hint: largest block region (cells) at t = T -- sizes the 1D CTA
   int ntaps;             // host hint: nonzero weights (selects a register-tap specialisation)
+  int64_t clip_lo, clip_hi;   // only outer-axis rows [clip_lo, clip_hi) are produced (pipelined run_host)
 };
 
 // Copy a box (embedded coordinates) from src to dst0 and dst1 (either may be null).
