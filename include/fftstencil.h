@@ -222,6 +222,22 @@ int fftstencil_describe_ex(int ndim, const int64_t* extents, const double* weigh
 int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* weights, int radius,
                               int T, int which, int axis, int t, double* out, int64_t cap);
 
+/* Host-only: the op list fftstencil_run_host issues for a single-GPU plan of these arguments
+ * with `chunks` = K and `depth` = Q (the FFTSTENCIL_E2E_PIPE / _DEPTH values), for tests of the
+ * schedule.  4 int64 per op, in issue order:
+ *   {0, y0, y1, 0}  copy input rows [y0, y1) host -> device, then the run stream waits for it;
+ *   {1, y0, y1, 0}  copy the fixed ring's rows [y0, y1) into both pass buffers;
+ *   {2, k, u0, u1}  pass k (1-based, t = T, the last pass total_steps mod T if nonzero) on
+ *                   outer tile rows [u0, u1): their fused tile pairs and the band cells in
+ *                   rows [row(u0), row(u1)), row(u) = 0 / u*S + h / n0 for u = 0 / inner / U;
+ *   {3, y0, y1, 0}  copy result rows [y0, y1) device -> host after all earlier ops.
+ * `out` must hold `cap` ops (4*cap int64); returns the number of ops (>= 0; out = NULL
+ * queries it) or FFTSTENCIL_EINVAL when the plan does not take the pipelined path (1D,
+ * h > S, fewer than 2*chunks outer tile rows, chunks < 2, depth < 1, total_steps <= 0). */
+int64_t fftstencil_e2e_schedule(int ndim, const int64_t* extents, const double* weights, int radius,
+                                int T, int64_t total_steps, int chunks, int depth, int64_t* out,
+                                int64_t cap);
+
 #ifdef __cplusplus
 }
 #endif

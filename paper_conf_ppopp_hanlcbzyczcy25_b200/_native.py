@@ -21,7 +21,8 @@ EXPORTS = ("fftstencil_plan_create", "fftstencil_run", "fftstencil_run_host", "f
            "fftstencil_plan_info", "fftstencil_last_error", "fftstencil_describe", "fftstencil_export_aux",
            "fftstencil_set_profiling", "fftstencil_profile_read", "fftstencil_plan_create_dist",
            "fftstencil_nccl_unique_id", "fftstencil_run_group", "fftstencil_describe_dist",
-           "fftstencil_plan_create_ex", "fftstencil_describe_ex", "fftstencil_run_emit")
+           "fftstencil_plan_create_ex", "fftstencil_describe_ex", "fftstencil_run_emit",
+           "fftstencil_e2e_schedule")
 
 
 class Info(ctypes.Structure):
@@ -110,6 +111,9 @@ def lib():
     L.fftstencil_export_aux.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                         ctypes.c_int, ctypes.c_int, dp, ctypes.c_int64]
     L.fftstencil_export_aux.restype = ctypes.c_int64
+    L.fftstencil_e2e_schedule.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int64,
+                                          ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64]
+    L.fftstencil_e2e_schedule.restype = ctypes.c_int64
     L.fftstencil_set_profiling.argtypes = [vp, ctypes.c_int]
     L.fftstencil_set_profiling.restype = ctypes.c_int
     L.fftstencil_profile_read.argtypes = [vp, dp, i64p, dp, i64p]

@@ -817,6 +817,26 @@ int fftstencil_describe_dist(int ndim, const int64_t* extents, const double* wei
   return FFTSTENCIL_OK;
 }
 
+int64_t fftstencil_e2e_schedule(int ndim, const int64_t* extents, const double* weights, int radius, int T,
+                                int64_t total_steps, int chunks, int depth, int64_t* out, int64_t cap) {
+  HostPlan hp;
+  std::string err;
+  int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, 1, 0, env_algo());
+  if (rc != FFTSTENCIL_OK) { set_error(err); return rc; }
+  std::vector<int64_t> ops;
+  if ((rc = build_e2e_schedule(hp, total_steps, chunks, depth, ops)) != FFTSTENCIL_OK) {
+    set_error("plan not eligible for the pipelined run_host schedule");
+    return rc;
+  }
+  const int64_t n = (int64_t)ops.size() / 4;
+  if (out) {
+    if (cap < n) { set_error("cap smaller than the number of ops"); return FFTSTENCIL_EINVAL; }
+    std::memcpy(out, ops.data(), ops.size() * sizeof(int64_t));
+  }
+  clear_error();
+  return n;
+}
+
 int64_t fftstencil_export_aux(int ndim, const int64_t* extents, const double* weights, int radius, int T,
                               int which, int axis, int t, double* out, int64_t cap) {
   HostPlan hp;
@@ -1111,21 +1131,19 @@ static int env_int(const char* name, int dflt) {
   return v && *v ? std::atoi(v) : dflt;
 }
 
-// 0: not eligible (the caller runs H2D, fftstencil_run, D2H back to back).
-static int pipe_chunks(const fftstencil_plan* p, int64_t total_steps) {
-  const HostPlan& hp = p->hp;
+// K, Q of the pipelined schedule; K = 0: disabled (the caller runs H2D, fftstencil_run, D2H).
+static int pipe_chunks(const fftstencil_plan* p) {
   const int K = env_int("FFTSTENCIL_E2E_PIPE", 6);   // 0 disables; else the number of row chunks
-  if (K < 2 || p->dist || p->small1d || hp.ndim < 2 || hp.periodic || hp.algo == 2 || total_steps <= 0) return 0;
-  if (hp.h > hp.S[0] || hp.pair_lo != 0 || hp.pair_hi != hp.pairs || hp.nt[0] < 2 * (int64_t)K) return 0;
-  return K;
+  return p->dist || p->small1d ? 0 : K;
 }
 
-static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_out, int64_t total_steps, int K,
-                              cudaStream_t caller) {
+static int pipe_depth() { return std::max(1, env_int("FFTSTENCIL_E2E_DEPTH", 16)); }
+
+static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_out,
+                              const std::vector<int64_t>& ops, int64_t total_steps, cudaStream_t caller) {
   const HostPlan& hp = p->hp;
   const int64_t U = hp.nt[0], n0 = hp.ext[0], S = hp.S[0], h = hp.h, ppu = hp.pairs_per_unit;
   const size_t rcells = p->row_cells;
-  const int Q = std::max(1, env_int("FFTSTENCIL_E2E_DEPTH", 16));
   const int T = hp.T;
   const int64_t nfull = total_steps / T;
   const int rem = (int)(total_steps % T);
@@ -1152,13 +1170,14 @@ static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_
     }
     s = p->pipe_stream;
   }
-  while (p->ev_copy.size() < (size_t)(2 * K + 4)) {
+  size_t nev = 4;
+  for (size_t i = 0; i < ops.size(); i += 4) nev += ops[i] == 0 || ops[i] == 3;
+  while (p->ev_copy.size() < nev) {
     cudaEvent_t ev;
     if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) return cuda_fail(e, "copy event");
     p->ev_copy.push_back(ev);
   }
   size_t evi = 0;
-  // s -> copy stream (the staging buffers are free once earlier work on s is done), and back
   auto hand = [&](cudaStream_t from, cudaStream_t to) -> cudaError_t {
     cudaEvent_t ev = p->ev_copy[evi++];
     cudaError_t r = cudaEventRecord(ev, from);
@@ -1167,7 +1186,6 @@ static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_
   const int occ = std::max(1, p->fused_grid / std::max(1, p->sm_count));
   const int reserve = std::max(0, env_int("FFTSTENCIL_E2E_BAND_SMS", 8));
   const int grid_cap = std::max(1, p->fused_grid - reserve * occ);
-  std::vector<int64_t> f((size_t)P + 1, 0);
   auto item = [&](int64_t k, int64_t a, int64_t b) -> int {
     const int t = k <= nfull ? T : rem;
     const double* src = k == 1 ? in : dsts[(k - 2) % 2];
@@ -1192,41 +1210,25 @@ static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_
     if (rc) return rc;
     return band_join(p, s);
   };
-  auto propagate = [&](auto cap) -> int {
-    for (int64_t k = 1; k <= P; ++k) {
-      int64_t want = f[k - 1] >= U ? U : std::max<int64_t>(0, f[k - 1] - 1);
-      want = std::min<int64_t>(want, cap(k));
-      if (want > f[k]) {
-        if (int rc = item(k, f[k], want)) return rc;
-        f[k] = want;
-      }
-    }
-    return FFTSTENCIL_OK;
-  };
   if (s != caller && (e = hand(caller, s)) != cudaSuccess) return cuda_fail(e, "pipeline fork");
   if ((e = hand(s, p->copy_stream)) != cudaSuccess) return cuda_fail(e, "copy fork");
   int rc = FFTSTENCIL_OK;
-  // head: input chunk c (units [U(c-1)/K, Uc/K)) -> ring rows -> the first Q passes advance
-  for (int c = 1; c <= K; ++c) {
-    const int64_t y0 = row_of(U * (c - 1) / K), y1 = row_of(U * c / K);
-    const size_t off = (size_t)y0 * rcells, bytes = (size_t)(y1 - y0) * rcells * sizeof(double);
-    if ((e = cudaMemcpyAsync(in + off, h_in + off, bytes, cudaMemcpyHostToDevice, p->copy_stream)) != cudaSuccess)
-      return cuda_fail(e, "H2D chunk");
-    if ((e = hand(p->copy_stream, s)) != cudaSuccess) return cuda_fail(e, "H2D join");
-    if ((rc = copy_ring_rows(p, in, out, P > 1 ? p->dScratch : nullptr, y0, y1, s))) return rc;
-    f[0] = U * c / K;
-    if ((rc = propagate([&](int64_t k) { return k <= Q ? U : (int64_t)0; }))) return rc;
-  }
-  // tail: chunk j of the result is final once pass P holds units [0, Uj/K)
-  for (int j = 1; j <= K; ++j) {
-    const int64_t bj = U * j / K;
-    if ((rc = propagate([&](int64_t k) { return k <= P - Q ? U : std::min<int64_t>(U, bj + (P - k)); }))) return rc;
-    if (f[P] < bj) { set_error("pipelined run_host: schedule did not reach the chunk"); return FFTSTENCIL_EINVAL; }
-    const int64_t y0 = row_of(U * (j - 1) / K), y1 = row_of(bj);
-    const size_t off = (size_t)y0 * rcells, bytes = (size_t)(y1 - y0) * rcells * sizeof(double);
-    if ((e = hand(s, p->copy_stream)) != cudaSuccess) return cuda_fail(e, "D2H fork");
-    if ((e = cudaMemcpyAsync(h_out + off, out + off, bytes, cudaMemcpyDeviceToHost, p->copy_stream)) != cudaSuccess)
-      return cuda_fail(e, "D2H chunk");
+  for (size_t i = 0; i < ops.size(); i += 4) {
+    const int64_t op = ops[i], x = ops[i + 1], y = ops[i + 2], z = ops[i + 3];
+    const size_t off = (size_t)x * rcells, bytes = (size_t)(y - x) * rcells * sizeof(double);
+    if (op == 0) {          // input rows [x, y) -> device; the run stream waits for them
+      if ((e = cudaMemcpyAsync(in + off, h_in + off, bytes, cudaMemcpyHostToDevice, p->copy_stream)) != cudaSuccess)
+        return cuda_fail(e, "H2D chunk");
+      if ((e = hand(p->copy_stream, s)) != cudaSuccess) return cuda_fail(e, "H2D join");
+    } else if (op == 1) {   // fixed ring rows [x, y) into both pass buffers
+      if ((rc = copy_ring_rows(p, in, out, P > 1 ? p->dScratch : nullptr, x, y, s))) return rc;
+    } else if (op == 2) {   // pass x on units [y, z)
+      if ((rc = item(x, y, z))) return rc;
+    } else {                // result rows [x, y) -> host after everything issued so far
+      if ((e = hand(s, p->copy_stream)) != cudaSuccess) return cuda_fail(e, "D2H fork");
+      if ((e = cudaMemcpyAsync(h_out + off, out + off, bytes, cudaMemcpyDeviceToHost, p->copy_stream)) != cudaSuccess)
+        return cuda_fail(e, "D2H chunk");
+    }
   }
   if ((e = hand(p->copy_stream, s)) != cudaSuccess) return cuda_fail(e, "D2H join");
   if (s != caller && (e = hand(s, caller)) != cudaSuccess) return cuda_fail(e, "pipeline join");
@@ -1250,10 +1252,11 @@ int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, i
     p->device_bytes += 2 * bytes;
   }
   int rc = FFTSTENCIL_OK;
-  const int K = pipe_chunks(p, total_steps);
-  if (K) {
+  const int K = pipe_chunks(p);
+  std::vector<int64_t> ops;
+  if (K && build_e2e_schedule(p->hp, total_steps, K, pipe_depth(), ops) == FFTSTENCIL_OK) {
     p->last_launches = 0;
-    if ((rc = run_host_pipelined(p, h_in, h_out, total_steps, K, (cudaStream_t)stream)) == FFTSTENCIL_OK &&
+    if ((rc = run_host_pipelined(p, h_in, h_out, ops, total_steps, (cudaStream_t)stream)) == FFTSTENCIL_OK &&
         (e = cudaStreamSynchronize(s)) != cudaSuccess)
       rc = cuda_fail(e, "stream synchronize");
   } else if ((e = cudaMemcpyAsync(p->dHostIn, h_in, bytes, cudaMemcpyHostToDevice, s)) != cudaSuccess) {

@@ -651,4 +651,52 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   return FFTSTENCIL_OK;
 }
 
+
+// ---- pipelined run_host schedule ----
+// Unit u (outer tile row) of pass k reads pass k-1's rows [uS, uS+L) = its output rows +- h,
+// i.e. units u-1..u+1 when h <= S.  Band and ring cells belong to the unit whose row range
+// R(u) = [row(u), row(u+1)) holds them (row(0) = 0, row(U) = n0), and their dependency cone
+// (+- h rows) stays within units u-1..u+1 too.  Frontiers f[k] (units [0, f[k]) of pass k
+// issued) with f[k] <= f[k-1] - 1 (or f[k-1] = U) satisfy the read dependency and the
+// ping-pong anti-dependency at once, so the ops run in issue order on one stream.
+int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std::vector<int64_t>& ops) {
+  ops.clear();
+  if (K < 2 || Q < 1 || p.ndim < 2 || p.periodic || p.algo == 2 || p.nranks != 1 || total_steps <= 0)
+    return FFTSTENCIL_EINVAL;
+  const int64_t U = p.nt[0], n0 = p.ext[0], S = p.S[0], h = p.h;
+  if (h > S || U < 2 * (int64_t)K || p.pair_lo != 0 || p.pair_hi != p.pairs) return FFTSTENCIL_EINVAL;
+  const int64_t P = total_steps / p.T + (total_steps % p.T ? 1 : 0);
+  auto row_of = [&](int64_t u) -> int64_t { return u <= 0 ? 0 : u >= U ? n0 : u * S + h; };
+  auto push = [&](int64_t op, int64_t x, int64_t y, int64_t z) {
+    ops.push_back(op); ops.push_back(x); ops.push_back(y); ops.push_back(z);
+  };
+  std::vector<int64_t> f((size_t)P + 1, 0);
+  auto propagate = [&](auto cap) {
+    for (int64_t k = 1; k <= P; ++k) {
+      int64_t want = f[k - 1] >= U ? U : std::max<int64_t>(0, f[k - 1] - 1);
+      want = std::min<int64_t>(want, cap(k));
+      if (want > f[k]) {
+        push(2, k, f[k], want);
+        f[k] = want;
+      }
+    }
+  };
+  // head: input chunk c, its ring rows, then the first Q passes advance behind it
+  for (int c = 1; c <= K; ++c) {
+    const int64_t y0 = row_of(U * (c - 1) / K), y1 = row_of(U * c / K);
+    push(0, y0, y1, 0);
+    push(1, y0, y1, 0);
+    f[0] = U * c / K;
+    propagate([&](int64_t k) { return k <= Q ? U : (int64_t)0; });
+  }
+  // tail: the last Q passes advance until pass P holds chunk j, which is then copied out
+  for (int j = 1; j <= K; ++j) {
+    const int64_t bj = U * j / K;
+    propagate([&](int64_t k) { return k <= P - Q ? U : std::min<int64_t>(U, bj + (P - k)); });
+    if (f[(size_t)P] < bj) { ops.clear(); return FFTSTENCIL_EINVAL; }
+    push(3, row_of(U * (j - 1) / K), row_of(bj), 0);
+  }
+  return FFTSTENCIL_OK;
+}
+
 }  // namespace fstencil

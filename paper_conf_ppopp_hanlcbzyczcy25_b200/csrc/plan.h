@@ -96,6 +96,15 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
                     HostPlan& p, std::string& err, int nranks = 1, int rank = 0, int algo = -1,
                     int periodic = 0);
 
+// Pipelined run_host schedule: ops of 4 int64 {op, x, y, z} in issue order.
+//   op 0: copy input rows [x, y) host -> device (then the run stream waits for it);
+//   op 1: copy the fixed ring's rows [x, y) from the input into both pass buffers;
+//   op 2: pass x (1-based) on outer tile rows ("units") [y, z): fused pairs and band rows;
+//   op 3: copy result rows [x, y) device -> host once everything before it is done.
+// Returns 0 with the ops, or FFTSTENCIL_EINVAL when the plan is not eligible (1D, periodic,
+// a slab plan, the unfused ablation, h > S, fewer than 2K units, no steps).
+int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std::vector<int64_t>& ops);
+
 // Dense-DFT tile cost model (executed FP64 tensor flops per cell-step) used to pick L/T.
 double model_flops_2d(int L, int S, int T);
 // Factored (CT 8 x 8, L = 64) tile: executed FP64 flops per cell-step (DMMA + twiddles + S_T).

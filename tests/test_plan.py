@@ -24,7 +24,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def test_library_exports_every_declared_symbol():
     hdr = open(os.path.join(ROOT, "include", "fftstencil.h")).read()
-    declared = set(re.findall(r"\b(fftstencil_[a-z_]+)\s*\(", hdr))
+    declared = set(re.findall(r"\b(fftstencil_[a-z0-9_]+)\s*\(", hdr))
     assert declared == set(_native.EXPORTS)
     lib = _native.lib()
     for name in declared:
