@@ -142,7 +142,7 @@ int fftstencil_run_emit(fftstencil_plan* plan, const double* in, const int64_t* 
  * result chunk by chunk while earlier chunks are copied out; results are bitwise equal to
  * fftstencil_run.  The copies run on a plan-owned stream ordered after / before `stream`.
  * Environment: FFTSTENCIL_E2E_PIPE=K (default 6, 0 = plain copy-run-copy),
- * FFTSTENCIL_E2E_DEPTH=Q (default 16), FFTSTENCIL_E2E_BAND_SMS (SMs left to the band, 8). */
+ * FFTSTENCIL_E2E_DEPTH=Q (default 16), FFTSTENCIL_E2E_BAND_SMS (SMs left to the band, 4). */
 int fftstencil_run_host(fftstencil_plan* plan, const double* h_in, double* h_out,
                         int64_t total_steps, void* stream);
 

@@ -1184,7 +1184,7 @@ static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_
     return r == cudaSuccess ? cudaStreamWaitEvent(to, ev, 0) : r;
   };
   const int occ = std::max(1, p->fused_grid / std::max(1, p->sm_count));
-  const int reserve = std::max(0, env_int("FFTSTENCIL_E2E_BAND_SMS", 8));
+  const int reserve = std::max(0, env_int("FFTSTENCIL_E2E_BAND_SMS", 4));
   const int grid_cap = std::max(1, p->fused_grid - reserve * occ);
   auto item = [&](int64_t k, int64_t a, int64_t b) -> int {
     const int t = k <= nfull ? T : rem;
