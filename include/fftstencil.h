@@ -98,6 +98,9 @@ typedef struct {
                                    on the FP64 ALU (default; FFTSTENCIL_ENGINE=dmma|alu)      */
   double alu_ops_per_pass;      /* engine 1: FP64 ALU instructions one fused launch executes
                                    (adds, multiplies and FMAs, each one)                    */
+  int last_run_pipelined;       /* 1 if the last fftstencil_run_host overlapped its copies with
+                                   row-skewed passes (pipelined schedule), 0 if it ran plain
+                                   copy-run-copy (FFTSTENCIL_E2E_PIPE=0, 1D, small grids, h > S) */
 } fftstencil_info;
 
 /* Plan creation flags (fftstencil_plan_create_ex / fftstencil_describe_ex). */

@@ -29,6 +29,15 @@ def _arrays(extents, weights, radius):
     return ext, w
 
 
+def _current_device():
+    """The CUDA device the C ABI binds a new plan to (the current one); None without torch/CUDA."""
+    try:
+        import torch
+        return torch.cuda.current_device() if torch.cuda.is_available() else None
+    except Exception:
+        return None
+
+
 def _i64p(a):
     return a.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
 
@@ -143,6 +152,7 @@ class Plan:
         if not h:
             raise FftStencilError(_native.EINVAL, last_error())
         self._h = ctypes.c_void_p(h)
+        self.device = _current_device()
         inf = self.info()
         self.extents = (inf["row_end"] - inf["row_begin"],) + self.global_extents[1:]
 
@@ -193,6 +203,8 @@ class Plan:
             raise TypeError(f"{name} must be a CUDA float64 torch tensor")
         if tuple(t.shape) != self.extents or not t.is_contiguous():
             raise ValueError(f"{name} must be contiguous with shape {self.extents}")
+        if self.device is not None and t.device.index != self.device:
+            raise ValueError(f"{name} is on cuda:{t.device.index}, the plan on cuda:{self.device}")
 
     def run(self, inp, out, total_steps: int, stream=None) -> None:
         """Enqueue total_steps time steps: out <- stencil^steps(inp) (asynchronous)."""
@@ -236,7 +248,11 @@ class Plan:
                     raise ValueError(f"{name} must be C-contiguous float64 with shape {self.extents}")
                 return a.ctypes.data
             import torch
-            if isinstance(a, torch.Tensor) and not a.is_cuda and a.dtype == torch.float64 and a.is_contiguous():
+            if isinstance(a, torch.Tensor) and not a.is_cuda and a.dtype == torch.float64:
+                # the C side copies prod(extents) doubles from / into this buffer: a wrong
+                # shape (e.g. a global grid passed to a slab plan) would run out of bounds
+                if tuple(a.shape) != self.extents or not a.is_contiguous():
+                    raise ValueError(f"{name} must be contiguous with shape {self.extents}")
                 return a.data_ptr()
             raise TypeError(f"{name} must be a host float64 array")
         sh = 0

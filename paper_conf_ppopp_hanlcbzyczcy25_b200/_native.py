@@ -58,6 +58,7 @@ class Info(ctypes.Structure):
         ("periodic", ctypes.c_int),
         ("engine", ctypes.c_int),
         ("alu_ops_per_pass", ctypes.c_double),
+        ("last_run_pipelined", ctypes.c_int),
     ]
 
     def as_dict(self) -> dict:
@@ -76,6 +77,7 @@ class Info(ctypes.Structure):
             "algo": ("dense", "factored", "unfused")[self.algo] if nd >= 2 else ("pfa", "factored")[self.algo],
             "periodic": bool(self.periodic),
             "engine": ("dmma", "alu")[self.engine], "alu_ops_per_pass": self.alu_ops_per_pass,
+            "last_run_pipelined": bool(self.last_run_pipelined),
         }
 
 

@@ -72,6 +72,7 @@ struct fftstencil_plan {
   int band_reference = 0;     // FFTSTENCIL_BAND=reference selects the first band kernel
   size_t band_smem = 0;
   int64_t last_launches = 0;
+  bool last_pipelined = false;   // the last run_host took the pipelined schedule
   // ---- decomposition (dist) ----
   bool dist = false;          // slab plan with halo buffers
   bool loopback = false;      // no communicator: run by fftstencil_run_group
@@ -93,6 +94,8 @@ struct fftstencil_plan {
   std::vector<int64_t> blk_lo;   // outer-axis start of each band block (blocks sorted by it)
   int64_t blk_hmax = 0;          // tallest band block along the outer axis
   int grid_cap = 0;              // > 0: fused launches use at most this many CTAs
+  int max_ctas = 0;              // FFTSTENCIL_MAX_CTAS (tests): cap on every fused launch's grid, so each
+                                 // persistent CTA walks many pairs through its refill / mbarrier loop
   double* dE[2] = {nullptr, nullptr};   // slab + halo buffers, rows [g0, g1)
   int ecur = 0;               // index of the buffer holding the current state
   // ---- profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run() ----
@@ -244,7 +247,8 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
   win.p_begin = pb;
   win.p_end = pe;
   const int64_t np = pe - pb;
-  const int64_t fg = p->grid_cap > 0 ? std::min(p->grid_cap, p->fused_grid) : p->fused_grid;
+  int64_t fg = p->grid_cap > 0 ? std::min(p->grid_cap, p->fused_grid) : p->fused_grid;
+  if (p->max_ctas > 0) fg = std::min<int64_t>(fg, p->max_ctas);
   Bound bd;
   bd.wrap = hp.periodic;
   bd.shift = hp.periodic ? -hp.h : 0;
@@ -733,6 +737,7 @@ int setup_device(fftstencil_plan* p) {
   // the register-full ALU kernel (one CTA per SM) would serialise it, so leave it its SMs
   if (hp.ndim == 1 && hp.algo == 1 && hp.engine == 1 && !hp.band_blocks.empty())
     p->fused_grid = (int)std::max<int64_t>(1, p->fused_grid - (int64_t)(hp.band_blocks.size() / 8));
+  if (const char* v = std::getenv("FFTSTENCIL_MAX_CTAS")) p->max_ctas = std::max(0, std::atoi(v));
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
   if (const char* v = std::getenv("FFTSTENCIL_BAND_STREAM")) p->band_concurrent = std::atoi(v) != 0;
   if (hp.band_blocks.empty()) p->band_concurrent = false;
@@ -1139,8 +1144,40 @@ static int pipe_chunks(const fftstencil_plan* p) {
 
 static int pipe_depth() { return std::max(1, env_int("FFTSTENCIL_E2E_DEPTH", 16)); }
 
+static int run_host_pipelined_ops(fftstencil_plan* p, const double* h_in, double* h_out,
+                                  const std::vector<int64_t>& ops, int64_t total_steps, cudaStream_t caller,
+                                  cudaStream_t& s);
+
+// On every exit, error or not, the copy stream and the pipeline stream are joined back into
+// the caller's stream, so the caller's synchronize covers every queued chunk copy: a caller
+// that frees its host buffers after an error cannot race a pending H2D / D2H.
 static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_out,
                               const std::vector<int64_t>& ops, int64_t total_steps, cudaStream_t caller) {
+  cudaStream_t s = caller;
+  const int rc = run_host_pipelined_ops(p, h_in, h_out, ops, total_steps, caller, s);
+  if (rc != FFTSTENCIL_OK) {
+    const std::string err = g_last_error;
+    cudaEvent_t ev;
+    if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess) {
+      for (cudaStream_t x : {p->copy_stream, s, p->band_stream}) {
+        if (!x || x == caller) continue;
+        if (cudaEventRecord(ev, x) == cudaSuccess) cudaStreamWaitEvent(caller, ev, 0);
+      }
+      cudaEventDestroy(ev);
+    }
+    p->band_pending = false;
+    p->grid_cap = 0;
+    p->band_clip_lo = 0;
+    p->band_clip_hi = INT64_MAX;
+    cudaGetLastError();
+    set_error(err);
+  }
+  return rc;
+}
+
+static int run_host_pipelined_ops(fftstencil_plan* p, const double* h_in, double* h_out,
+                                  const std::vector<int64_t>& ops, int64_t total_steps, cudaStream_t caller,
+                                  cudaStream_t& s) {
   const HostPlan& hp = p->hp;
   const int64_t U = hp.nt[0], n0 = hp.ext[0], S = hp.S[0], h = hp.h, ppu = hp.pairs_per_unit;
   const size_t rcells = p->row_cells;
@@ -1160,7 +1197,7 @@ static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_
   // the fused CTAs first, so they take all but the reserved SMs and the band lands on those
   // (placed first, the band's CTAs spread one per SM and hold back as many fused CTAs for their
   // whole ~45 us latency: measured ~40 us per item).  FFTSTENCIL_E2E_PRIO=0 uses the caller's.
-  cudaStream_t s = caller;
+  s = caller;
   if (env_int("FFTSTENCIL_E2E_PRIO", 1)) {
     if (!p->pipe_stream) {
       int least = 0, greatest = 0;
@@ -1254,18 +1291,21 @@ int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, i
   int rc = FFTSTENCIL_OK;
   const int K = pipe_chunks(p);
   std::vector<int64_t> ops;
+  p->last_pipelined = false;
   if (K && build_e2e_schedule(p->hp, total_steps, K, pipe_depth(), ops) == FFTSTENCIL_OK) {
     p->last_launches = 0;
-    if ((rc = run_host_pipelined(p, h_in, h_out, ops, total_steps, (cudaStream_t)stream)) == FFTSTENCIL_OK &&
-        (e = cudaStreamSynchronize(s)) != cudaSuccess)
-      rc = cuda_fail(e, "stream synchronize");
+    p->last_pipelined = true;
+    rc = run_host_pipelined(p, h_in, h_out, ops, total_steps, (cudaStream_t)stream);
+    // synchronise on success and on error (queued chunk copies still read / write the host buffers)
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess && rc == FFTSTENCIL_OK) rc = cuda_fail(e, "stream synchronize");
   } else if ((e = cudaMemcpyAsync(p->dHostIn, h_in, bytes, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
     rc = cuda_fail(e, "H2D copy");
-  } else if ((rc = fftstencil_run(p, p->dHostIn, p->dHostOut, total_steps, stream)) == FFTSTENCIL_OK) {
-    if ((e = cudaMemcpyAsync(h_out, p->dHostOut, bytes, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+  } else {
+    if ((rc = fftstencil_run(p, p->dHostIn, p->dHostOut, total_steps, stream)) == FFTSTENCIL_OK &&
+        (e = cudaMemcpyAsync(h_out, p->dHostOut, bytes, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
       rc = cuda_fail(e, "D2H copy");
-    else if ((e = cudaStreamSynchronize(s)) != cudaSuccess)
-      rc = cuda_fail(e, "stream synchronize");
+    // the H2D read of h_in may still be queued when the run fails: synchronise either way
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess && rc == FFTSTENCIL_OK) rc = cuda_fail(e, "stream synchronize");
   }
   if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
   if (rc == FFTSTENCIL_OK) clear_error();
@@ -1280,6 +1320,7 @@ int fftstencil_plan_info(const fftstencil_plan* p, fftstencil_info* info) {
   info->device_bytes = p->device_bytes;
   info->fused_grid = p->fused_grid;
   info->last_run_launches = p->last_launches;
+  info->last_run_pipelined = p->last_pipelined ? 1 : 0;
   clear_error();
   return FFTSTENCIL_OK;
 }

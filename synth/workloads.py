@@ -64,13 +64,46 @@ def classic_weights(shape: str, ndim: int, radius: int) -> np.ndarray:
     return w
 
 
+def signed_weights(shape: str, ndim: int, radius: int, seed: int = WEIGHT_SEED + 1,
+                   abs_sum: float = 1.6) -> np.ndarray:
+    """Signed, un-normalised weights: shape mask x U(-1, 1), scaled so sum|w| = abs_sum; the
+    centre tap is made positive and the largest (so the symbol's modulus can exceed 1 and
+    the field may grow: SURVEY reading Q19 "other weights are allowed")."""
+    m = mask(shape, ndim, radius)
+    rng = np.random.default_rng(seed)
+    w = rng.uniform(-1.0, 1.0, size=m.shape) * m
+    c = (radius,) * ndim
+    w[c] = np.abs(w).max() + 0.25
+    return (w * (abs_sum / np.abs(w).sum())).astype(np.float64)
+
+
+def gain_weights(shape: str, ndim: int, radius: int, gain: float = 1.2) -> np.ndarray:
+    """The seeded set scaled to sum w = gain (> 1): the symbol's modulus peaks at gain at
+    theta = 0, so a constant field grows by gain per step."""
+    return (seeded_weights(shape, ndim, radius) * gain).astype(np.float64)
+
+
 def stencil_weights(shape: str, ndim: int, radius: int, kind: str = "seeded") -> np.ndarray:
-    return seeded_weights(shape, ndim, radius) if kind == "seeded" else classic_weights(shape, ndim, radius)
+    if kind == "seeded":
+        return seeded_weights(shape, ndim, radius)
+    if kind == "signed":
+        return signed_weights(shape, ndim, radius)
+    if kind == "signed_unit":      # signed, sum|w| = 1 (bounded growth for long runs)
+        return signed_weights(shape, ndim, radius, abs_sum=1.0)
+    if kind == "gain":
+        return gain_weights(shape, ndim, radius)
+    return classic_weights(shape, ndim, radius)
 
 
 def grid(extents, cfg_id: int = 0) -> np.ndarray:
     rng = np.random.default_rng(GRID_SEED_BASE + cfg_id)
     return rng.random(tuple(int(e) for e in extents))
+
+
+def signed_grid(extents, cfg_id: int = 0) -> np.ndarray:
+    """float64 U(-1, 1) input (signed values; the benchmark grids are U[0, 1))."""
+    rng = np.random.default_rng(GRID_SEED_BASE + 7919 + cfg_id)
+    return rng.uniform(-1.0, 1.0, tuple(int(e) for e in extents))
 
 
 @dataclass(frozen=True)

@@ -16,7 +16,7 @@ import paper_conf_ppopp_hanlcbzyczcy25_b200 as fs
 from synth import workloads as wl
 
 
-def replay(ext, shape, r, T, steps, K, Q, mutate=None):
+def replay(ext, shape, r, T, steps, K, Q, mutate=None, check_cover=True):
     w = wl.seeded_weights(shape, len(ext), r)
     info = fs.describe(ext, w, r, T)
     h, S, n0 = info["halo"], info["valid"][0], ext[0]
@@ -33,6 +33,9 @@ def replay(ext, shape, r, T, steps, K, Q, mutate=None):
     out_buf = 0 if P % 2 else 1          # dsts[0] = out when P is odd
     h2d, d2h = np.zeros(n0, int), np.zeros(n0, int)
     cover = np.zeros((P + 1, U), int)
+    # rows of the output buffer already queued for copy-out: the D2H runs asynchronously on the
+    # copy stream while later items keep writing the same buffer, so none may touch them again
+    frozen = np.zeros(n0, bool)
     for op, x, y, z in ops:
         if op == 0:
             h2d[x:y] += 1
@@ -53,13 +56,17 @@ def replay(ext, shape, r, T, steps, K, Q, mutate=None):
                 assert (ver[src, rlo:rhi] == k - 1).all(), \
                     f"pass {k} units [{u0},{u1}) read rows not holding pass {k - 1}"
                 assert ring_ok[src, rlo:rhi].all()
+            if dst == out_buf:
+                assert not frozen[lo:hi].any(), f"pass {k} units [{u0},{u1}) write rows queued for copy-out"
             ver[dst, lo:hi] = k
         else:
             assert (ver[out_buf, x:y] == P).all(), "rows copied out before the last pass"
             assert ring_ok[out_buf, x:y].all()
             d2h[x:y] += 1
+            frozen[x:y] = True
     assert (h2d == 1).all() and (d2h == 1).all()
-    assert (cover[1:] == 1).all(), "every pass must produce every unit exactly once"
+    if check_cover:
+        assert (cover[1:] == 1).all(), "every pass must produce every unit exactly once"
     return ops, U, P
 
 
@@ -140,3 +147,17 @@ def test_replay_catches_item_before_its_input_chunk():
         return np.concatenate([ops[:c2], ops[it:it + 1], ops[c2:it], ops[it + 1:]])
     with pytest.raises(AssertionError):
         replay((1500, 200), "star", 1, 11, 100, 4, 6, mutate=mutate)
+
+
+def test_replay_catches_write_after_copy_out():
+    """A later item that rewrites rows already queued for copy-out (the D2H reads them
+    asynchronously) fails the frozen-rows check even where every version check passes: here a
+    pass-P item re-issued after the first copy-out on the units that copy covered."""
+    def mutate(ops):
+        i3 = next(i for i in range(len(ops)) if ops[i, 0] == 3)
+        P = int(ops[ops[:, 0] == 2, 1].max())
+        it = next(i for i in range(i3) if ops[i, 0] == 2 and ops[i, 1] == P)   # a pass-P item before it
+        return np.concatenate([ops[:i3 + 1], ops[it:it + 1], ops[i3 + 1:]])
+    replay((1500, 200), "star", 1, 11, 100, 4, 6, check_cover=False)          # the clean schedule passes
+    with pytest.raises(AssertionError, match="queued for copy-out"):
+        replay((1500, 200), "star", 1, 11, 100, 4, 6, mutate=mutate, check_cover=False)

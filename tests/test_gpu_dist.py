@@ -79,3 +79,27 @@ def test_nccl_single_rank_plan_runs(fs):
     torch.cuda.synchronize()
     ref = oracle.stencil_run(u0, w, 1, 9)
     assert np.abs(b.cpu().numpy() - ref).max() <= 1e-9
+
+
+def test_nccl_two_ranks_bitwise(fs, tmp_path):
+    """The NCCL halo exchange (ncclSend / ncclRecv on the plan's comm stream, overlapped with the
+    halo-free pairs) on two GPUs, bitwise equal to one GPU (G7).  Needs >= 2 visible devices."""
+    import os
+    import socket
+    import subprocess
+    import sys
+    if torch.cuda.device_count() < 2:
+        pytest.skip("needs >= 2 CUDA devices (NCCL refuses two ranks on one GPU)")
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    worker = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_nccl_worker.py")
+    env = dict(os.environ, NCCL_DEBUG="INFO")
+    res = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+                          "--master-addr=127.0.0.1", f"--master-port={port}", worker],
+                         capture_output=True, text=True, env=env, timeout=600)
+    log = res.stdout + res.stderr
+    (tmp_path / "nccl.log").write_text(log)
+    assert res.returncode == 0, log[-4000:]
+    assert log.count("bitwise OK") == 5, log[-4000:]
+    assert "Init COMPLETE" in log or "ncclCommInitRank" in log, "no NCCL communicator was initialised"

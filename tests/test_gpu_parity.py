@@ -311,16 +311,19 @@ def test_launch_count_reported(fs):
 
 
 # ---------------------------------------------------------------- full BASELINE sizes
-@pytest.mark.parametrize("name,T", [("heat2d", 8), ("box2d9p", 8), ("star2d13p", 4), ("box2d49p", 4),
-                                    ("box2d9p", 1), ("heat2d", 16)])
+@pytest.mark.parametrize("name,T", [("heat2d", 0), ("box2d9p", 0), ("star2d13p", 0), ("box2d49p", 0),
+                                    ("heat2d", 8), ("box2d9p", 8), ("box2d9p", 1), ("heat2d", 16)])
 def test_full_size_sampled(fs, name, T):
-    """10240^2 at parity steps 2T+3 (launch configuration of bench.py); sampled cells
-    (interior, band, ring, tile seams) against the oracle's single-cell evaluation."""
+    """10240^2 at parity steps 2T+3; T = 0 is bench.py's own plan (automatic T, the launch
+    configuration it times); sampled cells (interior, band, ring, tile seams) against the
+    oracle's single-cell evaluation."""
     wk = wl.CONFIGS[name]
     w = wk.weights()
     u0 = wk.grid()
-    steps = 2 * T + 3
+    T_plan = fs.describe(wk.extents, w, wk.radius, T)["T"]
+    steps = 2 * T_plan + 3
     got, p = run_gpu(fs, u0, w, wk.radius, T, steps)
+    assert p.info()["T"] == T_plan
     info = p.info()
     rng = np.random.default_rng(17)
     n = np.array(wk.extents)
@@ -339,13 +342,14 @@ def test_full_size_sampled(fs, name, T):
     assert got.min() >= u0.min() - 1e-9 and got.max() <= u0.max() + 1e-9
 
 
-@pytest.mark.parametrize("name,T", [("heat3d", 2), ("box3d27p", 2), ("heat3d", 1), ("box3d27p", 3)])
+@pytest.mark.parametrize("name,T", [("heat3d", 0), ("box3d27p", 0), ("heat3d", 1), ("box3d27p", 3)])
 def test_full_size_3d_sampled(fs, name, T):
-    """1024^3 at parity steps 2T+3; sampled cells against the single-cell oracle."""
+    """1024^3 at parity steps 2T+3 (T = 0: bench.py's automatic plan); sampled cells against
+    the single-cell oracle."""
     wk = wl.CONFIGS[name]
     w = wk.weights()
     u0 = wk.grid()
-    steps = 2 * T + 3
+    steps = 2 * fs.describe(wk.extents, w, wk.radius, T)["T"] + 3
     got, p = run_gpu(fs, u0, w, wk.radius, T, steps)
     info = p.info()
     rng = np.random.default_rng(23)
@@ -472,11 +476,8 @@ def test_parity_2d_engines(fs, monkeypatch, engine, tma, ext, shape, r, T, steps
     monkeypatch.setenv("FFTSTENCIL_TMA", tma)
     w = wl.stencil_weights(shape, len(ext), r, kind)
     u0 = wl.grid(ext, 13)
-    try:
-        got, p = run_gpu(fs, u0, w, r, T, steps)
-    except Exception as e:   # a tile too small for the requested T: the factored 64-tile needs S >= 8
-        pytest.skip(str(e))
-    assert p.info()["engine"] == engine
+    got, p = run_gpu(fs, u0, w, r, T, steps)
+    assert p.info()["engine"] == engine and p.info()["algo"] == "factored"
     ref = oracle.stencil_run(u0, w, r, steps)
     assert rel_err(got, ref) <= TOL, (rel_err(got, ref), p.info())
 

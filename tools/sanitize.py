@@ -10,7 +10,7 @@ import paper_conf_ppopp_hanlcbzyczcy25_b200 as fs  # noqa: E402
 from synth import workloads as wl  # noqa: E402
 
 torch.cuda.set_device(0)
-F, D = "FFTSTENCIL_ALGO", "FFTSTENCIL_ENGINE"
+F, D, C = "FFTSTENCIL_ALGO", "FFTSTENCIL_ENGINE", "FFTSTENCIL_MAX_CTAS"
 cases = [((150, 140), "box", 1, 4, 9, {}), ((150, 140), "box", 1, 4, 9, {F: "dense"}),
          ((150, 140), "box", 1, 4, 9, {F: "factored", D: "dmma"}),
          ((130, 98), "star", 2, 3, 7, {"FFTSTENCIL_TMA": "0"}),
@@ -19,7 +19,13 @@ cases = [((150, 140), "box", 1, 4, 9, {}), ((150, 140), "box", 1, 4, 9, {F: "den
          ((33, 35, 37), "star", 1, 2, 3, {"FFTSTENCIL_TMA": "0"}), ((900,), "star", 1, 8, 19, {}),
          ((16384,), "star", 1, 1024, 1030, {F: "factored"}),                      # 1D ALU, TMA rows
          ((9000,), "star", 3, 352, 400, {F: "factored"}),                         # 1D ALU, cp.async
-         ((9000,), "star", 3, 352, 400, {F: "factored", D: "dmma"})]
+         ((9000,), "star", 3, 352, 400, {F: "factored", D: "dmma"}),
+         # steady state of the persistent ALU kernels: one CTA, each group walks 5-20 pairs
+         # through the TMA refill / mbarrier-parity loop (and the cp.async loop)
+         ((300, 290), "box", 1, 8, 19, {C: "1"}), ((300, 290), "box", 1, 8, 19, {C: "1", "FFTSTENCIL_TMA": "0"}),
+         ((60, 50, 45), "star", 1, 2, 5, {C: "1"}), ((60, 50, 45), "star", 1, 2, 5, {C: "1", "FFTSTENCIL_TMA": "0"}),
+         ((65536,), "star", 2, 512, 1100, {C: "1", F: "factored"}),
+         ((90001,), "star", 1, 300, 650, {C: "1", F: "factored"})]
 for ext, shape, r, T, steps, env in cases:
     for k, v in env.items():
         os.environ[k] = v
