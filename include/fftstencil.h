@@ -109,7 +109,14 @@ enum {
                                neighbours wrap modulo the extents; single GPU */
 };
 
-/* Build a plan (host precompute + device upload).  Returns NULL on error. */
+/* Build a plan (host precompute + device upload).  Returns NULL on error.
+ * What it computes: the tile size and fused depth T (the role of Eq. 5, re-derived
+ * as a B200 cost model), the per-axis DFT tables (Algorithm 1 inputs F, L254),
+ * the powered spectra S_t = sigma^t / prod(L) for t = 1..T (Eq. 10; reading Q6/Q7), the
+ * overlap-save tile schedule (Eq. 3, Eq. 4) and the boundary band blocks; only the
+ * tile-sized auxiliary data is kept on the device (L200: 2(2L^2+L), not the grid's).
+ * Ownership: the caller keeps `extents` and `weights`; the plan owns its device memory.
+ * Errors: NULL + last_error (EINVAL for bad arguments, ECUDA / ENOMEM on device failure). */
 fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const double* weights,
                                         int radius, int T);
 
@@ -117,8 +124,12 @@ fftstencil_plan* fftstencil_plan_create(int ndim, const int64_t* extents, const 
 fftstencil_plan* fftstencil_plan_create_ex(int ndim, const int64_t* extents, const double* weights,
                                            int radius, int T, int flags);
 
-/* Enqueue `total_steps` (>= 0) time steps on `stream` (a cudaStream_t; NULL = the
- * legacy default stream).  `in` and `out` are device pointers to prod(extents) FP64
+/* The hot path.  Enqueue `total_steps` (>= 0) time steps on `stream` (a cudaStream_t; NULL =
+ * the legacy default stream): floor(total_steps / T) fused passes with S_T and one with
+ * S_(total_steps mod T) (the temporal driver, §4, Fig. 2 left L111-L128; reading
+ * Q15), each pass = per tile pair: halo'd load, forward DFT, * S_t, inverse DFT, crop and
+ * stitch (Algorithm 1, Stitching Eq. 7) in one kernel (Fusing L190-L198),
+ * plus the band cells' direct steps (reading Q5).  `in` and `out` are device pointers to prod(extents) FP64
  * values on the plan's device; the caller owns them.  `in` is read only unless it
  * aliases `out` (allowed).  total_steps == 0 copies in to out.  Asynchronous: no host
  * synchronisation.  Returns FFTSTENCIL_OK or a negative code.
@@ -167,7 +178,9 @@ fftstencil_plan* fftstencil_plan_create_dist(int ndim, const int64_t* extents, c
                                              int radius, int T, int nranks, int rank,
                                              const void* nccl_unique_id);
 
-/* Writes a new 128-byte ncclUniqueId into `out` (rank 0 of a group). */
+/* Writes a new 128-byte ncclUniqueId into `out` (caller-owned, >= 128 bytes; rank 0 of a
+ * group).  ENCCL if NCCL cannot create one.  No PAPER.md passage: the paper is single-GPU;
+ * the decomposition is SURVEY §8(a) row a10. */
 int fftstencil_nccl_unique_id(void* out);
 
 /* Runs loopback ranks 0..nranks-1 (plans[k] created with rank k, nccl_unique_id NULL, on the
@@ -180,10 +193,14 @@ int fftstencil_run_group(fftstencil_plan* const* plans, const double* const* in,
 int fftstencil_describe_dist(int ndim, const int64_t* extents, const double* weights, int radius,
                              int T, int nranks, int rank, fftstencil_info* info);
 
-/* Release everything the plan owns.  NULL is a no-op. */
+/* Release everything the plan owns (device tables, scratch grids, streams, events, the NCCL
+ * communicator).  NULL is a no-op.  Must not race a pending fftstencil_run on the plan:
+ * synchronise its stream first. */
 void fftstencil_destroy(fftstencil_plan* plan);
 
-/* Plan geometry and cost model. */
+/* Plan geometry and cost model (tile, valid window S = L - 2h of Eq. 4 / reading Q4, T,
+ * pair counts of Eq. 9, algorithmic flops per cell-step, FP64 ALU instructions per launch,
+ * launches of the last run).  `info` is caller-owned.  EINVAL for NULL arguments. */
 int fftstencil_plan_info(const fftstencil_plan* plan, fftstencil_info* info);
 
 /* Per-kernel timing for roofline reporting.  With profiling enabled, fftstencil_run
