@@ -46,7 +46,7 @@ NVFLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "
            "-I", INCLUDE, "-I", CSRC, "-I", NCCL_INC, *DEFS]
 CXXFLAGS = ["-O2", "-std=c++17", "-fPIC", "-I", INCLUDE, "-I", CSRC, *DEFS]
 
-CU = ["capi.cu", "kernel_fft2d.cu", "kernel_fft2d_ct.cu", "kernel_fft1d.cu", "kernel_fft1d_ct.cu", "kernel_fft3d.cu", "kernel_fft3d_ct.cu", "kernel_fft3d_bf.cu", "kernel_fft3d_b3.cu", "kernel_fft2d_bf.cu", "kernel_fft1d_bf.cu", "kernel_band.cu", "kernel_small1d.cu"]
+CU = ["capi.cu", "kernel_fft2d.cu", "kernel_fft2d_ct.cu", "kernel_fft1d.cu", "kernel_fft1d_ct.cu", "kernel_fft3d.cu", "kernel_fft3d_ct.cu", "kernel_fft3d_bf.cu", "kernel_fft2d_bf.cu", "kernel_fft1d_bf.cu", "kernel_band.cu", "kernel_small1d.cu"]
 CPP = ["plan.cpp"]
 HEADERS = ["plan.h", "kernels.cuh", "device_common.cuh", "tma.cuh", "ct_line.cuh", "fft_radix.cuh"]
 

@@ -355,9 +355,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
       const uint64_t dims[3] = {(uint64_t)hp.ext[2], (uint64_t)hp.ext[1], (uint64_t)(hp.g1 - hp.g0)};
       const uint32_t box[3] = {16, 16, 16};
       const bool use_tma = p->use_tma && !hp.periodic && encode_tensor_map(&tm, src, 3, dims, box, hp.engine == 1);
-      if (hp.engine == 1 && hp.kernel3d == 0)
-        e = launch_fused3d_b3(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
-      else if (hp.engine == 1)
+      if (hp.engine == 1)
         e = launch_fused3d_bf(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
       else
         e = launch_fused3d_ct(a, use_tma ? &tm : nullptr, (int)std::min<int64_t>(fg, np), s);
@@ -714,8 +712,7 @@ int setup_device(fftstencil_plan* p) {
     if (e != cudaSuccess) return cuda_fail(e, "fused 2D kernel configuration");
   } else if (hp.ndim == 3 && hp.algo == 1) {
     if (const char* v = std::getenv("FFTSTENCIL_TMA")) p->use_tma = std::atoi(v) != 0;
-    e = hp.engine == 1 ? (hp.kernel3d == 0 ? fused3d_b3_configure(&occ) : fused3d_bf_configure(&occ))
-                       : fused3d_ct_configure(&occ);
+    e = hp.engine == 1 ? fused3d_bf_configure(&occ) : fused3d_ct_configure(&occ);
     if (e != cudaSuccess) return cuda_fail(e, "factored 3D kernel configuration");
   } else if (hp.ndim == 3) {
     e = fused3d_configure(&occ);

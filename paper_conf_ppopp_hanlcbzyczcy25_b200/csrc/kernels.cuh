@@ -199,10 +199,6 @@ cudaError_t launch_fused2d_bf(const Fft2dArgs& a, const CUtensorMap* tm, int gri
 size_t fused3d_bf_smem(bool tma);
 cudaError_t fused3d_bf_configure(int* max_blocks_per_sm);
 cudaError_t launch_fused3d_bf(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
-// three-pass pair-shuffle 3D kernel (kernel_fft3d_b3.cu), the default 3D ALU engine
-size_t fused3d_b3_smem();
-cudaError_t fused3d_b3_configure(int* max_blocks_per_sm);
-cudaError_t launch_fused3d_b3(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s);
 
 constexpr int kBandThreads = 256;
 cudaError_t band_configure(size_t smem);

@@ -125,20 +125,6 @@ static double model_flops_3d_bf(int S, int T) {
   return (168.0 * lines_3d_bf(S) + 6.0 * 4096.0) / (2.0 * S * (double)S * S * T);
 }
 static double alu_ops_3d_bf(int S) { return 160.0 * lines_3d_bf(S) + 4.0 * 4096.0; }
-// Three-pass pair-shuffle kernel (kernel_fft3d_b3.cu), per pair: P1 on 128 lanes (2 FFT-16,
-// pair DFT-4 over j = 64 local + 64 cross, 2 x 16 twiddles = 576); P2 on 128 lanes (2 + 2 FFT-16,
-// forward pair DFT-4, S_T = 128, inverse pair DFT-4 and twiddles on the S output planes
-// 8 S + 8 S... = 896 + 16 S); P3 on the 8 S lanes of the output planes (pair DFT-4 128 + 2
-// inverse FFT-16 320 = 448).  Flops: FFT-16 168, pair DFT-4 8 per element, cmul 6.
-static double alu_ops_3d_b3(int S) { return 128.0 * (576.0 + 896.0 + 16.0 * S) + 8.0 * S * 448.0; }
-static double flops_3d_b3(int S) {
-  return 128.0 * (2 * 168.0 + 128.0 + 32 * 6.0 + 4 * 168.0 + 128.0 + 32 * 6.0 + S * (16.0 + 12.0)) +
-         8.0 * S * (128.0 + 2 * 168.0);
-}
-static int env_kernel3d() {
-  const char* v = std::getenv("FFTSTENCIL_3D_KERNEL");
-  return v && !std::strcmp(v, "lines") ? 1 : 0;
-}
 // Relative cost of one executed flop on the ALU engine vs a DMMA flop: both share the FP64
 // pipe (profiles/r01_fp64_shared.txt); adds cost a full FMA slot (~0.55 flop per slot-flop)
 // and the passes are shared-memory heavy -- assumed until measured.
@@ -348,17 +334,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
       p.fused_smem = (size_t)(2 * 16 * 20 + 2 * 16 * (16 * 20 + 4)) * sizeof(double);
     } else if (engine) {
       p.engine = 1;
-      p.kernel3d = env_kernel3d();
       p.mma_flops_per_pair = 0;
-      if (p.kernel3d == 0) {
-        p.flops_per_cell_step = flops_3d_b3(p.S[0]) / (2.0 * S * S * S * bestT);
-        p.alu_ops_per_pair = alu_ops_3d_b3(p.S[0]);
-        p.fused_smem = (size_t)6 * 16 * 16 * 16 * sizeof(double) + 1024;   // 3 pair buffers (S_T in TMEM)
-      } else {
-        p.flops_per_cell_step = model_flops_3d_bf(p.S[0], bestT);
-        p.alu_ops_per_pair = alu_ops_3d_bf(p.S[0]);
-        p.fused_smem = (size_t)6 * 16 * 16 * 16 * sizeof(double) + 1024;   // 2 pair buffers + S_T
-      }
+      p.flops_per_cell_step = model_flops_3d_bf(p.S[0], bestT);
+      p.alu_ops_per_pair = alu_ops_3d_bf(p.S[0]);
+      p.fused_smem = (size_t)6 * 16 * 16 * 16 * sizeof(double) + 1024;   // 2 pair buffers + S_T
     } else {
       p.flops_per_cell_step = model_flops_3d_ct(p.S[0], bestT);
       p.mma_flops_per_pair = prod_dmma_flops(kCmul3_3d) * groups_3d_ct(p.S[0]);

@@ -59,8 +59,6 @@ struct HostPlan {
   int engine = 0;                  // line-DFT engine of the factored 3D tile: 0 DFT-8 GEMMs on the
                                    // FP64 tensor pipe (kernel_fft3d_ct.cu), 1 radix-4 FFTs on the
                                    // FP64 ALU (kernel_fft3d_bf.cu); FFTSTENCIL_ENGINE=dmma|alu
-  int kernel3d = 0;                // 3D ALU engine: 0 three-pass pair-shuffle kernel (kernel_fft3d_b3.cu),
-                                   // 1 five-pass line kernel (kernel_fft3d_bf.cu); FFTSTENCIL_3D_KERNEL=pairs|lines
   double alu_ops_per_pair = 0;     // FP64 ALU instructions per pair (engine 1: adds, muls, FMAs)
   int64_t nt[3] = {1, 1, 1};       // tiles per user axis
   int64_t tiles = 0, pairs = 0;
