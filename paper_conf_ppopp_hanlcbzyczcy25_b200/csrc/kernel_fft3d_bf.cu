@@ -67,21 +67,25 @@ __device__ __forceinline__ void stc(double* b, int o, double re, double im) {
 // Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
 __device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
 
-// BF3_PINGPONG = 1: the two groups take turns at shared memory (ping-pong schedule, as
-// kernel_fft2d_bf.cu's BF_PINGPONG): each pass is a memory phase (previous pass's stores,
-// barrier, this pass's loads) then a compute phase; group g waits on barrier 3 + g before a
-// memory phase and arrives on the other group's barrier once its loads have returned.
-#ifndef BF3_PINGPONG
-#define BF3_PINGPONG 0
-#endif
-__device__ __forceinline__ void pp_begin(int grp, bool first_phase) {
-  if (BF3_PINGPONG && !(grp == 0 && first_phase))
-    asm volatile("bar.sync %0, %1;\n" ::"r"(3 + grp), "r"(2 * NT) : "memory");
+// tensor memory: 16 consecutive 32-bit columns of this warp's lane quarter
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),
+        "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
 }
-__device__ __forceinline__ void pp_end(int grp, bool last_phase, double a0, double a1, double a2, double a3) {
-  if (BF3_PINGPONG && !(grp == 1 && last_phase))
-    asm volatile("bar.arrive %0, %1;\n" ::"r"(4 - grp), "r"(2 * NT), "d"(a0), "d"(a1), "d"(a2), "d"(a3) : "memory");
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
+          taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
 }
+__device__ __forceinline__ double u2d(uint32_t lo, uint32_t hi) { return __hiloint2double((int)hi, (int)lo); }
+constexpr uint32_t kTmemCols = 128;
 
 struct PairGeom {
   int64_t o0, o1, oa2, ob2;
@@ -102,66 +106,90 @@ __device__ __forceinline__ PairGeom pair_geom(const Fft3dArgs& a, int64_t p) {
 }
 
 // One CTA per SM = two independent 256-thread groups, each transforming its own sequence of
-// tile pairs in its own 64 KB buffer (the other group's work hides a group's TMA latency and
-// barrier waits); S_T (64 KB) is staged once and shared: 192 KB.  Thread t of a group owns
-// line (t >> 4, t & 15) of every pass, so a warp's P1 rows and P2 lines lie in the same two
-// l0-planes (P1 -> P2 needs only __syncwarp), and likewise P4 -> P5 on the output planes.
-// TMA = false: cp.async loads (periodic wrap-around, or a pitch TMA cannot describe).
+// tile pairs (the other group's work hides a group's TMA latency and barrier waits).  Thread
+// t of a group owns line (t >> 4, t & 15) of every pass, so a warp's P1 rows and P2 lines lie
+// in the same two l0-planes (P1 -> P2 needs only __syncwarp), and likewise P4 -> P5.
+// Local pair j of the CTA (global pair p_begin + 2 blockIdx.x + (j & 1) + (j >> 1) 2 gridDim.x)
+// belongs to group j & 1.  TMA: three 64 KB pair buffers in a ring, pair j in buffer j % 3;
+// when a group has read pair j for the last time (P5's loads) it refills that buffer with
+// pair j + 3 (the OTHER group's next-but-one pair), so every pair's boxes are issued about
+// one and a half pairs ahead of their use (with two buffers, only during P5).  TMA = false:
+// cp.async loads into the group's own buffer (periodic wrap-around, or a pitch TMA cannot
+// describe).
 template <bool TMA, bool WRAP = false>
 __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ unsigned char smem_raw[];
   const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
   double* base = reinterpret_cast<double*>(smem_raw + (mis ? kAlign - mis : 0));   // stays in the shared window
-  double* sS = base + 4 * PLANE;   // S_T interleaved (re, im), natural [k0][k1][k2]
-  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ __align__(8) uint64_t full[3];
+  __shared__ uint32_t tmem_base;
+  const int warp = threadIdx.x >> 5;
   const int grp = threadIdx.x >> 8, tid = threadIdx.x & (NT - 1);
   const int hi = tid >> 4, lo = tid & 15;
   const int S = a.S, h = a.h;
-  double* sR = base + grp * 2 * PLANE;
-  double* sI = sR + PLANE;
-  if (threadIdx.x == 0) {
-    tma::mbar_init(&bar[0], 1);
-    tma::mbar_init(&bar[1], 1);
+  if (threadIdx.x == 0)
+    for (int b = 0; b < 3; ++b) tma::mbar_init(&full[b], 1);
+  // ---- S_T into tensor memory: lane 32 (warp & 3) + lane holds P3 column tid's 16 values at
+  // columns 64 ((warp >> 2) & 1) + 4 k0 + {re lo, re hi, im lo, im hi}; group 0 writes, group 1
+  // (same warp & 7 -> same tid) shares them ----
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(tma::smem_addr(&tmem_base)),
+                 "r"(kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
   }
-  for (int e = threadIdx.x; e < PLANE; e += 2 * NT) stc(sS, 2 * e, __ldg(a.Sre + e), __ldg(a.Sim + e));   // once per launch
+  asm volatile("tcgen05.fence::before_thread_sync;\n");
   __syncthreads();
-  const int64_t stride = 2 * (int64_t)gridDim.x;
-  const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
-  auto issue = [&](int64_t p) {
-    const PairGeom g = pair_geom(a, p);
-    tma::mbar_expect_tx(&bar[grp], (g.has_b ? 2u : 1u) * PLANE * 8u);
-    tma::load_3d(sR, &tm, (int)g.oa2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
-    if (g.has_b) tma::load_3d(sI, &tm, (int)g.ob2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
-  };
-  if (TMA && tid == 0 && p0 < a.win.p_end) issue(p0);
-
-  // pairs of this group and of group 0 (which owns as many as group 1 or one more)
-  const int64_t pb0 = a.win.p_begin + 2 * (int64_t)blockIdx.x;
-  const int64_t n0 = pb0 < a.win.p_end ? (a.win.p_end - pb0 + stride - 1) / stride : 0;
-  const int64_t nmine = p0 < a.win.p_end ? (a.win.p_end - p0 + stride - 1) / stride : 0;
-  const int64_t niter = BF3_PINGPONG ? n0 : nmine;
-  uint32_t parity = 0;
-  for (int64_t it = 0; it < niter; ++it) {
-    const int64_t p = p0 + it * stride;
-    const bool last = it == niter - 1;
-    if (it >= nmine) {   // ping-pong turns without work (group 1)
+  asm volatile("tcgen05.fence::after_thread_sync;\n");
+  const uint32_t tmem_s = tmem_base + ((uint32_t)(32 * (warp & 3)) << 16) + 64 * ((warp >> 2) & 1);
+  if (grp == 0) {
 #pragma unroll 1
-      for (int k = 0; k < 5; ++k) {
-        pp_begin(grp, false);
-        pp_end(grp, last && k == 4, 0.0, 0.0, 0.0, 0.0);
+    for (int q = 0; q < 4; ++q) {
+      uint32_t v[16];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const int k0 = 4 * q + e;
+        const double re = __ldg(a.Sre + (k0 << 8) + tid), im = __ldg(a.Sim + (k0 << 8) + tid);
+        v[4 * e] = (uint32_t)__double2loint(re);
+        v[4 * e + 1] = (uint32_t)__double2hiint(re);
+        v[4 * e + 2] = (uint32_t)__double2loint(im);
+        v[4 * e + 3] = (uint32_t)__double2hiint(im);
       }
-      continue;
+      tmem_st16(tmem_s + 16 * q, v);
     }
+    asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;\n");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;\n");
+
+  const int64_t pb = a.win.p_begin + 2 * (int64_t)blockIdx.x, gstride = 2 * (int64_t)gridDim.x;
+  auto pair_of = [&](int64_t j) { return pb + (j & 1) + (j >> 1) * gstride; };
+  auto issue = [&](int64_t j) {   // pair j's boxes into buffer j % 3
+    const int64_t p = pair_of(j);
+    if (p >= a.win.p_end) return;
     const PairGeom g = pair_geom(a, p);
-    pp_begin(grp, it == 0);   // M of P1: the tile's arrival and P1's loads
+    double* dR = base + (int)(j % 3) * 2 * PLANE;
+    uint64_t* bar = &full[j % 3];
+    tma::mbar_expect_tx(bar, (g.has_b ? 2u : 1u) * PLANE * 8u);
+    tma::load_3d(dR, &tm, (int)g.oa2, (int)g.o1, (int)(g.o0 - a.win.g0), bar);
+    if (g.has_b) tma::load_3d(dR + PLANE, &tm, (int)g.ob2, (int)g.o1, (int)(g.o0 - a.win.g0), bar);
+  };
+  if (TMA && threadIdx.x == 0)
+    for (int j = 0; j < 3; ++j) issue(j);
+
+  for (int64_t j = grp; pair_of(j) < a.win.p_end; j += 2) {
+    const int64_t p = pair_of(j);
+    const PairGeom g = pair_geom(a, p);
+    double* sR = base + (TMA ? (int)(j % 3) : grp) * 2 * PLANE;
+    double* sI = sR + PLANE;
     if (TMA) {
-      tma::mbar_wait(&bar[grp], parity);
-      parity ^= 1;
+      tma::mbar_wait(&full[j % 3], (uint32_t)((j / 3) & 1));
       if (!g.has_b) {
         for (int e = tid; e < PLANE; e += NT) sI[e] = 0.0;
         group_sync(grp);
       }
     } else {
+      group_sync(grp);   // the group's previous pair has left the buffer
       for (int e = tid; e < 2 * PLANE; e += NT) {
         const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
         int64_t g0 = g.o0 + l0, g1 = g.o1 + l1, g2 = (t ? g.ob2 : g.oa2) + l2;
@@ -178,9 +206,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     double xr[16], xi[16];
     // ---- P1: forward axis 2 (thread = row (l0, l1) = (hi, lo)); TMA planes -> interleaved ----
     load_row(sR, sI, hi, lo, xr, xi);
-    pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
     radix::fft16<false>(xr, xi);
-    pp_begin(grp, false);   // M of P2: P1's stores and P2's loads
 #pragma unroll
     for (int l2 = 0; l2 < 16; ++l2) stc(sR, cofs(hi, lo, l2), xr[l2], xi[l2]);
     __syncwarp();
@@ -191,9 +217,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
       xr[l1] = v.x;
       xi[l1] = v.y;
     }
-    pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
     radix::fft16<false>(xr, xi);
-    pp_begin(grp, false);   // M of P3
 #pragma unroll
     for (int l1 = 0; l1 < 16; ++l1) stc(sR, cofs(hi, l1, lo), xr[l1], xi[l1]);
     group_sync(grp);
@@ -206,15 +230,16 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
         xr[l0] = v.x;
         xi[l0] = v.y;
       }
-      pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
       radix::fft16<false>(xr, xi);
 #pragma unroll
-      for (int k0 = 0; k0 < 16; ++k0) {
-        const double2 sv = ldc(sS, ((k0 << 8) + tid) << 1);
-        radix::cmul(xr[k0], xi[k0], sv.x, sv.y);
+      for (int q = 0; q < 4; ++q) {
+        uint32_t v[16];
+        tmem_ld16(tmem_s + 16 * q, v);
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          radix::cmul(xr[4 * q + e], xi[4 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
       }
       radix::fft16<true>(xr, xi);
-      pp_begin(grp, false);   // M of P4
 #pragma unroll
       for (int l0 = 0; l0 < 16; ++l0)
         if (l0 >= h && l0 < h + S) stc(sR, b + (l0 << 8), xr[l0], xi[l0]);
@@ -229,9 +254,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
         xi[l1] = v.y;
       }
     }
-    pp_end(grp, false, xr[0], xi[0], xr[15], xi[15]);
     if (hi < S) radix::fft16<true>(xr, xi);
-    pp_begin(grp, false);   // M of P5
     if (hi < S) {
 #pragma unroll
       for (int l1 = 0; l1 < 16; ++l1)
@@ -252,8 +275,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     // refill it while the last transform and the stores run
     if (TMA) tma::fence_proxy_async();
     group_sync(grp);
-    if (TMA && tid == 0 && p + stride < a.win.p_end) issue(p + stride);
-    pp_end(grp, last, xr[0], xi[0], xr[15], xi[15]);
+    if (TMA && tid == 0) issue(j + 3);
     if (p5) {
       const int l0 = h + hi, l1 = h + lo;
       radix::fft16<true>(xr, xi);
@@ -283,11 +305,15 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
       }
     }
   }
+  asm volatile("tcgen05.fence::before_thread_sync;\n");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;\n");
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem_base), "r"(kTmemCols));
 }
 
 }  // namespace
 
-// Two group buffers + S_T.
+// Three pair buffers (TMA ring; the cp.async path uses two of them); S_T is in tensor memory.
 size_t fused3d_bf_smem(bool) { return (size_t)6 * PLANE * sizeof(double) + kAlign; }
 
 cudaError_t fused3d_bf_configure(int* max_blocks) {

@@ -72,7 +72,9 @@ double model_flops_2d_ct(int S, int T) {
   return f / (2.0 * S * (double)S * T);
 }
 
-static constexpr double kEffCt = 0.70;   // assumed until measured (profiles/)
+// measured: fused-kernel algorithmic flop rate / 37.18 TF/s on B200, Heat-2D / Box-2D9P /
+// Star-2D13P / Box-2D49P 0.82-0.84 (profiles/r01_configs.txt)
+static constexpr double kEffCt = 0.83;
 
 // Butterfly ALU engine (kernel_fft2d_bf.cu, 64 = 4 x 16 per axis), per pair and per thread of
 // the 256 that transform it: P1 and P5 eight DFT-4 (128 adds) + 24 complex twiddle multiplies
@@ -92,7 +94,9 @@ static constexpr int kP15Flops2d = BF_TW_COMB ? 128 + 90 : 272 + (BF_TW_REG ? 22
 static double flops_pair_2d_bf(int) { return 256.0 * (2 * kP15Flops2d + 2 * 168 + 432); }
 static double alu_ops_2d_bf(int) { return 256.0 * (2 * kP15Instr2d + 2 * 160 + 384); }
 static double model_flops_2d_bf(int S, int T) { return flops_pair_2d_bf(S) / (2.0 * S * (double)S * T); }
-static constexpr double kEff2dBf = 0.35;   // flops per FP64-pipe slot-flop x pipe efficiency (assumed)
+// measured: Heat-2D 1325 GSt/s x 8.65 flop = 11.5 TF (0.31 of 37.18), Box-2D49P 422 x 26.2 =
+// 11.1 TF (0.30) (BENCH_r01.json, profiles/r01_s3_sweep.txt)
+static constexpr double kEff2dBf = 0.30;
 
 // Measured DMMA issue efficiency of the fused 2D kernel per tile side (fraction of the
 // 37.18 TF/s peak, B200, profiles/r01_sweep.txt / r01_variants.txt): the plan minimises
@@ -125,10 +129,10 @@ static double model_flops_3d_bf(int S, int T) {
   return (168.0 * lines_3d_bf(S) + 6.0 * 4096.0) / (2.0 * S * (double)S * S * T);
 }
 static double alu_ops_3d_bf(int S) { return 160.0 * lines_3d_bf(S) + 4.0 * 4096.0; }
-// Relative cost of one executed flop on the ALU engine vs a DMMA flop: both share the FP64
-// pipe (profiles/r01_fp64_shared.txt); adds cost a full FMA slot (~0.55 flop per slot-flop)
-// and the passes are shared-memory heavy -- assumed until measured.
-static constexpr double kEff3dBf = 0.45;
+// Flop rate of the ALU engine relative to the 37.18 TF/s DMMA peak (both share the FP64 pipe,
+// profiles/r01_fp64_shared.txt), measured: Heat-3D 214 GSt/s x 36.6 flop = 7.8 TF (0.21)
+// (profiles/r01_s3_sweep.txt, gpurun_out r02 Heat-3D runs).
+static constexpr double kEff3dBf = 0.21;
 // FFTSTENCIL_ENGINE=dmma|alu pins the line engine of the factored 2D and 3D tiles (ablation);
 // default alu.
 static int env_engine() {
@@ -137,7 +141,7 @@ static int env_engine() {
   return 1;
 }
 static constexpr double kEff3d = 0.70;     // dense 3D: executed DMMA efficiency (profiles/r01_sweep.txt)
-static constexpr double kEff3dCt = 0.60;   // factored 3D: assumed until measured
+static constexpr double kEff3dCt = 0.62;   // factored 3D: measured 0.617 (profiles/r01_configs.txt)
 
 static double model_flops_3d(int L, int S, int T) {
   const double Sp = round8(S), l = L;
@@ -155,14 +159,16 @@ static constexpr double kEff1d = 0.73;     // PFA 8x7: executed DMMA efficiency 
 // 6 flops each).
 static double flops_pair_1d_ct() { return kProdFlops * 512.0 + 6.0 * 7.0 * 4096.0; }
 static double model_flops_1d_ct(int S, int T) { return flops_pair_1d_ct() / (2.0 * S * (double)T); }
-static constexpr double kEff1dCt = 0.70;   // assumed until measured
+static constexpr double kEff1dCt = 0.59;   // measured 0.586-0.605 on 2^29 cells (profiles/r01_configs.txt)
 // Butterfly ALU engine (kernel_fft1d_bf.cu), per pair and per thread of 256: P1/P3/P5/P7 four
 // DFT-4 + 12 twiddle multiplies (112 instr., 136 flops), P2/P6 a DFT-16 + 31 complex multiplies
 // (w4096 powers: 284 instr., 354 flops), P4 two DFT-16 + 16 spectrum multiplies (384, 432).
 static double flops_pair_1d_bf() { return 256.0 * (4 * 136 + 2 * 354 + 432); }
 static double alu_ops_1d_bf() { return 256.0 * (4 * 112 + 2 * 284 + 384); }
 static double model_flops_1d_bf(int S, int T) { return flops_pair_1d_bf() / (2.0 * S * (double)T); }
-static constexpr double kEff1dBf = 0.35;
+// measured: Heat-1D 2^29, T = 1024: 103.9 k GSt/s x 0.103 flop = 10.7 TF (0.29 of 37.18)
+// (profiles/r01_s3_sweep.txt)
+static constexpr double kEff1dBf = 0.29;
 
 static int env_engine();
 
