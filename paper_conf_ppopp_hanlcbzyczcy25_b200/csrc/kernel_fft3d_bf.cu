@@ -67,26 +67,6 @@ __device__ __forceinline__ void stc(double* b, int o, double re, double im) {
 // Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
 __device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
 
-// tensor memory: 16 consecutive 32-bit columns of this warp's lane quarter
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
-      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),
-        "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-      : "r"(taddr));
-  asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
-}
-__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
-  asm volatile(
-      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
-          taddr),
-      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
-      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
-      : "memory");
-}
-__device__ __forceinline__ double u2d(uint32_t lo, uint32_t hi) { return __hiloint2double((int)hi, (int)lo); }
-constexpr uint32_t kTmemCols = 128;
-
 struct PairGeom {
   int64_t o0, o1, oa2, ob2;
   bool has_b;
@@ -106,90 +86,50 @@ __device__ __forceinline__ PairGeom pair_geom(const Fft3dArgs& a, int64_t p) {
 }
 
 // One CTA per SM = two independent 256-thread groups, each transforming its own sequence of
-// tile pairs (the other group's work hides a group's TMA latency and barrier waits).  Thread
-// t of a group owns line (t >> 4, t & 15) of every pass, so a warp's P1 rows and P2 lines lie
-// in the same two l0-planes (P1 -> P2 needs only __syncwarp), and likewise P4 -> P5.
-// Local pair j of the CTA (global pair p_begin + 2 blockIdx.x + (j & 1) + (j >> 1) 2 gridDim.x)
-// belongs to group j & 1.  TMA: three 64 KB pair buffers in a ring, pair j in buffer j % 3;
-// when a group has read pair j for the last time (P5's loads) it refills that buffer with
-// pair j + 3 (the OTHER group's next-but-one pair), so every pair's boxes are issued about
-// one and a half pairs ahead of their use (with two buffers, only during P5).  TMA = false:
-// cp.async loads into the group's own buffer (periodic wrap-around, or a pitch TMA cannot
-// describe).
+// tile pairs in its own 64 KB buffer (the other group's work hides a group's TMA latency and
+// barrier waits); S_T (64 KB) is staged once and shared: 192 KB.  Thread t of a group owns
+// line (t >> 4, t & 15) of every pass, so a warp's P1 rows and P2 lines lie in the same two
+// l0-planes (P1 -> P2 needs only __syncwarp), and likewise P4 -> P5 on the output planes.
+// TMA = false: cp.async loads (periodic wrap-around, or a pitch TMA cannot describe).
 template <bool TMA, bool WRAP = false>
 __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ unsigned char smem_raw[];
   const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
   double* base = reinterpret_cast<double*>(smem_raw + (mis ? kAlign - mis : 0));   // stays in the shared window
-  __shared__ __align__(8) uint64_t full[3];
-  __shared__ uint32_t tmem_base;
-  const int warp = threadIdx.x >> 5;
+  double* sS = base + 4 * PLANE;   // S_T interleaved (re, im), natural [k0][k1][k2]
+  __shared__ __align__(8) uint64_t bar[2];
   const int grp = threadIdx.x >> 8, tid = threadIdx.x & (NT - 1);
   const int hi = tid >> 4, lo = tid & 15;
   const int S = a.S, h = a.h;
-  if (threadIdx.x == 0)
-    for (int b = 0; b < 3; ++b) tma::mbar_init(&full[b], 1);
-  // ---- S_T into tensor memory: lane 32 (warp & 3) + lane holds P3 column tid's 16 values at
-  // columns 64 ((warp >> 2) & 1) + 4 k0 + {re lo, re hi, im lo, im hi}; group 0 writes, group 1
-  // (same warp & 7 -> same tid) shares them ----
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(tma::smem_addr(&tmem_base)),
-                 "r"(kTmemCols));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
+  double* sR = base + grp * 2 * PLANE;
+  double* sI = sR + PLANE;
+  if (threadIdx.x == 0) {
+    tma::mbar_init(&bar[0], 1);
+    tma::mbar_init(&bar[1], 1);
   }
-  asm volatile("tcgen05.fence::before_thread_sync;\n");
+  for (int e = threadIdx.x; e < PLANE; e += 2 * NT) stc(sS, 2 * e, __ldg(a.Sre + e), __ldg(a.Sim + e));   // once per launch
   __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;\n");
-  const uint32_t tmem_s = tmem_base + ((uint32_t)(32 * (warp & 3)) << 16) + 64 * ((warp >> 2) & 1);
-  if (grp == 0) {
-#pragma unroll 1
-    for (int q = 0; q < 4; ++q) {
-      uint32_t v[16];
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int k0 = 4 * q + e;
-        const double re = __ldg(a.Sre + (k0 << 8) + tid), im = __ldg(a.Sim + (k0 << 8) + tid);
-        v[4 * e] = (uint32_t)__double2loint(re);
-        v[4 * e + 1] = (uint32_t)__double2hiint(re);
-        v[4 * e + 2] = (uint32_t)__double2loint(im);
-        v[4 * e + 3] = (uint32_t)__double2hiint(im);
-      }
-      tmem_st16(tmem_s + 16 * q, v);
-    }
-    asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;\n");
-  __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;\n");
-
-  const int64_t pb = a.win.p_begin + 2 * (int64_t)blockIdx.x, gstride = 2 * (int64_t)gridDim.x;
-  auto pair_of = [&](int64_t j) { return pb + (j & 1) + (j >> 1) * gstride; };
-  auto issue = [&](int64_t j) {   // pair j's boxes into buffer j % 3
-    const int64_t p = pair_of(j);
-    if (p >= a.win.p_end) return;
+  const int64_t stride = 2 * (int64_t)gridDim.x;
+  const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
+  auto issue = [&](int64_t p) {
     const PairGeom g = pair_geom(a, p);
-    double* dR = base + (int)(j % 3) * 2 * PLANE;
-    uint64_t* bar = &full[j % 3];
-    tma::mbar_expect_tx(bar, (g.has_b ? 2u : 1u) * PLANE * 8u);
-    tma::load_3d(dR, &tm, (int)g.oa2, (int)g.o1, (int)(g.o0 - a.win.g0), bar);
-    if (g.has_b) tma::load_3d(dR + PLANE, &tm, (int)g.ob2, (int)g.o1, (int)(g.o0 - a.win.g0), bar);
+    tma::mbar_expect_tx(&bar[grp], (g.has_b ? 2u : 1u) * PLANE * 8u);
+    tma::load_3d(sR, &tm, (int)g.oa2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
+    if (g.has_b) tma::load_3d(sI, &tm, (int)g.ob2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
   };
-  if (TMA && threadIdx.x == 0)
-    for (int j = 0; j < 3; ++j) issue(j);
+  if (TMA && tid == 0 && p0 < a.win.p_end) issue(p0);
 
-  for (int64_t j = grp; pair_of(j) < a.win.p_end; j += 2) {
-    const int64_t p = pair_of(j);
+  uint32_t parity = 0;
+  for (int64_t p = p0; p < a.win.p_end; p += stride) {
     const PairGeom g = pair_geom(a, p);
-    double* sR = base + (TMA ? (int)(j % 3) : grp) * 2 * PLANE;
-    double* sI = sR + PLANE;
     if (TMA) {
-      tma::mbar_wait(&full[j % 3], (uint32_t)((j / 3) & 1));
+      tma::mbar_wait(&bar[grp], parity);
+      parity ^= 1;
       if (!g.has_b) {
         for (int e = tid; e < PLANE; e += NT) sI[e] = 0.0;
         group_sync(grp);
       }
     } else {
-      group_sync(grp);   // the group's previous pair has left the buffer
       for (int e = tid; e < 2 * PLANE; e += NT) {
         const int t = e >> 12, l0 = (e >> 8) & 15, l1 = (e >> 4) & 15, l2 = e & 15;
         int64_t g0 = g.o0 + l0, g1 = g.o1 + l1, g2 = (t ? g.ob2 : g.oa2) + l2;
@@ -232,12 +172,9 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
       }
       radix::fft16<false>(xr, xi);
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        uint32_t v[16];
-        tmem_ld16(tmem_s + 16 * q, v);
-#pragma unroll
-        for (int e = 0; e < 4; ++e)
-          radix::cmul(xr[4 * q + e], xi[4 * q + e], u2d(v[4 * e], v[4 * e + 1]), u2d(v[4 * e + 2], v[4 * e + 3]));
+      for (int k0 = 0; k0 < 16; ++k0) {
+        const double2 sv = ldc(sS, ((k0 << 8) + tid) << 1);
+        radix::cmul(xr[k0], xi[k0], sv.x, sv.y);
       }
       radix::fft16<true>(xr, xi);
 #pragma unroll
@@ -275,7 +212,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     // refill it while the last transform and the stores run
     if (TMA) tma::fence_proxy_async();
     group_sync(grp);
-    if (TMA && tid == 0) issue(j + 3);
+    if (TMA && tid == 0 && p + stride < a.win.p_end) issue(p + stride);
     if (p5) {
       const int l0 = h + hi, l1 = h + lo;
       radix::fft16<true>(xr, xi);
@@ -305,15 +242,11 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
       }
     }
   }
-  asm volatile("tcgen05.fence::before_thread_sync;\n");
-  __syncthreads();
-  asm volatile("tcgen05.fence::after_thread_sync;\n");
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem_base), "r"(kTmemCols));
 }
 
 }  // namespace
 
-// Three pair buffers (TMA ring; the cp.async path uses two of them); S_T is in tensor memory.
+// Two group buffers + S_T.
 size_t fused3d_bf_smem(bool) { return (size_t)6 * PLANE * sizeof(double) + kAlign; }
 
 cudaError_t fused3d_bf_configure(int* max_blocks) {
