@@ -122,16 +122,25 @@ __device__ __forceinline__ void dft4x4(double (&xr)[4][4], double (&xi)[4][4]) {
     dft4<INV>(xr[i][0], xi[i][0], xr[i][1], xi[i][1], xr[i][2], xi[i][2], xr[i][3], xi[i][3]);
 }
 
+// Shared twiddle table layout: w64^m sits at 16-byte word kTwPos[m], a permutation of 0..63
+// chosen (by a colouring search) so that the column twiddles w64^(cc i) of a quarter-warp
+// (cc = 8q..8q+7, i = 1, 2, 3) fall in eight different bank slots: with the natural layout
+// i = 2 hit four slots twice each (the 2-way conflicts ncu counted, ~8 % of the kernel's
+// shared-memory wavefronts).  The row twiddles w64^(rr i) are one address per
+// half-warp (broadcast).
+__constant__ unsigned char kTwPos[64] = {0, 2, 5, 4, 6, 3, 1, 7, 11, 13, 12, 8, 10, 9, 15, 14, 18, 16, 19, 24, 20, 23, 21, 32, 40, 48, 22, 26, 31, 56, 17, 25, 33, 27, 41, 49, 28, 57, 34, 29, 42, 50, 30, 58, 35, 39, 43, 51, 59, 36, 44, 52, 60, 37, 45, 53, 61, 38, 46, 54, 62, 47, 55, 63};
+
 // element [i][j] *= w64^(+-(rr i + cc j)) (conjugate if INV): a row and a column twiddle, all
-// six powers from the shared w64^m table.
+// six powers from the shared w64^m table (prow / pcol: the thread's table words of w64^(rr i) and
+// w64^(cc i), i = 1..3, looked up once per launch, one byte each).
 template <bool INV>
-__device__ __forceinline__ void twiddle4x4(double (&xr)[4][4], double (&xi)[4][4], const double2* tw, int rr,
-                                           int cc) {
+__device__ __forceinline__ void twiddle4x4(double (&xr)[4][4], double (&xi)[4][4], const double2* tw,
+                                           uint32_t prow, uint32_t pcol) {
   double2 pr[4], pc[4];
 #pragma unroll
-  for (int i = 1; i < 4; ++i) {
-    pr[i] = tw[(rr * i) & 63];
-    pc[i] = tw[(cc * i) & 63];
+  for (int i = 1; i < 4; ++i) {   // byte i - 1 of prow / pcol: the word of w64^(rr i) / w64^(cc i)
+    pr[i] = tw[(prow >> (8 * i - 8)) & 63];
+    pc[i] = tw[(pcol >> (8 * i - 8)) & 63];
   }
 #pragma unroll
   for (int i = 1; i < 4; ++i) {
@@ -207,7 +216,8 @@ __device__ __forceinline__ void block_store(double* sR, double* sI, int rr, int 
 template <bool TMA>
 __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double* sS, const double2* tw,
                                             const Fft2dArgs& a, const Geom& g, int warp, int lane, int grp,
-                                            const CUtensorMap* tm, uint64_t* bar, bool has_next, const Geom& gnext) {
+                                            const CUtensorMap* tm, uint64_t* bar, bool has_next, const Geom& gnext,
+                                            uint32_t prow, uint32_t pcol) {
   const int S = a.S, h = a.h;
   const int rr = (warp << 1) | (lane >> 4), cc = lane & 15;     // P1/P5 block classes
   const int rc = lane + ((warp & 1) << 5), blk = warp >> 1;      // P3 column, row block
@@ -218,7 +228,7 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
     double br[4][4], bi[4][4];
     load_block<true>(sR, sI, rr, cc, br, bi);
     dft4x4<false>(br, bi);
-    twiddle4x4<false>(br, bi, tw, rr, cc);
+    twiddle4x4<false>(br, bi, tw, prow, pcol);
     block_store(sR, sI, rr, cc, br, bi);
   }
   // ---- P2: axis 1, DFT-16 along row r2, block b2 ----
@@ -249,7 +259,7 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
   if (TMA) tma::fence_proxy_async();   // the buffer is refilled by TMA after the barrier
   group_sync(grp);
   if (TMA && warp == 0 && lane == 0 && has_next) issue_pair(a, tm, gnext, sR, bar);
-  twiddle4x4<true>(br, bi, tw, rr, cc);
+  twiddle4x4<true>(br, bi, tw, prow, pcol);
   dft4x4<true>(br, bi);
   // column predicates once per pass (valid window [h, h + S), grid limit, tile b present), in
   // 32-bit arithmetic: every column coordinate and limit is < 2^31 (plan: extents < 2^31)
@@ -294,7 +304,17 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
     tma::mbar_init(&bar[0], 1);
     tma::mbar_init(&bar[1], 1);
   }
-  if (threadIdx.x < L) tw[threadIdx.x] = make_double2(a.Fre[threadIdx.x], a.Fim[threadIdx.x]);
+  if (threadIdx.x < L) tw[kTwPos[threadIdx.x]] = make_double2(a.Fre[threadIdx.x], a.Fim[threadIdx.x]);
+  // table words of this thread's P1/P5 twiddles (rr, cc as in tile_passes), one byte per power
+  uint32_t prow = 0, pcol = 0;
+  {
+    const int rr = (warp << 1) | (lane >> 4), cc = lane & 15;
+#pragma unroll
+    for (int i = 1; i < 4; ++i) {
+      prow |= (uint32_t)kTwPos[(rr * i) & 63] << (8 * i - 8);
+      pcol |= (uint32_t)kTwPos[(cc * i) & 63] << (8 * i - 8);
+    }
+  }
   for (int e = threadIdx.x; e < PLANE; e += 2 * NT)   // once per launch
     *reinterpret_cast<double2*>(sS + 2 * e) = make_double2(__ldg(a.Sre + e), __ldg(a.Sim + e));
   __syncthreads();
@@ -327,7 +347,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
     }
     const bool has_next = p + stride < a.win.p_end;
     const Geom gnext = geom(a, has_next ? p + stride : p);
-    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gnext);
+    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gnext, prow, pcol);
   }
 }
 

@@ -75,3 +75,39 @@ def test_alu_peak_between_opcode_rates():
     for mix in bench.ALU_KERNEL_MIX.values():
         p = bench.alu_peak_tops(mix)
         assert min(bench.FP64_RATES_TOPS.values()) < p < max(bench.FP64_RATES_TOPS.values())
+
+
+def test_default_workloads_and_per_config_cover_baseline():
+    """N = 1 headline = the largest single-GPU BASELINE config (Heat-3D 1024^3, configs[3]);
+    N > 1 = configs[4]'s weak slab; every BASELINE config appears in the per_config list."""
+    assert bench.default_workload(1) == "heat3d"
+    assert all(bench.default_workload(n) == "heat3d_weak" for n in (2, 4, 8))
+    labels = {lab.split()[0] for _, _, _, lab in bench.PER_CONFIG}
+    assert {"configs[0]", "configs[1]", "configs[2]", "configs[3]", "configs[4]"} <= labels
+    names = {n for n, *_ in bench.PER_CONFIG}
+    for n in names:
+        assert n in wl.CONFIGS
+    # configs[1]'s T sweep covers 1..16 for both stencils
+    sweep = {(n, t) for n, t, _, lab in bench.PER_CONFIG if "sweep" in lab}
+    assert {t for _, t in sweep} >= {1, 2, 4, 8, 16}
+
+
+def test_gpus_without_torchrun_relaunches(monkeypatch):
+    """`bench.py --gpus N > 1` outside torch.distributed re-executes itself under
+    torch.distributed.run with N ranks on 127.0.0.1 (it must not silently measure one GPU)."""
+    import subprocess
+    calls = []
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    monkeypatch.setattr(subprocess, "call", lambda cmd: calls.append(cmd) or 0)
+    assert bench.main(["--gpus", "4", "--steps", "2"]) == 0
+    (cmd,) = calls
+    assert "torch.distributed.run" in cmd and "--nproc-per-node=4" in cmd and "--master-addr=127.0.0.1" in cmd
+    assert cmd[-3:] == ["--gpus", "4", "--steps", "2"][-3:]
+
+
+def test_world_size_mismatch_is_an_error(monkeypatch):
+    import pytest
+    monkeypatch.setenv("WORLD_SIZE", "2")
+    monkeypatch.setenv("RANK", "0")
+    with pytest.raises(SystemExit):
+        bench.main(["--gpus", "4"])
