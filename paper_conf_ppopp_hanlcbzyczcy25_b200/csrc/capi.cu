@@ -44,6 +44,11 @@ int env_algo() {
 }
 
 void set_error(const std::string& s) { g_last_error = s; }
+
+int env_int(const char* name, int dflt) {
+  const char* v = std::getenv(name);
+  return v && *v ? std::atoi(v) : dflt;
+}
 void clear_error() { g_last_error.clear(); }
 
 }  // namespace
@@ -86,6 +91,7 @@ struct fftstencil_plan {
   cudaStream_t band_stream = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_band = nullptr;
   bool band_pending = false;
+
   int64_t band_clip_lo = 0, band_clip_hi = INT64_MAX;   // outer rows the band pass produces
   // ---- pipelined run_host: chunked H2D / D2H on their own stream (FFTSTENCIL_E2E_PIPE) ----
   cudaStream_t copy_stream = nullptr;
@@ -231,6 +237,8 @@ void prof_end(fftstencil_plan* p, long i, cudaStream_t s) {
   if (i >= 0) cudaEventRecord(p->ev_pool[(size_t)i + 1], s);
 }
 
+int band_args(const fftstencil_plan* p, const double* src, double* dst, int t, BandArgs& b);
+
 // One fused launch over pairs [pb, pe): src -> dst with t steps (t <= T), tile geometry of
 // T.  The buffers hold global outer rows [g0, g1); only rows [row_lo, row_hi) are written.
 int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int64_t pb, int64_t pe,
@@ -373,8 +381,9 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
 // The band pass of one fused pass.  Concurrent mode: forked from `s` (after everything
 // already enqueued there, i.e. after the pass that produced `src`) onto the band stream;
 // band_join() makes `s` wait for it before the next pass touches either buffer.
-int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s,
-                     bool forked = false) {
+// The band blocks of one pass (rows [band_clip_lo, band_clip_hi) when clipped: the pipelined
+// run_host) as kernel arguments; returns the number of blocks.
+int band_args(const fftstencil_plan* p, const double* src, double* dst, int t, BandArgs& b) {
   const HostPlan& hp = p->hp;
   int64_t i0 = 0, i1 = (int64_t)(hp.band_blocks.size() / 8);
   if (p->band_clip_lo > 0 || p->band_clip_hi < INT64_MAX) {   // blocks meeting the clip rows
@@ -382,8 +391,6 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
     i1 = std::lower_bound(p->blk_lo.begin(), p->blk_lo.end(), p->band_clip_hi) - p->blk_lo.begin();
   }
   const int nb = (int)std::max<int64_t>(0, i1 - i0);
-  if (nb == 0) return FFTSTENCIL_OK;
-  BandArgs b;
   b.src = src;
   b.dst = dst;
   for (int q = 0; q < 3; ++q) { b.n[q] = hp.n[q]; b.active[q] = q >= 3 - hp.ndim; }
@@ -401,6 +408,13 @@ int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, 
   for (double wv : hp.w) b.ntaps += wv != 0.0;
   b.clip_lo = p->band_clip_lo;
   b.clip_hi = p->band_clip_hi;
+  return nb;
+}
+
+int launch_band_pass(fftstencil_plan* p, const double* src, double* dst, int t, cudaStream_t s,
+                     bool forked = false) {
+  BandArgs b;
+  if (band_args(p, src, dst, t, b) == 0) return FFTSTENCIL_OK;
   cudaStream_t bs = s;
   if (p->band_concurrent && !forked) {
     cudaError_t e = cudaEventRecord(p->ev_fork, s);
@@ -1131,14 +1145,16 @@ static int copy_ring_rows(fftstencil_plan* p, const double* src, double* d0, dou
   return FFTSTENCIL_OK;
 }
 
-static int env_int(const char* name, int dflt) {
-  const char* v = std::getenv(name);
-  return v && *v ? std::atoi(v) : dflt;
-}
 
 // K, Q of the pipelined schedule; K = 0: disabled (the caller runs H2D, fftstencil_run, D2H).
+// Default K: one input chunk per ~700 MB, 6..12 chunks -- the first H2D chunk and the last D2H
+// chunk cannot overlap anything, so big grids want more chunks, but every chunk adds partial
+// launches (measured: Heat-2D 839 MB K = 6 / 12 -> 90.4 / 93.5 ms per e2e step; Heat-3D 8.6 GB
+// K = 6 / 12 / 24 -> 586 / 569 / 575 ms, profiles/r02_e2e_chunks.txt).
 static int pipe_chunks(const fftstencil_plan* p) {
-  const int K = env_int("FFTSTENCIL_E2E_PIPE", 6);   // 0 disables; else the number of row chunks
+  const double gb = (double)p->grid_cells * sizeof(double) / 7e8;
+  const int dflt = (int)std::min(12.0, std::max(6.0, std::floor(gb + 0.5)));
+  const int K = env_int("FFTSTENCIL_E2E_PIPE", dflt);   // 0 disables; else the number of row chunks
   return p->dist || p->small1d ? 0 : K;
 }
 
@@ -1227,6 +1243,7 @@ static int run_host_pipelined_ops(fftstencil_plan* p, const double* h_in, double
     const int t = k <= nfull ? T : rem;
     const double* src = k == 1 ? in : dsts[(k - 2) % 2];
     double* dst = dsts[(k - 1) % 2];
+
     // fork the band first (it needs only what `s` holds so far), launch the fused tiles on all
     // but `reserve` SMs, then the band: its latency-bound CTAs (t sequential steps) run beside
     // the fused CTAs on the reserved SMs instead of after them

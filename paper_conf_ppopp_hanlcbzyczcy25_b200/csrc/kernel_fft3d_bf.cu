@@ -119,8 +119,12 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
   };
   if (TMA && tid == 0 && p0 < a.win.p_end) issue(p0);
 
+  // iteration count form of the pair loop (measured ~1-2 % faster than `for (p = p0; p < end;
+  // p += stride)`, same work: the compiler schedules the counted loop better)
+  const int64_t nmine = p0 < a.win.p_end ? (a.win.p_end - p0 + stride - 1) / stride : 0;
   uint32_t parity = 0;
-  for (int64_t p = p0; p < a.win.p_end; p += stride) {
+  for (int64_t it = 0; it < nmine; ++it) {
+    const int64_t p = p0 + it * stride;
     const PairGeom g = pair_geom(a, p);
     if (TMA) {
       tma::mbar_wait(&bar[grp], parity);

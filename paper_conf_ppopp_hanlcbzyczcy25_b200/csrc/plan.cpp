@@ -80,8 +80,17 @@ static constexpr double kEffCt = 0.83;
 // the 256 that transform it: P1 and P5 eight DFT-4 (128 adds) + 24 complex twiddle multiplies
 // (96 instr., 144 flops); P2 and P4 one DFT-16 (160 instr., 168 flops); P3 two DFT-16 + 16
 // spectrum multiplies (384 instr., 432 flops) -- independent of S (no crop before the stores).
-static constexpr int kP15Instr2d = 224;
-static constexpr int kP15Flops2d = 272;
+// BF_TW_REG (ablation, kernel_fft2d_bf.cu): P1 and P5 also form the squares and cubes of the
+// two twiddle bases (16 instr., 22 flops per pass; measured 1% slower than table loads).
+// BF_TW_COMB (default 0): one combined twiddle per element, 15 instead of 24 multiplies.
+#ifndef BF_TW_REG
+#define BF_TW_REG 0
+#endif
+#ifndef BF_TW_COMB
+#define BF_TW_COMB 0
+#endif
+static constexpr int kP15Instr2d = BF_TW_COMB ? 128 + 60 : 224 + (BF_TW_REG ? 16 : 0);
+static constexpr int kP15Flops2d = BF_TW_COMB ? 128 + 90 : 272 + (BF_TW_REG ? 22 : 0);
 static double flops_pair_2d_bf(int) { return 256.0 * (2 * kP15Flops2d + 2 * 168 + 432); }
 static double alu_ops_2d_bf(int) { return 256.0 * (2 * kP15Instr2d + 2 * 160 + 384); }
 static double model_flops_2d_bf(int S, int T) { return flops_pair_2d_bf(S) / (2.0 * S * (double)S * T); }

@@ -38,19 +38,35 @@ def test_smem_wavefront_model():
 
 
 def _sass_mix(obj):
-    """(DADD, DMUL, DFMA) static counts of the TMA instantiation (<true, false>) in `obj`."""
+    """(DADD, DMUL, DFMA) static counts of the TMA instantiation (<true, false>) in `obj`,
+    without the band-folding subroutine (the CALL right before the kernel's final EXIT, up to
+    its RET): the mix weights the FP64 peak of the tile passes, which is what bench.py reports."""
     import re
     import subprocess
     out = subprocess.run(["cuobjdump", "-sass", obj], capture_output=True, text=True).stdout
-    counts = {"DADD": 0, "DMUL": 0, "DFMA": 0}
-    inside = False
+    lines, inside = [], False
     for ln in out.splitlines():
         if "Function" in ln:
             inside = "ILb1ELb0E" in ln
             continue
-        if inside:
-            for m in re.finditer(r"\b(DADD|DMUL|DFMA)\b", ln):
-                counts[m.group(1)] += 1
+        m = re.match(r"\s*/\*([0-9a-f]+)\*/\s+(.*)", ln)
+        if inside and m:
+            lines.append((int(m.group(1), 16), m.group(2)))
+    skip = None
+    for k, (addr, txt) in enumerate(lines):
+        if re.match(r"EXIT\b", txt):                     # the kernel's final, unconditional EXIT
+            call = next((t for _, t in reversed(lines[max(0, k - 4):k]) if "CALL" in t), None)
+            if call:
+                lo = int(re.search(r"0x([0-9a-f]+)", call).group(1), 16)
+                hi = next(a for a, t in lines if a > lo and t.startswith("RET"))
+                skip = (lo, hi)
+            break
+    counts = {"DADD": 0, "DMUL": 0, "DFMA": 0}
+    for addr, txt in lines:
+        if skip and skip[0] <= addr <= skip[1]:
+            continue
+        for mm in re.finditer(r"\b(DADD|DMUL|DFMA)\b", txt):
+            counts[mm.group(1)] += 1
     return counts["DADD"], counts["DMUL"], counts["DFMA"]
 
 
