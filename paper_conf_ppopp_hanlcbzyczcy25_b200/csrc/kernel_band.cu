@@ -129,35 +129,53 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
   }
   if (hi[a.oax] <= lo[a.oax]) return;   // block outside the clip rows (whole CTA)
   const int r = a.r, wd = 2 * r + 1;
-  if (threadIdx.x == 0) {
-    int n = 0;
-    const int nw = (a.active[0] ? wd : 1) * (a.active[1] ? wd : 1) * (a.active[2] ? wd : 1);
-    int k = 0;
-    for (int o0 = a.active[0] ? -r : 0; o0 <= (a.active[0] ? r : 0); ++o0)
-      for (int o1 = a.active[1] ? -r : 0; o1 <= (a.active[1] ? r : 0); ++o1)
-        for (int o2 = a.active[2] ? -r : 0; o2 <= (a.active[2] ? r : 0); ++o2, ++k) {
-          const double wv = a.w[k];
-          if (wv != 0.0 && n < kMaxTaps) {
-            s_off[n] = (o0 * D[1] + o1) * D[2] + o2;
-            s_w[n] = wv;
-            ++n;
-          }
+  // Tap table: the nonzero weights in offset-cube order (the summation order of every cell, so
+  // results stay bitwise equal to the reference band kernel) with their flattened region
+  // offsets.  Warp 0 builds it 32 weights at a time (ballot + prefix count): one thread's loop
+  // of dependent global loads cost microseconds per block, and a 3D band is tens of thousands
+  // of small blocks (profiles/r02_band3d.txt).
+  const int W1 = a.active[1] ? wd : 1, W2 = a.active[2] ? wd : 1;
+  const int nw = (a.active[0] ? wd : 1) * W1 * W2;
+  if (threadIdx.x < 32) {
+    const int lane = threadIdx.x;
+    int base = 0;
+    for (int k0 = 0; k0 < nw; k0 += 32) {
+      const int k = k0 + lane;
+      const double wv = k < nw ? a.w[k] : 0.0;
+      const unsigned m = __ballot_sync(0xffffffffu, wv != 0.0);
+      if (wv != 0.0) {
+        const int pos = base + __popc(m & ((1u << lane) - 1u));
+        if (pos < kMaxTaps) {
+          const int i2 = k % W2, i1 = (k / W2) % W1, i0 = k / (W1 * W2);
+          const int o0 = a.active[0] ? i0 - r : 0, o1 = a.active[1] ? i1 - r : 0, o2 = a.active[2] ? i2 - r : 0;
+          s_off[pos] = (o0 * D[1] + o1) * D[2] + o2;
+          s_w[pos] = wv;
         }
-    s_ntaps = n;
-    (void)nw;
+      }
+      base += __popc(m);
+    }
+    if (lane == 0) s_ntaps = min(base, kMaxTaps);
   }
   const int vol = D[0] * D[1] * D[2];
   double* b0 = sb;
   double* b1 = sb + vol;
-  const int rows = D[0] * D[1];
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5, ny = NTH / 32;
-  for (int row = ty; row < rows; row += ny) {
-    const int i0 = row / D[1], i1 = row - i0 * D[1];
-    const double* src = a.src + ((rl[0] + i0 - off[0]) * a.n[1] + (rl[1] + i1 - off[1])) * a.n[2] + (rl[2] - off[2]);
-    for (int i2 = tx; i2 < D[2]; i2 += 32) {
-      const double v = src[i2];
-      b0[row * D[2] + i2] = v;
-      if (BAND_LEAN) b1[row * D[2] + i2] = v;   // the fixed ring lives in both buffers
+  {
+    // region load, flattened over all threads (thin faces have rows of a few cells: a warp per
+    // row left most lanes idle); (i0, i1, i2) advanced by carries
+    const int D12 = D[1] * D[2];
+    int i0 = threadIdx.x / D12, i1 = (threadIdx.x - i0 * D12) / D[2], i2 = threadIdx.x - i0 * D12 - i1 * D[2];
+    const int d0 = NTH / D12, d1 = (NTH - d0 * D12) / D[2], d2 = NTH - d0 * D12 - d1 * D[2];
+    const double* src0 = a.src + ((rl[0] - off[0]) * a.n[1] + (rl[1] - off[1])) * a.n[2] + (rl[2] - off[2]);
+    for (int e = threadIdx.x; e < vol; e += NTH) {
+      const double v = src0[((int64_t)i0 * a.n[1] + i1) * a.n[2] + i2];
+      b0[e] = v;
+      if (BAND_LEAN) b1[e] = v;   // the fixed ring lives in both buffers
+      i2 += d2;
+      i1 += d1;
+      i0 += d0;
+      if (i2 >= D[2]) { i2 -= D[2]; ++i1; }
+      if (i1 >= D[1]) { i1 -= D[1]; ++i0; }
     }
   }
   __syncthreads();
@@ -288,14 +306,24 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
     __syncthreads();
     double* t = b0; b0 = b1; b1 = t;
   }
+  // output store, flattened like the load (a face block of axis 2 has one-cell rows)
   const int O0 = (int)(hi[0] - lo[0]), O1 = (int)(hi[1] - lo[1]), O2 = (int)(hi[2] - lo[2]);
-  for (int row = ty; row < O0 * O1; row += ny) {
-    const int j0 = row / O1, j1 = row - j0 * O1;
-    const int64_t c0 = lo[0] + j0, c1 = lo[1] + j1;
-    double* dst = a.dst + ((c0 - off[0]) * a.n[1] + (c1 - off[1])) * a.n[2] + (lo[2] - off[2]);
-    const double* srow = b0 + ((c0 - rl[0]) * D[1] + (c1 - rl[1])) * D[2] + (lo[2] - rl[2]);
-    for (int j2 = tx; j2 < O2; j2 += 32) dst[j2] = srow[j2];
+  const int O12 = O1 * O2, ovol = O0 * O12;
+  int j0 = threadIdx.x / O12, j1 = (threadIdx.x - j0 * O12) / O2, j2 = threadIdx.x - j0 * O12 - j1 * O2;
+  const int f0 = NTH / O12, f1 = (NTH - f0 * O12) / O2, f2 = NTH - f0 * O12 - f1 * O2;
+  double* dst0 = a.dst + ((lo[0] - off[0]) * a.n[1] + (lo[1] - off[1])) * a.n[2] + (lo[2] - off[2]);
+  const double* sb0 = b0 + ((lo[0] - rl[0]) * D[1] + (lo[1] - rl[1])) * D[2] + (lo[2] - rl[2]);
+  for (int e = threadIdx.x; e < ovol; e += NTH) {
+    dst0[((int64_t)j0 * a.n[1] + j1) * a.n[2] + j2] = sb0[(j0 * D[1] + j1) * D[2] + j2];
+    j2 += f2;
+    j1 += f1;
+    j0 += f0;
+    if (j2 >= O2) { j2 -= O2; ++j1; }
+    if (j1 >= O1) { j1 -= O1; ++j0; }
   }
+  (void)tx;
+  (void)ty;
+  (void)ny;
 }
 
 __global__ void box_copy_kernel(const BoxCopyArgs a) {
