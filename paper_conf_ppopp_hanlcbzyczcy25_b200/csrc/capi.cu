@@ -753,6 +753,11 @@ int setup_device(fftstencil_plan* p) {
     p->fused_grid = (int)std::max<int64_t>(1, p->fused_grid - (int64_t)(hp.band_blocks.size() / 8));
   if (const char* v = std::getenv("FFTSTENCIL_MAX_CTAS")) p->max_ctas = std::max(0, std::atoi(v));
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
+  // 3D: the band (tens of thousands of small blocks) runs before the fused kernel on the run
+  // stream -- concurrently, its CTAs hold SMs the register-full fused CTAs then wait for
+  // (Heat-3D 224.1 concurrent vs 228.1 serialised, profiles/r02_band3d.txt); 2D keeps the side
+  // stream (its band is ~45 us and hides in the fused kernel's tail: 1326 vs 1300)
+  if (hp.ndim == 3) p->band_concurrent = false;
   if (const char* v = std::getenv("FFTSTENCIL_BAND_STREAM")) p->band_concurrent = std::atoi(v) != 0;
   if (hp.band_blocks.empty()) p->band_concurrent = false;
   if (p->band_concurrent) {

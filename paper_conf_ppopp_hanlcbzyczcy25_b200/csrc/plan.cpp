@@ -614,7 +614,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
   // per buffer (still 6 CTAs per SM, bound by registers) recompute less halo per band cell and
   // fit the 10240^2 band into about one wave (Heat-2D +1.5%; 3D measured best at 1536,
   // profiles/r01_s3_ab_band_budget.txt).  FFTSTENCIL_BAND_BUDGET overrides (cells per buffer).
-  int budget_cells = p.engine == 1 && p.ndim == 2 ? 2240 : 1536;
+  // cells per band block buffer: 2240 for 2D ALU plans (profiles/r01_s3_ab_band_budget.txt), 4608
+  // for 3D ALU plans (fewer, larger blocks once the block setup is cheap: band alone 0.40 ->
+  // 0.26 ms per Heat-3D pass, profiles/r02_band3d.txt), 1536 otherwise
+  int budget_cells = p.engine == 1 && p.ndim == 2 ? 2240 : p.engine == 1 && p.ndim == 3 ? 4608 : 1536;
   if (const char* v = std::getenv("FFTSTENCIL_BAND_BUDGET")) budget_cells = std::max(256, std::atoi(v));
   const int grow = 2 * r * p.T;
   for (const Box& b : p.band_boxes) {
