@@ -690,20 +690,29 @@ int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std
       }
     }
   };
+  // Chunk boundaries (outer tile rows): K regular chunks, with the FIRST input chunk and the LAST
+  // output chunk split 1/4 + 3/4 -- nothing overlaps the first H2D chunk or the last D2H chunk,
+  // so those two are the small ones (Heat-2D: 2 x 2.4 ms exposed copies at K = 6 -> 2 x 0.6 ms).
+  const int64_t q4 = std::max<int64_t>(1, U / (4 * (int64_t)K));
+  std::vector<int64_t> ib{0, q4}, ob{0};
+  for (int c = 1; c <= K; ++c) ib.push_back(U * c / K);
+  for (int j = 1; j < K; ++j) ob.push_back(U * j / K);
+  ob.push_back(U - q4);
+  ob.push_back(U);
   // head: input chunk c, its ring rows, then the first Q passes advance behind it
-  for (int c = 1; c <= K; ++c) {
-    const int64_t y0 = row_of(U * (c - 1) / K), y1 = row_of(U * c / K);
+  for (size_t c = 1; c < ib.size(); ++c) {
+    const int64_t y0 = row_of(ib[c - 1]), y1 = row_of(ib[c]);
     push(0, y0, y1, 0);
     push(1, y0, y1, 0);
-    f[0] = U * c / K;
+    f[0] = ib[c];
     propagate([&](int64_t k) { return k <= Q ? U : (int64_t)0; });
   }
   // tail: the last Q passes advance until pass P holds chunk j, which is then copied out
-  for (int j = 1; j <= K; ++j) {
-    const int64_t bj = U * j / K;
+  for (size_t j = 1; j < ob.size(); ++j) {
+    const int64_t bj = ob[j];
     propagate([&](int64_t k) { return k <= P - Q ? U : std::min<int64_t>(U, bj + (P - k)); });
     if (f[(size_t)P] < bj) { ops.clear(); return FFTSTENCIL_EINVAL; }
-    push(3, row_of(U * (j - 1) / K), row_of(bj), 0);
+    push(3, row_of(ob[j - 1]), row_of(bj), 0);
   }
   return FFTSTENCIL_OK;
 }
