@@ -141,6 +141,7 @@ PER_CONFIG = [
     ("box3d27p", 0, 100, "configs[3]"),
     ("box2d9p_weak", 0, 1000, "configs[4] per-GPU slab, 1 GPU"),
     ("heat3d_weak", 0, 100, "configs[4] per-GPU slab, 1 GPU"),
+    ("heat1d_512m", 0, 1000, "PAPER.md Table 3 L332 size (context)"),
 ]
 
 
@@ -385,6 +386,17 @@ def roofline_of(info, prof, passes, exact_cells, workload):
     return roof
 
 
+def nccl_summary(path):
+    """A few facts from rank 0's NCCL_DEBUG=INFO log (communicator setup of the halo exchange)."""
+    try:
+        txt = open(path, errors="replace").read()
+    except OSError:
+        return {"log": path, "found": False}
+    return {"log": os.path.relpath(path, ROOT), "found": True, "init_complete": txt.count("Init COMPLETE"),
+            "nvls": "NVLS" in txt, "p2p_or_nvlink": ("P2P" in txt) or ("NVL" in txt),
+            "lines": txt.count("\n")}
+
+
 def exact_cells_of(info, gext):
     h = info["halo"]
     exact = max(0, min(info["row_end"], gext[0] - h) - max(info["row_begin"], h))   # this rank's exact rows
@@ -502,7 +514,14 @@ def main(argv=None):
     import torch.distributed as dist
     import paper_conf_ppopp_hanlcbzyczcy25_b200 as fs
 
+    nccl_log = None
     if world > 1:
+        # the library's own communicator (ncclCommInitRank in fftstencil_plan_create_dist) logs
+        # its setup -- transport, NVLS, channels -- to a file, so stdout keeps the one JSON line
+        nccl_log = os.path.join(ROOT, "gpurun_out", f"nccl_rank{rank}.log")
+        os.makedirs(os.path.dirname(nccl_log), exist_ok=True)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_FILE", nccl_log)
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
@@ -564,6 +583,8 @@ def main(argv=None):
             "clocks": main_res["clocks"],
             "per_config": per_config,
         }
+        if nccl_log:
+            line["config"]["nccl"] = nccl_summary(nccl_log)
         s = json.dumps(line)
         print(s, flush=True)
         if args.json_out:
