@@ -138,3 +138,29 @@ def test_signed_unnormalised_weights_grow(fs, ext, shape, r, T, steps):
     err = check(got, u0, w, r, steps, info)
     assert np.abs(got).max() > np.abs(u0).max(), "expected growth for max|sigma| > 1"
     assert err <= TOL
+
+
+# the selectable engines' persistent loops too (DMMA factored 2D / 3D / 1D, dense 2D with its
+# cp.async double buffer, dense 3D, PFA 1D): one CTA, so every CTA walks many pairs
+ENGINE_CAPPED = [
+    ((300, 290), "box", 1, 8, 19, {"FFTSTENCIL_ALGO": "factored", "FFTSTENCIL_ENGINE": "dmma"}),
+    ((300, 290), "box", 1, 8, 19, {"FFTSTENCIL_ALGO": "factored", "FFTSTENCIL_ENGINE": "dmma", "FFTSTENCIL_TMA": "0"}),
+    ((60, 50, 45), "star", 1, 2, 5, {"FFTSTENCIL_ALGO": "factored", "FFTSTENCIL_ENGINE": "dmma"}),
+    ((65536,), "star", 2, 512, 1100, {"FFTSTENCIL_ALGO": "factored", "FFTSTENCIL_ENGINE": "dmma"}),
+    ((260, 250), "star", 1, 8, 19, {"FFTSTENCIL_ALGO": "dense", "FFTSTENCIL_VARIANT": "1"}),
+    ((260, 250), "star", 1, 8, 19, {"FFTSTENCIL_ALGO": "dense", "FFTSTENCIL_VARIANT": "0"}),
+    ((60, 50, 45), "box", 1, 2, 5, {"FFTSTENCIL_ALGO": "dense"}),
+    ((3001,), "star", 1, 8, 21, {"FFTSTENCIL_SMALL1D": "0"}),
+]
+
+
+@pytest.mark.parametrize("ext,shape,r,T,steps,env", ENGINE_CAPPED)
+def test_capped_grid_other_engines(fs, monkeypatch, ext, shape, r, T, steps, env):
+    monkeypatch.setenv("FFTSTENCIL_MAX_CTAS", "1")
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    w = wl.seeded_weights(shape, len(ext), r)
+    u0 = wl.grid(ext, 7)
+    got, info = run(fs, u0, w, r, T, steps)
+    assert info["pair_end"] - info["pair_begin"] >= 8, info
+    check(got, u0, w, r, steps, info)
