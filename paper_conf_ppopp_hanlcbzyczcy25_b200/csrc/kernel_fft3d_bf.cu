@@ -71,11 +71,36 @@ struct PairGeom {
   int64_t o0, o1, oa2, ob2;
   bool has_b;
 };
+// p is the launch's traversal index in [p_begin, p_end) (whole outer tile rows): in natural order
+// it is the pair index itself; with blk0 > 0 the launch visits blocks of blk0 outer tile rows x
+// blk1 tile lines (all pairs of each line), block rows in order, so the tiles whose halo planes
+// / rows overlap are transformed close together in time and the overlap is re-read from L2 (a
+// 1024^3 outer tile row of 16-plane tiles is 134 MB, more than the 126 MB L2: in natural order the
+// next row's four overlapping planes come back from HBM).
 __device__ __forceinline__ PairGeom pair_geom(const Fft3dArgs& a, int64_t p) {
   // pair / tile indices fit 32 bits (the plan's pair count is far below 2^31)
-  const int S = a.S, npr = (int)a.npr, nt1 = (int)a.nt1, pi = (int)p;
-  const int line = pi / npr, pj = pi - line * npr;
-  const int t0 = line / nt1, t1 = line - t0 * nt1;
+  const int S = a.S, npr = (int)a.npr, nt1 = (int)a.nt1;
+  int t0, t1, pj;
+  if (a.blk0 > 0) {
+    const int ppu = nt1 * npr, u0 = (int)(a.win.p_begin / ppu), nu = (int)((a.win.p_end - a.win.p_begin) / ppu);
+    const int q = (int)(p - a.win.p_begin);
+    const int b0 = q / (a.blk0 * ppu);                       // block row (outer tile rows)
+    const int s0 = min(a.blk0, nu - b0 * a.blk0);            // its height (last one partial)
+    const int q1 = q - b0 * a.blk0 * ppu;
+    const int b1 = q1 / (s0 * a.blk1 * npr);                 // block within the row (tile lines)
+    const int s1 = min(a.blk1, nt1 - b1 * a.blk1);
+    const int q2 = q1 - b1 * s0 * a.blk1 * npr;
+    pj = q2 % npr;
+    const int r = q2 / npr;                                  // (t0, t1) within the block, t1 fastest
+    t0 = u0 + b0 * a.blk0 + r / s1;
+    t1 = b1 * a.blk1 + r % s1;
+  } else {
+    const int pi = (int)p;
+    const int line = pi / npr;
+    pj = pi - line * npr;
+    t0 = line / nt1;
+    t1 = line - t0 * nt1;
+  }
   PairGeom g;
   g.o0 = (int64_t)t0 * S + a.bd.shift;
   g.o1 = (int64_t)t1 * S + a.bd.shift;
@@ -111,13 +136,27 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
   __syncthreads();
   const int64_t stride = 2 * (int64_t)gridDim.x;
   const int64_t p0 = a.win.p_begin + 2 * (int64_t)blockIdx.x + grp;
-  auto issue = [&](int64_t p) {
+  // TMA box origins of a group's next pair (x = axis 2 of tile a, y, z, x of tile b or -1), computed
+  // by the issuing thread at the top of an iteration, when few registers are live: the refill is
+  // issued mid-transform, with the 32 line registers live
+  __shared__ int nxt[2][4];
+  auto prepare = [&](int64_t p) {
     const PairGeom g = pair_geom(a, p);
-    tma::mbar_expect_tx(&bar[grp], (g.has_b ? 2u : 1u) * PLANE * 8u);
-    tma::load_3d(sR, &tm, (int)g.oa2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
-    if (g.has_b) tma::load_3d(sI, &tm, (int)g.ob2, (int)g.o1, (int)(g.o0 - a.win.g0), &bar[grp]);
+    nxt[grp][0] = (int)g.oa2;
+    nxt[grp][1] = (int)g.o1;
+    nxt[grp][2] = (int)(g.o0 - a.win.g0);
+    nxt[grp][3] = g.has_b ? (int)g.ob2 : INT32_MIN;
   };
-  if (TMA && tid == 0 && p0 < a.win.p_end) issue(p0);
+  auto issue = [&]() {
+    const int x = nxt[grp][0], y = nxt[grp][1], z = nxt[grp][2], xb = nxt[grp][3];
+    tma::mbar_expect_tx(&bar[grp], (xb != INT32_MIN ? 2u : 1u) * PLANE * 8u);
+    tma::load_3d(sR, &tm, x, y, z, &bar[grp]);
+    if (xb != INT32_MIN) tma::load_3d(sI, &tm, xb, y, z, &bar[grp]);
+  };
+  if (TMA && tid == 0 && p0 < a.win.p_end) {
+    prepare(p0);
+    issue();
+  }
 
   // iteration count form of the pair loop (measured ~1-2 % faster than `for (p = p0; p < end;
   // p += stride)`, same work: the compiler schedules the counted loop better)
@@ -127,6 +166,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     const int64_t p = p0 + it * stride;
     const PairGeom g = pair_geom(a, p);
     if (TMA) {
+      if (tid == 0 && p + stride < a.win.p_end) prepare(p + stride);
       tma::mbar_wait(&bar[grp], parity);
       parity ^= 1;
       if (!g.has_b) {
@@ -216,7 +256,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
     // refill it while the last transform and the stores run
     if (TMA) tma::fence_proxy_async();
     group_sync(grp);
-    if (TMA && tid == 0 && p + stride < a.win.p_end) issue(p + stride);
+    if (TMA && tid == 0 && p + stride < a.win.p_end) issue();
     if (p5) {
       const int l0 = h + hi, l1 = h + lo;
       radix::fft16<true>(xr, xi);

@@ -88,6 +88,10 @@ struct Fft3dArgs {
   const double* Fim;
   const double* Sre;     // powered spectrum in [k1][k2][k0] order
   const double* Sim;
+  // ALU kernel traversal order (kernel_fft3d_bf.cu pair_geom): blocks of blk0 outer tile rows x
+  // blk1 tile lines, so the axis-0 / axis-1 halo overlap of neighbouring tiles is re-read from L2
+  // instead of HBM; 0 = natural pair order.  Launch ranges are whole outer tile rows.
+  int blk0, blk1;
 };
 
 // Direct T-step recomputation of the boundary band (kernel_band.cu).
