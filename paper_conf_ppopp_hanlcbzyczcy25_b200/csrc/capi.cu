@@ -100,6 +100,7 @@ struct fftstencil_plan {
   std::vector<int64_t> blk_lo;   // outer-axis start of each band block (blocks sorted by it)
   int64_t blk_hmax = 0;          // tallest band block along the outer axis
   int grid_cap = 0;              // > 0: fused launches use at most this many CTAs
+  bool st256 = true;             // 3D ALU kernel: 32-byte output stores (FFTSTENCIL_ST256=0: 16-byte only)
   int trav_blk = 0;              // 3D ALU kernel traversal blocks (FFTSTENCIL_3D_TRAV=6: 6 x 6 tile lines; measured slower)
   int max_ctas = 0;              // FFTSTENCIL_MAX_CTAS (tests): cap on every fused launch's grid, so each
                                  // persistent CTA walks many pairs through its refill / mbarrier loop
@@ -359,6 +360,19 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     a.Sre = Sre;
     a.Sim = Sim;
     a.blk0 = a.blk1 = 0;
+    a.st32 = a.st16 = 0;
+    {
+      const bool al32 = (hp.S[0] % 4) == 0 && (hp.ext[2] % 4) == 0 && bd.shift % 4 == 0 &&
+                        (reinterpret_cast<uintptr_t>(dst) & 31) == 0 && p->st256;
+      for (int l2 = hp.h; l2 < hp.h + hp.S[0]; l2 += 2) {
+        if (al32 && (l2 & 3) == 0 && l2 + 4 <= hp.h + hp.S[0]) {
+          a.st32 |= 1 << l2;
+          l2 += 2;
+        } else {
+          a.st16 |= 1 << l2;
+        }
+      }
+    }
     if (hp.algo == 1 && hp.engine == 1 && !hp.periodic) {   // blocked traversal (kernel_fft3d_bf.cu)
       a.blk0 = a.blk1 = p->trav_blk;
       const int64_t ppu = hp.nt[1] * hp.npr;
@@ -760,6 +774,7 @@ int setup_device(fftstencil_plan* p) {
     p->fused_grid = (int)std::max<int64_t>(1, p->fused_grid - (int64_t)(hp.band_blocks.size() / 8));
   if (const char* v = std::getenv("FFTSTENCIL_MAX_CTAS")) p->max_ctas = std::max(0, std::atoi(v));
   if (const char* v = std::getenv("FFTSTENCIL_3D_TRAV")) p->trav_blk = std::max(0, std::atoi(v));
+  if (const char* v = std::getenv("FFTSTENCIL_ST256")) p->st256 = std::atoi(v) != 0;
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
   // 3D: the band (tens of thousands of small blocks) runs before the fused kernel on the run
   // stream -- concurrently, its CTAs hold SMs the register-full fused CTAs then wait for

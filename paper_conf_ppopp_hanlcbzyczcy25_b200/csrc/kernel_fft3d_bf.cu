@@ -67,6 +67,11 @@ __device__ __forceinline__ void stc(double* b, int o, double re, double im) {
 // Barrier of one 256-thread group (ids 1, 2; id 0 is __syncthreads).
 __device__ __forceinline__ void group_sync(int grp) { asm volatile("bar.sync %0, %1;\n" ::"r"(grp + 1), "r"(NT) : "memory"); }
 
+// 256-bit global store (sm_100): four doubles at a 32-byte aligned address, one whole sector.
+__device__ __forceinline__ void st256(double* p, double a, double b, double c, double d) {
+  asm volatile("st.global.v4.f64 [%0], {%1, %2, %3, %4};\n" ::"l"(p), "d"(a), "d"(b), "d"(c), "d"(d) : "memory");
+}
+
 struct PairGeom {
   int64_t o0, o1, oa2, ob2;
   bool has_b;
@@ -268,11 +273,15 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
                          g.oa2 + h + S <= a.bd.lim2 && (!g.has_b || g.ob2 + h + S <= a.bd.lim2);
         if (vec) {
 #pragma unroll
-          for (int l2 = 0; l2 < 16; l2 += 2)
-            if (l2 >= h && l2 < h + S) {
+          for (int l2 = 0; l2 < 16; l2 += 2) {
+            if ((a.st32 >> l2) & 1) {   // whole 32-byte sectors (launch mask, see Fft3dArgs)
+              st256(drow + g.oa2 + l2, xr[l2], xr[l2 + 1], xr[l2 + 2], xr[l2 + 3]);
+              if (g.has_b) st256(drow + g.ob2 + l2, xi[l2], xi[l2 + 1], xi[l2 + 2], xi[l2 + 3]);
+            } else if ((a.st16 >> l2) & 1) {
               *reinterpret_cast<double2*>(drow + g.oa2 + l2) = make_double2(xr[l2], xr[l2 + 1]);
               if (g.has_b) *reinterpret_cast<double2*>(drow + g.ob2 + l2) = make_double2(xi[l2], xi[l2 + 1]);
             }
+          }
         } else {
 #pragma unroll
           for (int l2 = 0; l2 < 16; ++l2)

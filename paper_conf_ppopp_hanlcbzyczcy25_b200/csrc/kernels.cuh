@@ -92,6 +92,10 @@ struct Fft3dArgs {
   // blk1 tile lines, so the axis-0 / axis-1 halo overlap of neighbouring tiles is re-read from L2
   // instead of HBM; 0 = natural pair order.  Launch ranges are whole outer tile rows.
   int blk0, blk1;
+  // ALU kernel output rows (vector path): bit l2 of st32 = 32-byte store of l2 .. l2 + 3, of st16 =
+  // 16-byte store of l2, l2 + 1, for l2 in [h, h + S).  launch_fused sets st32 only when every
+  // tile row starts 32-byte aligned (S, n2 multiples of 4, no shift, dst 32-byte aligned).
+  int st32, st16;
 };
 
 // Direct T-step recomputation of the boundary band (kernel_band.cu).

@@ -1,0 +1,9 @@
+# 3D ALU kernel: 32-byte (st.global.v4.f64) output stores vs 16-byte (FFTSTENCIL_ST256=0)
+timeout 900 python -m pytest -q -x -m gpu tests/test_gpu_parity.py tests/test_gpu_steady_state.py tests/test_gpu_e2e_pipe.py tests/test_gpu_dist.py -k "3d or heat3d or box3d" 2>&1 | tail -2
+run() {  # st256 workload
+  FFTSTENCIL_ST256=$1 timeout 300 python bench.py --workload $2 --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-per-config 2>/dev/null | tail -1 | python -c "import json,sys;d=json.loads(sys.stdin.read());r=d['roofline'];print('st256=$1 $2', round(d['value'],1), 'frac', round(r['frac'],3), 'fused_ms', round(r['fused_ms_avg'],4), 'ms/step', round(d['ms_per_step'],2), d['clocks']['sm_mhz'])"
+}
+for rep in 1 2; do for w in heat3d box3d27p; do run 0 $w; run 1 $w; done; done
+for b in 0 1; do
+  FFTSTENCIL_ST256=$b timeout 600 ncu --metrics gpu__time_duration.sum,l1tex__t_sectors_pipe_lsu_mem_global_op_st.sum,l1tex__t_requests_pipe_lsu_mem_global_op_st.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -k regex:fft3d_bf -s 1 -c 1 --csv python bench.py --workload heat3d --time-steps 6 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --no-per-config 2>/dev/null | grep -E "sectors|requests|dram|duration" | awk -F'","' '{print "ncu st256='$b'", $(NF-2), $NF}'
+done
