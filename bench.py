@@ -480,14 +480,15 @@ def measure(fs, torch, dist, dev, world, rank, name, T, time_steps, steps, warmu
         if world > 1:
             dist.all_reduce(ems, op=dist.ReduceOp.MAX)
         e_ms = float(ems.item())
-        piped = plan.info()["last_run_pipelined"]
+        pinfo = plan.info()
+        piped = pinfo["last_run_pipelined"]
         res["e2e"] = {"value": gstencils(cells, time_steps * k_e, e_ms), "unit": "GStencils/s",
                       "h2d_bytes_per_step": world * int(u0.nbytes), "d2h_bytes_per_step": world * int(u0.nbytes),
                       "steps": k_e, "ms_per_step": e_ms / k_e, "api": "fftstencil_run_host (pinned host buffers)",
                       "pipelined": piped,
                       "overlap": ("copies overlapped with row-skewed passes: "
-                                  f"K={os.environ.get('FFTSTENCIL_E2E_PIPE', '6')} row chunks, "
-                                  f"Q={os.environ.get('FFTSTENCIL_E2E_DEPTH', '16')} skewed passes (DESIGN.md §6)")
+                                  f"K={pinfo['last_run_chunks']} row chunks, "
+                                  f"Q={pinfo['last_run_depth']} skewed passes (DESIGN.md §6)")
                       if piped else "none: copy-run-copy (the plan does not take the pipelined schedule)"}
         if not np.isfinite(h_out.numpy()).all():
             raise RuntimeError("non-finite output")

@@ -101,6 +101,8 @@ typedef struct {
   int last_run_pipelined;       /* 1 if the last fftstencil_run_host overlapped its copies with
                                    row-skewed passes (pipelined schedule), 0 if it ran plain
                                    copy-run-copy (FFTSTENCIL_E2E_PIPE=0, 1D, small grids, h > S) */
+  int last_run_chunks;          /* that run's pipelined schedule: K input / output row chunks   */
+  int last_run_depth;           /*   and Q skewed passes at each end (0 / 0 when not pipelined) */
 } fftstencil_info;
 
 /* Plan creation flags (fftstencil_plan_create_ex / fftstencil_describe_ex). */

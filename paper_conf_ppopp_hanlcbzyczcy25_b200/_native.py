@@ -59,6 +59,8 @@ class Info(ctypes.Structure):
         ("engine", ctypes.c_int),
         ("alu_ops_per_pass", ctypes.c_double),
         ("last_run_pipelined", ctypes.c_int),
+        ("last_run_chunks", ctypes.c_int),
+        ("last_run_depth", ctypes.c_int),
     ]
 
     def as_dict(self) -> dict:
@@ -78,6 +80,7 @@ class Info(ctypes.Structure):
             "periodic": bool(self.periodic),
             "engine": ("dmma", "alu")[self.engine], "alu_ops_per_pass": self.alu_ops_per_pass,
             "last_run_pipelined": bool(self.last_run_pipelined),
+            "last_run_chunks": self.last_run_chunks, "last_run_depth": self.last_run_depth,
         }
 
 

@@ -78,6 +78,7 @@ struct fftstencil_plan {
   size_t band_smem = 0;
   int64_t last_launches = 0;
   bool last_pipelined = false;   // the last run_host took the pipelined schedule
+  int last_chunks = 0, last_depth = 0;   // and its K / Q
   // ---- decomposition (dist) ----
   bool dist = false;          // slab plan with halo buffers
   bool loopback = false;      // no communicator: run by fftstencil_run_group
@@ -1186,7 +1187,13 @@ static int pipe_chunks(const fftstencil_plan* p) {
   return p->dist || p->small1d ? 0 : K;
 }
 
-static int pipe_depth() { return std::max(1, env_int("FFTSTENCIL_E2E_DEPTH", 16)); }
+// Default Q: enough skewed passes at each end to cover one direction's copies (~49 GB/s each way
+// concurrently, measured): Heat-2D 10240^2 Q = 16 (sweep: 16 best, 20 -1 %, 12 -5 %), 3D 1024^3
+// Q = 20 (8.6 GB = 176 ms per direction vs 8.9 ms per pass: Q = 16 / 20 / 24 -> 530 / 514 / 516 ms
+// per e2e step, profiles/r02_e2e3d.txt).
+static int pipe_depth(const fftstencil_plan* p) {
+  return std::max(1, env_int("FFTSTENCIL_E2E_DEPTH", p->hp.ndim == 3 ? 20 : 16));
+}
 
 static int run_host_pipelined_ops(fftstencil_plan* p, const double* h_in, double* h_out,
                                   const std::vector<int64_t>& ops, int64_t total_steps, cudaStream_t caller,
@@ -1337,9 +1344,11 @@ int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, i
   const int K = pipe_chunks(p);
   std::vector<int64_t> ops;
   p->last_pipelined = false;
-  if (K && build_e2e_schedule(p->hp, total_steps, K, pipe_depth(), ops) == FFTSTENCIL_OK) {
+  if (K && build_e2e_schedule(p->hp, total_steps, K, pipe_depth(p), ops) == FFTSTENCIL_OK) {
     p->last_launches = 0;
     p->last_pipelined = true;
+    p->last_chunks = K;
+    p->last_depth = pipe_depth(p);
     rc = run_host_pipelined(p, h_in, h_out, ops, total_steps, (cudaStream_t)stream);
     // synchronise on success and on error (queued chunk copies still read / write the host buffers)
     if ((e = cudaStreamSynchronize(s)) != cudaSuccess && rc == FFTSTENCIL_OK) rc = cuda_fail(e, "stream synchronize");
@@ -1366,6 +1375,8 @@ int fftstencil_plan_info(const fftstencil_plan* p, fftstencil_info* info) {
   info->fused_grid = p->fused_grid;
   info->last_run_launches = p->last_launches;
   info->last_run_pipelined = p->last_pipelined ? 1 : 0;
+  info->last_run_chunks = p->last_pipelined ? p->last_chunks : 0;
+  info->last_run_depth = p->last_pipelined ? p->last_depth : 0;
   clear_error();
   return FFTSTENCIL_OK;
 }

@@ -15,6 +15,9 @@
 #ifndef BAND_LEAN
 #define BAND_LEAN 1   // 0: per-cell ring test and index recomputation (the session-2 loop)
 #endif
+#ifndef BAND_CPASYNC
+#define BAND_CPASYNC 1   // 0: synchronous region loads (round-2 kernel, ablation)
+#endif
 #ifndef BAND_TAPREG
 #define BAND_TAPREG 1   // 0: taps always read from shared memory (ablation)
 #endif
@@ -168,14 +171,29 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
     const int d0 = NTH / D12, d1 = (NTH - d0 * D12) / D[2], d2 = NTH - d0 * D12 - d1 * D[2];
     const double* src0 = a.src + ((rl[0] - off[0]) * a.n[1] + (rl[1] - off[1])) * a.n[2] + (rl[2] - off[2]);
     for (int e = threadIdx.x; e < vol; e += NTH) {
-      const double v = src0[((int64_t)i0 * a.n[1] + i1) * a.n[2] + i2];
-      b0[e] = v;
-      if (BAND_LEAN) b1[e] = v;   // the fixed ring lives in both buffers
+      const double* gp = src0 + ((int64_t)i0 * a.n[1] + i1) * a.n[2] + i2;
+      if (BAND_CPASYNC) {
+        // asynchronous 8-byte copies: a thread's ~14 region loads are all in flight at once
+        // (the synchronous loop waited one global-load latency per cell: ncu long_scoreboard)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"((unsigned)__cvta_generic_to_shared(b0 + e)),
+                     "l"(gp));
+      } else {
+        const double v = *gp;
+        b0[e] = v;
+        if (BAND_LEAN) b1[e] = v;   // the fixed ring lives in both buffers
+      }
       i2 += d2;
       i1 += d1;
       i0 += d0;
       if (i2 >= D[2]) { i2 -= D[2]; ++i1; }
       if (i1 >= D[1]) { i1 -= D[1]; ++i0; }
+    }
+    if (BAND_CPASYNC) {
+      asm volatile("cp.async.commit_group;\n" ::);
+      asm volatile("cp.async.wait_all;\n" ::: "memory");
+      // a thread's own copies are visible to it after the wait: the fixed ring goes to b1 too
+      if (BAND_LEAN)
+        for (int e = threadIdx.x; e < vol; e += NTH) b1[e] = b0[e];
     }
   }
   __syncthreads();

@@ -77,7 +77,10 @@ def test_pipelined_run_host_bitwise(fs, ext, shape, r, T, steps, K, Q):
         h_out = torch.full(u0.shape, np.nan, dtype=torch.float64).pin_memory()
         p.run_host(h_in.numpy(), h_out.numpy(), steps)
         n_pipe = p.info()["last_run_launches"]
-        assert p.info()["last_run_pipelined"]
+        pi = p.info()
+        assert pi["last_run_pipelined"]
+        # default Q (capi.cu pipe_depth): 20 skewed passes for 3D plans, 16 otherwise
+        assert (pi["last_run_chunks"], pi["last_run_depth"]) == (K, Q if Q is not None else (20 if len(ext) == 3 else 16))
         got = h_out.numpy().copy()
         # pageable host buffers take the same schedule
         out2 = np.full_like(u0, np.nan)
