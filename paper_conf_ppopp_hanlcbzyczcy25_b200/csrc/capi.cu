@@ -51,6 +51,14 @@ int env_int(const char* name, int dflt) {
 }
 void clear_error() { g_last_error.clear(); }
 
+// Pipelined run_host schedule knobs (plan.h build_e2e_schedule), read by run_host and by the
+// exported fftstencil_e2e_schedule alike so the CPU replay tests see the schedule that runs:
+// FFTSTENCIL_E2E_DEPTH_TAIL (tail skew depth, default = the head's), FFTSTENCIL_E2E_RAMP (1).
+// Measured (profiles/r02_e2e_ramp2.txt): ramp 2 and a deeper tail are within noise or slower
+// (Heat-3D 507 vs 509-511 ms, Heat-2D 88.3-89.4 vs 88.9-89.7 ms per e2e step), so the defaults stay.
+int pipe_tail_depth() { return env_int("FFTSTENCIL_E2E_DEPTH_TAIL", 0); }
+int pipe_ramp() { return env_int("FFTSTENCIL_E2E_RAMP", 1); }
+
 }  // namespace
 
 struct fftstencil_plan {
@@ -872,7 +880,7 @@ int64_t fftstencil_e2e_schedule(int ndim, const int64_t* extents, const double* 
   int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, 1, 0, env_algo());
   if (rc != FFTSTENCIL_OK) { set_error(err); return rc; }
   std::vector<int64_t> ops;
-  if ((rc = build_e2e_schedule(hp, total_steps, chunks, depth, ops)) != FFTSTENCIL_OK) {
+  if ((rc = build_e2e_schedule(hp, total_steps, chunks, depth, ops, pipe_tail_depth(), pipe_ramp())) != FFTSTENCIL_OK) {
     set_error("plan not eligible for the pipelined run_host schedule");
     return rc;
   }
@@ -1344,7 +1352,7 @@ int fftstencil_run_host(fftstencil_plan* p, const double* h_in, double* h_out, i
   const int K = pipe_chunks(p);
   std::vector<int64_t> ops;
   p->last_pipelined = false;
-  if (K && build_e2e_schedule(p->hp, total_steps, K, pipe_depth(p), ops) == FFTSTENCIL_OK) {
+  if (K && build_e2e_schedule(p->hp, total_steps, K, pipe_depth(p), ops, pipe_tail_depth(), pipe_ramp()) == FFTSTENCIL_OK) {
     p->last_launches = 0;
     p->last_pipelined = true;
     p->last_chunks = K;

@@ -101,6 +101,24 @@ __global__ void __launch_bounds__(kBandThreads) band_kernel(const BandArgs a) {
 // without per-cell divisions.  Same definition and result as band_kernel.
 constexpr int kMaxTaps = 512;
 
+// x / d for 0 <= x < 2^20, d >= 1 (block-geometry indices): a float reciprocal estimate (relative
+// error ~2^-21, so at most one off) and one correction step -- ~9 instructions instead of the
+// ~25 of a 32-bit integer division; a 3D band block does ~16 of them per warp (ncu: the
+// per-block index setup was ~40 % of the band kernel's instructions, profiles/r02_band_async_ncu.txt).
+#ifndef BAND_FDIV
+#define BAND_FDIV 1   // 0: integer division (ablation)
+#endif
+__device__ __forceinline__ int fdiv(int x, int d) {
+#if BAND_FDIV
+  int q = __float2int_rz(__fdividef((float)x, (float)d));
+  const int r = x - q * d;
+  q += (r >= d) - (r < 0);
+  return q;
+#else
+  return x / d;
+#endif
+}
+
 // NTH = 256, (256, 6): at most 40 registers (one band CTA fits beside the DMMA engines' fused
 // CTAs); NTH = 1024 for the 1D band, whose two blocks run t (~1000) sequential steps on SMs
 // the fused kernel leaves free (capi.cu), so per-step latency is what counts.
@@ -149,7 +167,7 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
       if (wv != 0.0) {
         const int pos = base + __popc(m & ((1u << lane) - 1u));
         if (pos < kMaxTaps) {
-          const int i2 = k % W2, i1 = (k / W2) % W1, i0 = k / (W1 * W2);
+          const int kq = fdiv(k, W2), i2 = k - kq * W2, i0 = fdiv(kq, W1), i1 = kq - i0 * W1;
           const int o0 = a.active[0] ? i0 - r : 0, o1 = a.active[1] ? i1 - r : 0, o2 = a.active[2] ? i2 - r : 0;
           s_off[pos] = (o0 * D[1] + o1) * D[2] + o2;
           s_w[pos] = wv;
@@ -167,8 +185,8 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
     // region load, flattened over all threads (thin faces have rows of a few cells: a warp per
     // row left most lanes idle); (i0, i1, i2) advanced by carries
     const int D12 = D[1] * D[2];
-    int i0 = threadIdx.x / D12, i1 = (threadIdx.x - i0 * D12) / D[2], i2 = threadIdx.x - i0 * D12 - i1 * D[2];
-    const int d0 = NTH / D12, d1 = (NTH - d0 * D12) / D[2], d2 = NTH - d0 * D12 - d1 * D[2];
+    int i0 = fdiv(threadIdx.x, D12), i1 = fdiv(threadIdx.x - i0 * D12, D[2]), i2 = threadIdx.x - i0 * D12 - i1 * D[2];
+    const int d0 = fdiv(NTH, D12), d1 = fdiv(NTH - d0 * D12, D[2]), d2 = NTH - d0 * D12 - d1 * D[2];
     const double* src0 = a.src + ((rl[0] - off[0]) * a.n[1] + (rl[1] - off[1])) * a.n[2] + (rl[2] - off[2]);
     for (int e = threadIdx.x; e < vol; e += NTH) {
       const double* gp = src0 + ((int64_t)i0 * a.n[1] + i1) * a.n[2] + i2;
@@ -258,9 +276,9 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
       }
       if (w3[0] > 0 && w3[1] > 0 && w3[2] > 0) {
         const int V12 = w3[1] * w3[2], nc = w3[0] * V12;
-        int j0 = threadIdx.x / V12, j1 = (threadIdx.x - j0 * V12) / w3[2];
+        int j0 = fdiv(threadIdx.x, V12), j1 = fdiv(threadIdx.x - j0 * V12, w3[2]);
         int j2 = threadIdx.x - j0 * V12 - j1 * w3[2];
-        const int e0 = NTH / V12, e1 = (NTH - e0 * V12) / w3[2];
+        const int e0 = fdiv(NTH, V12), e1 = fdiv(NTH - e0 * V12, w3[2]);
         const int e2 = NTH - e0 * V12 - e1 * w3[2];
         const int D12 = D[1] * D[2];
         const int de = e2 + e1 * D[2] + e0 * D12;       // index step per NTH cells, before carries
@@ -299,9 +317,9 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
     // cone box of this step, flattened over all threads (no idle lanes on narrow faces);
     // the (k0, k1, k2) decomposition is advanced by carries, not recomputed by divisions
     const int W12 = W1 * W2, ncone = W0 * W12;
-    int k0 = threadIdx.x / W12, k1 = (threadIdx.x - k0 * W12) / W2;
+    int k0 = fdiv(threadIdx.x, W12), k1 = fdiv(threadIdx.x - k0 * W12, W2);
     int k2 = threadIdx.x - k0 * W12 - k1 * W2;
-    const int d0 = NTH / W12, d1 = (NTH - d0 * W12) / W2;
+    const int d0 = fdiv(NTH, W12), d1 = fdiv(NTH - d0 * W12, W2);
     const int d2 = NTH - d0 * W12 - d1 * W2;
     for (int f = threadIdx.x; f < ncone; f += NTH) {
       const int i0 = clo[0] + k0, i1 = clo[1] + k1, i2 = clo[2] + k2;
@@ -327,8 +345,8 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
   // output store, flattened like the load (a face block of axis 2 has one-cell rows)
   const int O0 = (int)(hi[0] - lo[0]), O1 = (int)(hi[1] - lo[1]), O2 = (int)(hi[2] - lo[2]);
   const int O12 = O1 * O2, ovol = O0 * O12;
-  int j0 = threadIdx.x / O12, j1 = (threadIdx.x - j0 * O12) / O2, j2 = threadIdx.x - j0 * O12 - j1 * O2;
-  const int f0 = NTH / O12, f1 = (NTH - f0 * O12) / O2, f2 = NTH - f0 * O12 - f1 * O2;
+  int j0 = fdiv(threadIdx.x, O12), j1 = fdiv(threadIdx.x - j0 * O12, O2), j2 = threadIdx.x - j0 * O12 - j1 * O2;
+  const int f0 = fdiv(NTH, O12), f1 = fdiv(NTH - f0 * O12, O2), f2 = NTH - f0 * O12 - f1 * O2;
   double* dst0 = a.dst + ((lo[0] - off[0]) * a.n[1] + (lo[1] - off[1])) * a.n[2] + (lo[2] - off[2]);
   const double* sb0 = b0 + ((lo[0] - rl[0]) * D[1] + (lo[1] - rl[1])) * D[2] + (lo[2] - rl[2]);
   for (int e = threadIdx.x; e < ovol; e += NTH) {

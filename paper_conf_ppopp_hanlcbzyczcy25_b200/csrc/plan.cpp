@@ -668,8 +668,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
 // (+- h rows) stays within units u-1..u+1 too.  Frontiers f[k] (units [0, f[k]) of pass k
 // issued) with f[k] <= f[k-1] - 1 (or f[k-1] = U) satisfy the read dependency and the
 // ping-pong anti-dependency at once, so the ops run in issue order on one stream.
-int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std::vector<int64_t>& ops) {
+int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std::vector<int64_t>& ops, int Qt,
+                       int ramp) {
   ops.clear();
+  if (Qt <= 0) Qt = Q;
   if (K < 2 || Q < 1 || p.ndim < 2 || p.periodic || p.algo == 2 || p.nranks != 1 || total_steps <= 0)
     return FFTSTENCIL_EINVAL;
   const int64_t U = p.nt[0], n0 = p.ext[0], S = p.S[0], h = p.h;
@@ -693,11 +695,19 @@ int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std
   // Chunk boundaries (outer tile rows): K regular chunks, with the FIRST input chunk and the LAST
   // output chunk split 1/4 + 3/4 -- nothing overlaps the first H2D chunk or the last D2H chunk,
   // so those two are the small ones (Heat-2D: 2 x 2.4 ms exposed copies at K = 6 -> 2 x 0.6 ms).
+  // ramp = 2 also splits the LAST input chunk 3/4 + 1/4 and the FIRST output chunk 1/4 + 3/4: the
+  // head's drain after the last H2D (every head pass catching up on that chunk) and the tail's
+  // fill before the first D2H (the tail passes advancing to it) scale with those chunks' size.
   const int64_t q4 = std::max<int64_t>(1, U / (4 * (int64_t)K));
   std::vector<int64_t> ib{0, q4}, ob{0};
-  for (int c = 1; c <= K; ++c) ib.push_back(U * c / K);
-  for (int j = 1; j < K; ++j) ob.push_back(U * j / K);
-  ob.push_back(U - q4);
+  if (ramp >= 2) ob.push_back(q4);
+  for (int c = 1; c <= K; ++c) {
+    if (ramp >= 2 && c == K && U - q4 > ib.back()) ib.push_back(U - q4);
+    ib.push_back(U * c / K);
+  }
+  for (int j = 1; j < K; ++j)
+    if (U * j / K > ob.back()) ob.push_back(U * j / K);
+  if (U - q4 > ob.back()) ob.push_back(U - q4);
   ob.push_back(U);
   // head: input chunk c, its ring rows, then the first Q passes advance behind it
   for (size_t c = 1; c < ib.size(); ++c) {
@@ -710,7 +720,7 @@ int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std
   // tail: the last Q passes advance until pass P holds chunk j, which is then copied out
   for (size_t j = 1; j < ob.size(); ++j) {
     const int64_t bj = ob[j];
-    propagate([&](int64_t k) { return k <= P - Q ? U : std::min<int64_t>(U, bj + (P - k)); });
+    propagate([&](int64_t k) { return k <= P - Qt ? U : std::min<int64_t>(U, bj + (P - k)); });
     if (f[(size_t)P] < bj) { ops.clear(); return FFTSTENCIL_EINVAL; }
     push(3, row_of(ob[j - 1]), row_of(bj), 0);
   }

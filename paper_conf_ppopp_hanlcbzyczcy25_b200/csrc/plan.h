@@ -103,7 +103,10 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
 //   op 3: copy result rows [x, y) device -> host once everything before it is done.
 // Returns 0 with the ops, or FFTSTENCIL_EINVAL when the plan is not eligible (1D, periodic,
 // a slab plan, the unfused ablation, h > S, fewer than 2K units, no steps).
-int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std::vector<int64_t>& ops);
+// Qt: skewed passes of the tail (<= 0: Q); ramp: 1 small first input / last output chunk, 2 also a
+// small last input / first output chunk.
+int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std::vector<int64_t>& ops, int Qt = 0,
+                       int ramp = 1);
 
 // Dense-DFT tile cost model (executed FP64 tensor flops per cell-step) used to pick L/T.
 double model_flops_2d(int L, int S, int T);

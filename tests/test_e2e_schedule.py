@@ -91,7 +91,9 @@ def test_schedule_replays(ext, shape, r, T, steps, K, Q):
     ops, U, P = replay(ext, shape, r, T, steps, K, Q)
     n_items = int((ops[:, 0] == 2).sum())
     assert n_items >= P                 # at least one item per pass
-    assert n_items <= P + 2 * K * min(Q, P)
+    # at most K + 2 input and K + 2 output pieces (plan.cpp: ramp 1 splits the first input and
+    # the last output chunk 1/4 + 3/4, ramp 2 also the last input and the first output chunk)
+    assert n_items <= P + 2 * (K + 2) * min(Q, P)
 
 
 def test_head_overlaps_copies():
@@ -161,3 +163,14 @@ def test_replay_catches_write_after_copy_out():
     replay((1500, 200), "star", 1, 11, 100, 4, 6, check_cover=False)          # the clean schedule passes
     with pytest.raises(AssertionError, match="queued for copy-out"):
         replay((1500, 200), "star", 1, 11, 100, 4, 6, mutate=mutate, check_cover=False)
+
+
+@pytest.mark.parametrize("ramp,tail", [(1, None), (2, 24), (2, 3), (1, 30)])
+@pytest.mark.parametrize("ext,shape,r,T,steps,K,Q", [CASES[0], CASES[3], CASES[5], CASES[8]])
+def test_schedule_replays_ramp_and_tail_depth(monkeypatch, ramp, tail, ext, shape, r, T, steps, K, Q):
+    """The schedule knobs the A/B runs use (FFTSTENCIL_E2E_RAMP, FFTSTENCIL_E2E_DEPTH_TAIL) keep
+    every replay invariant."""
+    monkeypatch.setenv("FFTSTENCIL_E2E_RAMP", str(ramp))
+    if tail is not None:
+        monkeypatch.setenv("FFTSTENCIL_E2E_DEPTH_TAIL", str(tail))
+    replay(ext, shape, r, T, steps, K, Q)
