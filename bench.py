@@ -118,6 +118,8 @@ def parse(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-per-config", action="store_true", help="skip the other BASELINE configs (N = 1)")
     ap.add_argument("--json-out", default="")
+    ap.add_argument("--transport", default="peer", choices=["peer", "nccl"],
+                    help="N > 1 halo exchange: CUDA-IPC peer pushes + stream-memory signals (default) or NCCL send/recv")
     return ap.parse_args(argv)
 
 
@@ -405,15 +407,29 @@ def exact_cells_of(info, gext):
     return exact
 
 
+def max_over_ranks(torch, dist, dev, world, x: float) -> float:
+    """Max of a per-rank float over the group (a CPU tensor on a gloo group, CUDA on NCCL)."""
+    if world == 1:
+        return x
+    on_gpu = dist.get_backend() == "nccl"
+    t = torch.tensor([x], dtype=torch.float64, device=dev if on_gpu else "cpu")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def measure(fs, torch, dist, dev, world, rank, name, T, time_steps, steps, warmup, weights="seeded",
-            clocks=False, e2e=False, keep_input=False):
+            clocks=False, e2e=False, keep_input=False, transport="peer"):
     """Time `steps` fftstencil_run calls of `time_steps` time steps each on workload `name`
     (weak scaling: each rank holds the workload's rows, the global grid stacks them)."""
     wk = wl.CONFIGS[name]
     w = wk.weights(weights)
     gext = (wk.extents[0] * world,) + tuple(wk.extents[1:])
     cells = int(np.prod(gext))
-    if world > 1:
+    if world > 1 and transport == "peer":
+        plan = fs.Plan(gext, w, wk.radius, T, nranks=world, rank=rank, transport="peer")
+        plan.connect_peers()
+        u0 = wl.grid(plan.extents, wk.cfg_id * 1000 + rank)   # this rank's slab, seeded per slab
+    elif world > 1:
         obj = [fs.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         plan = fs.Plan(gext, w, wk.radius, T, nranks=world, rank=rank, nccl_id=obj[0])
@@ -449,10 +465,7 @@ def measure(fs, torch, dist, dev, world, rank, name, T, time_steps, steps, warmu
     plan.set_profiling(False)
     launches = plan.info()["last_run_launches"]
     ms = ev0.elapsed_time(ev1)
-    ms_t = torch.tensor([ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
-    ms_max = float(ms_t.item())
+    ms_max = max_over_ranks(torch, dist, dev, world, ms)
     passes = steps * -(-time_steps // info["T"])
     res = {"workload": name, "value": gstencils(cells, time_steps * steps, ms_max), "unit": "GStencils/s",
            "ms_per_step": ms_max / steps, "steps": steps, "time_steps_per_step": time_steps,
@@ -476,10 +489,7 @@ def measure(fs, torch, dist, dev, world, rank, name, T, time_steps, steps, warmu
             plan.run_host(h_in, h_out, time_steps, stream)
         e1.record(stream)
         barrier()
-        ems = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(ems, op=dist.ReduceOp.MAX)
-        e_ms = float(ems.item())
+        e_ms = max_over_ranks(torch, dist, dev, world, e0.elapsed_time(e1))
         pinfo = plan.info()
         piped = pinfo["last_run_pipelined"]
         res["e2e"] = {"value": gstencils(cells, time_steps * k_e, e_ms), "unit": "GStencils/s",
@@ -492,6 +502,8 @@ def measure(fs, torch, dist, dev, world, rank, name, T, time_steps, steps, warmu
                       if piped else "none: copy-run-copy (the plan does not take the pipelined schedule)"}
         if not np.isfinite(h_out.numpy()).all():
             raise RuntimeError("non-finite output")
+    if world > 1:
+        barrier()   # no rank frees buffers a neighbour still has mapped (peer transport)
     plan.close()
     if keep_input:
         res["_u0"] = u0
@@ -516,7 +528,8 @@ def main(argv=None):
     import paper_conf_ppopp_hanlcbzyczcy25_b200 as fs
 
     nccl_log = None
-    if world > 1:
+    shared = os.environ.get("FFTSTENCIL_BENCH_SHARE_GPU") == "1"
+    if world > 1 and args.transport == "nccl":
         # the library's own communicator (ncclCommInitRank in fftstencil_plan_create_dist) logs
         # its setup -- transport, NVLS, channels -- to a file, so stdout keeps the one JSON line
         nccl_log = os.path.join(ROOT, "gpurun_out", f"nccl_rank{rank}.log")
@@ -525,6 +538,12 @@ def main(argv=None):
         os.environ.setdefault("NCCL_DEBUG_FILE", nccl_log)
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif world > 1:
+        # peer transport: the library moves the halos itself (CUDA IPC); the harness only needs
+        # a barrier and a max over ranks, over gloo.  FFTSTENCIL_BENCH_SHARE_GPU=1 (harness test
+        # on a one-GPU box) puts every rank on device 0 -- not a scaling measurement.
+        torch.cuda.set_device(local % torch.cuda.device_count() if shared else local)
+        dist.init_process_group("gloo")
     else:
         torch.cuda.set_device(0)
     dev = torch.device("cuda", torch.cuda.current_device())
@@ -533,7 +552,7 @@ def main(argv=None):
     time_steps = args.time_steps or wk.bench_steps
     main_res = measure(fs, torch, dist, dev, world, rank, name, args.T or wk.T, time_steps, args.steps,
                        args.warmup, args.weights, clocks=True, e2e=not args.no_e2e,
-                       keep_input=world == 1 and not args.no_cpu_baseline)
+                       keep_input=world == 1 and not args.no_cpu_baseline, transport=args.transport)
 
     u_main = main_res.pop("_u0", None)
     cpu = None
@@ -575,7 +594,9 @@ def main(argv=None):
                        "grid": main_res["grid"], "time_steps_per_step": time_steps, "T": main_res["T"],
                        "tile": main_res["tile"], "valid": main_res["valid"],
                        "parallelism": "single GPU" if world == 1 else
-                       f"outer-axis decomposition over {world} GPUs, NCCL halo exchange of r*T rows per pass",
+                       f"outer-axis decomposition over {world} GPUs, r*T halo rows per pass "
+                       + ("pushed into the neighbours' buffers (CUDA IPC peer copies, stream-memory signal/wait)"
+                          if args.transport == "peer" else "by NCCL send/recv"),
                        "l2": f"inputs {int(np.prod(wk.extents)) * 8 / 1e6:.0f} MB per GPU > 126 MB L2 (no flush needed)"},
             "roofline": main_res["roofline"],
             "cpu_baseline": cpu,
@@ -586,6 +607,10 @@ def main(argv=None):
         }
         if nccl_log:
             line["config"]["nccl"] = nccl_summary(nccl_log)
+        if world > 1:
+            line["config"]["transport"] = args.transport
+        if world > 1 and shared:
+            line["shared_gpu"] = "every rank on device 0 (FFTSTENCIL_BENCH_SHARE_GPU=1): a harness test, not a scaling number"
         s = json.dumps(line)
         print(s, flush=True)
         if args.json_out:

@@ -180,6 +180,28 @@ fftstencil_plan* fftstencil_plan_create_dist(int ndim, const int64_t* extents, c
                                              int radius, int T, int nranks, int rank,
                                              const void* nccl_unique_id);
 
+/* ---- peer-memory transport: the same decomposition without NCCL ----
+ * Each rank's two slab buffers and a two-word flag array are shared with its neighbours through
+ * CUDA IPC.  After every pass a rank copies its h = radius*T boundary rows straight into the
+ * neighbours' halo rows (copy engine over NVLink; a same-device copy when two processes share
+ * one GPU) and bumps the neighbours' flag word with a stream memory write; before its
+ * halo-dependent tile pairs a rank's stream waits (stream memory wait, no host round trip, no
+ * spinning kernel) until both neighbours have signalled as often as it has.  Halo-free pairs
+ * run before the wait, so the exchange overlaps them.  Results are bitwise equal to one GPU.
+ * Every rank must make the same sequence of fftstencil_run calls (same total_steps): the
+ * ranks advance in lockstep (P + 1 signals per run of P passes).
+ * Creation is local (no collective); then each rank exports its handle
+ * (fftstencil_peer_handle, FFTSTENCIL_PEER_HANDLE_BYTES), the ranks exchange them (any host
+ * channel: torch.distributed, files, ...) and each connects to its neighbours
+ * (fftstencil_peer_connect: lower = rank-1's handle or NULL for rank 0, upper = rank+1's or NULL
+ * for the last rank).  fftstencil_run before connecting fails with EINVAL.  The devices of
+ * neighbouring ranks must be peer capable (NVLink/NVSwitch), or the same device. */
+#define FFTSTENCIL_PEER_HANDLE_BYTES 256
+fftstencil_plan* fftstencil_plan_create_dist_peer(int ndim, const int64_t* extents, const double* weights,
+                                                  int radius, int T, int nranks, int rank);
+int fftstencil_peer_handle(const fftstencil_plan* plan, void* out, int64_t cap);
+int fftstencil_peer_connect(fftstencil_plan* plan, const void* lower, const void* upper);
+
 /* Writes a new 128-byte ncclUniqueId into `out` (caller-owned, >= 128 bytes; rank 0 of a
  * group).  ENCCL if NCCL cannot create one.  No PAPER.md passage: the paper is single-GPU;
  * the decomposition is SURVEY §8(a) row a10. */

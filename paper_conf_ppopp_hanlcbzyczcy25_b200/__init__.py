@@ -131,10 +131,13 @@ class Plan:
     """A FlashFFTStencil plan bound to the current CUDA device."""
 
     def __init__(self, extents, weights, radius: int, T: int = 0, nranks: int = 1, rank: int = 0,
-                 nccl_id: bytes | None = None, loopback: bool = False, periodic: bool = False):
+                 nccl_id: bytes | None = None, loopback: bool = False, periodic: bool = False,
+                 transport: str | None = None):
         """extents are GLOBAL.  nranks > 1: this process's rank of the outer-axis decomposition;
         pass the group's nccl_id (bytes from nccl_unique_id()), or loopback=True for a rank
-        run with run_group on one device.  in/out tensors then hold this rank's slab
+        run with run_group on one device, or transport="peer" for the CUDA-IPC peer-memory
+        transport (then exchange peer_handle() bytes and call peer_connect, or connect_peers()
+        under torch.distributed).  in/out tensors then hold this rank's slab
         (rows [row_begin, row_end) of info())."""
         ext, w = _arrays(extents, weights, radius)
         self.global_extents = tuple(int(e) for e in ext)
@@ -143,6 +146,9 @@ class Plan:
         if nranks == 1:
             h = self._lib.fftstencil_plan_create_ex(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
                                                     _native.PERIODIC if periodic else 0)
+        elif transport == "peer":
+            h = self._lib.fftstencil_plan_create_dist_peer(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T),
+                                                           int(nranks), int(rank))
         else:
             if nccl_id is None and not loopback:
                 raise ValueError("nranks > 1 needs nccl_id (or loopback=True)")
@@ -155,6 +161,32 @@ class Plan:
         self.device = _current_device()
         inf = self.info()
         self.extents = (inf["row_end"] - inf["row_begin"],) + self.global_extents[1:]
+
+    # -- peer transport --
+    def peer_handle(self) -> bytes:
+        """This rank's FFTSTENCIL_PEER_HANDLE_BYTES handle blob (CUDA IPC handles + slab geometry)."""
+        buf = ctypes.create_string_buffer(_native.PEER_HANDLE_BYTES)
+        rc = self._lib.fftstencil_peer_handle(self._h, buf, _native.PEER_HANDLE_BYTES)
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+        return buf.raw
+
+    def peer_connect(self, lower: bytes | None, upper: bytes | None) -> None:
+        """Open the neighbours' handles (None where there is no neighbour)."""
+        lb = ctypes.create_string_buffer(bytes(lower), _native.PEER_HANDLE_BYTES) if lower is not None else None
+        ub = ctypes.create_string_buffer(bytes(upper), _native.PEER_HANDLE_BYTES) if upper is not None else None
+        rc = self._lib.fftstencil_peer_connect(self._h, lb, ub)
+        if rc != 0:
+            raise FftStencilError(rc, last_error())
+
+    def connect_peers(self, group=None) -> None:
+        """Exchange handles over torch.distributed (any backend) and connect to the neighbours."""
+        import torch.distributed as dist
+        inf = self.info()
+        rank, world = inf["rank"], inf["nranks"]
+        handles = [None] * world
+        dist.all_gather_object(handles, self.peer_handle(), group=group)
+        self.peer_connect(handles[rank - 1] if rank > 0 else None, handles[rank + 1] if rank < world - 1 else None)
 
     # -- lifetime --
     def close(self):

@@ -22,7 +22,9 @@ EXPORTS = ("fftstencil_plan_create", "fftstencil_run", "fftstencil_run_host", "f
            "fftstencil_set_profiling", "fftstencil_profile_read", "fftstencil_plan_create_dist",
            "fftstencil_nccl_unique_id", "fftstencil_run_group", "fftstencil_describe_dist",
            "fftstencil_plan_create_ex", "fftstencil_describe_ex", "fftstencil_run_emit",
-           "fftstencil_e2e_schedule")
+           "fftstencil_e2e_schedule", "fftstencil_plan_create_dist_peer", "fftstencil_peer_handle",
+           "fftstencil_peer_connect")
+PEER_HANDLE_BYTES = 256   # FFTSTENCIL_PEER_HANDLE_BYTES
 
 
 class Info(ctypes.Structure):
@@ -126,6 +128,13 @@ def lib():
     L.fftstencil_plan_create_dist.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                               ctypes.c_int, vp]
     L.fftstencil_plan_create_dist.restype = vp
+    L.fftstencil_plan_create_dist_peer.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                                   ctypes.c_int]
+    L.fftstencil_plan_create_dist_peer.restype = vp
+    L.fftstencil_peer_handle.argtypes = [vp, vp, ctypes.c_int64]
+    L.fftstencil_peer_handle.restype = ctypes.c_int
+    L.fftstencil_peer_connect.argtypes = [vp, vp, vp]
+    L.fftstencil_peer_connect.restype = ctypes.c_int
     L.fftstencil_nccl_unique_id.argtypes = [vp]
     L.fftstencil_nccl_unique_id.restype = ctypes.c_int
     L.fftstencil_run_group.argtypes = [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.c_int,

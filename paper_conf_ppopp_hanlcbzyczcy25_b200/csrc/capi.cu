@@ -114,6 +114,14 @@ struct fftstencil_plan {
   int max_ctas = 0;              // FFTSTENCIL_MAX_CTAS (tests): cap on every fused launch's grid, so each
                                  // persistent CTA walks many pairs through its refill / mbarrier loop
   double* dE[2] = {nullptr, nullptr};   // slab + halo buffers, rows [g0, g1)
+  // ---- peer-memory transport (no NCCL; fftstencil_plan_create_dist_peer) ----
+  bool peer = false;            // halo rows pushed into the neighbours' buffers through CUDA IPC
+  bool peer_connected = false;
+  uint32_t* dFlags = nullptr;   // [0]: epoch signalled by the lower neighbour, [1]: by the upper one
+  double* pE[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};   // [lower, upper][buffer] (IPC-mapped)
+  uint32_t* pFlags[2] = {nullptr, nullptr};                       // the neighbours' dFlags
+  int64_t pG0[2] = {0, 0};      // the neighbours' window starts g0
+  uint32_t epoch = 0;           // signals sent so far (both neighbours send the same count)
   int ecur = 0;               // index of the buffer holding the current state
   // ---- profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run() ----
   bool profiling = false;
@@ -127,6 +135,25 @@ namespace {
 using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+// Stream memory operations (driver API through the runtime's entry-point query, like the
+// tensor-map encoder): the peer transport's cross-process signal and wait.
+using StreamValue32Fn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+StreamValue32Fn stream_fn(const char* name) {
+  void* f = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &f, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess)
+    return nullptr;
+  return (StreamValue32Fn)f;
+}
+StreamValue32Fn write_value_fn() {
+  static StreamValue32Fn fn = stream_fn("cuStreamWriteValue32");
+  return fn;
+}
+StreamValue32Fn wait_value_fn() {
+  static StreamValue32Fn fn = stream_fn("cuStreamWaitValue32");
+  return fn;
+}
 
 EncodeTiledFn encode_fn() {
   static EncodeTiledFn fn = [] {
@@ -169,6 +196,12 @@ void free_plan(fftstencil_plan* p) {
   cudaGetDevice(&cur);
   cudaSetDevice(p->device);
   if (p->comm) ncclCommDestroy(p->comm);
+  for (int side = 0; side < 2; ++side) {
+    for (int b = 0; b < 2; ++b)
+      if (p->pE[side][b]) cudaIpcCloseMemHandle(p->pE[side][b]);
+    if (p->pFlags[side]) cudaIpcCloseMemHandle(p->pFlags[side]);
+  }
+  cudaFree(p->dFlags);
   if (p->comm_stream) cudaStreamDestroy(p->comm_stream);
   if (p->ev_ready) cudaEventDestroy(p->ev_ready);
   if (p->ev_xchg) cudaEventDestroy(p->ev_xchg);
@@ -615,6 +648,88 @@ int nccl_exchange(fftstencil_plan* p, cudaStream_t s) {
   return FFTSTENCIL_OK;
 }
 
+// ---- peer transport: push own boundary rows into the neighbours' halo rows, signal, wait ----
+// Rows [row_lo, row_lo + h) of buffer `b` go to the lower neighbour's halo (its rows from
+// row_lo on, at its local row row_lo - g0_lower); rows [row_hi - h, row_hi) to the upper
+// neighbour's (its local rows from 0).  Copy engine over NVLink (same-device copy when the
+// "neighbour" is another process on this GPU), ordered on `s` after the pass that wrote them.
+int peer_push(fftstencil_plan* p, int b, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  const size_t rc_ = p->row_cells, bytes = (size_t)hp.h * rc_ * sizeof(double);
+  cudaError_t e = cudaSuccess;
+  if (hp.rank > 0)
+    e = cudaMemcpyAsync(p->pE[0][b] + (size_t)(hp.row_lo - p->pG0[0]) * rc_, p->dE[b] + (size_t)(hp.row_lo - hp.g0) * rc_,
+                        bytes, cudaMemcpyDeviceToDevice, s);
+  if (e == cudaSuccess && hp.rank < hp.nranks - 1)
+    e = cudaMemcpyAsync(p->pE[1][b] + (size_t)(hp.row_hi - hp.h - p->pG0[1]) * rc_,
+                        p->dE[b] + (size_t)(hp.row_hi - hp.h - hp.g0) * rc_, bytes, cudaMemcpyDeviceToDevice, s);
+  return e == cudaSuccess ? FFTSTENCIL_OK : cuda_fail(e, "peer halo push");
+}
+
+// Epoch ++ written into both neighbours' flag words (stream-ordered after the push; the write
+// carries a memory barrier, so the neighbour sees the rows before the flag).
+int peer_signal(fftstencil_plan* p, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  ++p->epoch;
+  CUresult r = CUDA_SUCCESS;
+  if (hp.rank > 0) r = write_value_fn()((CUstream)s, (CUdeviceptr)(p->pFlags[0] + 1), p->epoch, 0);
+  if (r == CUDA_SUCCESS && hp.rank < hp.nranks - 1)
+    r = write_value_fn()((CUstream)s, (CUdeviceptr)(p->pFlags[1] + 0), p->epoch, 0);
+  if (r != CUDA_SUCCESS) {
+    set_error("cuStreamWriteValue32 failed (" + std::to_string((int)r) + ")");
+    return FFTSTENCIL_ECUDA;
+  }
+  return FFTSTENCIL_OK;
+}
+
+// `s` waits until both neighbours have signalled as often as this rank.
+int peer_wait(fftstencil_plan* p, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  // peer copies land in this device's memory before the writer's flag (the write-value carries a
+  // memory barrier); no remote-write flush is needed (that flag is for third-party RDMA writers)
+  const unsigned flags = CU_STREAM_WAIT_VALUE_GEQ;
+  CUresult r = CUDA_SUCCESS;
+  if (hp.rank > 0) r = wait_value_fn()((CUstream)s, (CUdeviceptr)(p->dFlags + 0), p->epoch, flags);
+  if (r == CUDA_SUCCESS && hp.rank < hp.nranks - 1)
+    r = wait_value_fn()((CUstream)s, (CUdeviceptr)(p->dFlags + 1), p->epoch, flags);
+  if (r != CUDA_SUCCESS) {
+    set_error("cuStreamWaitValue32 failed (" + std::to_string((int)r) + ")");
+    return FFTSTENCIL_ECUDA;
+  }
+  return FFTSTENCIL_OK;
+}
+
+// One run over the peer transport.  Per run every rank signals P + 1 times (after the copy-in,
+// after every pass but the last, at the end), so the ranks stay in lockstep:
+//   wait (neighbours done with the previous run: its halo rows are free) -> copy-in, push
+//   buffer 0, signal -> per pass: halo-free pairs, wait, edge pairs + band, push dst, signal.
+// A neighbour writes this rank's buffer b only after the pass that last read it (it waited
+// for that pass's signal first), and never the owned rows the passes write.
+int run_dist_peer(fftstencil_plan* p, const double* in, double* out, int64_t total_steps, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  int rc;
+  if ((rc = peer_wait(p, s))) return rc;
+  if ((rc = dist_begin(p, in, s))) return rc;
+  if ((rc = peer_push(p, 0, s)) || (rc = peer_signal(p, s))) return rc;
+  const int T = hp.T;
+  const int64_t nfull = total_steps / T, P = nfull + (total_steps % T ? 1 : 0);
+  for (int64_t i = 0; i < P; ++i) {
+    const int t = i < nfull ? T : (int)(total_steps % T);
+    const double* src = p->dE[p->ecur];
+    double* dst = p->dE[p->ecur ^ 1];
+    if ((rc = launch_fused(p, src, dst, t, hp.ipair_lo, hp.ipair_hi, s))) return rc;
+    if ((rc = peer_wait(p, s))) return rc;
+    if ((rc = launch_fused(p, src, dst, t, hp.pair_lo, hp.ipair_lo, s))) return rc;
+    if ((rc = launch_fused(p, src, dst, t, hp.ipair_hi, hp.pair_hi, s))) return rc;
+    if ((rc = launch_band_pass(p, src, dst, t, s))) return rc;
+    if ((rc = band_join(p, s))) return rc;
+    p->ecur ^= 1;
+    if (i + 1 < P && ((rc = peer_push(p, p->ecur, s)) || (rc = peer_signal(p, s)))) return rc;
+  }
+  if ((rc = dist_end(p, out, s))) return rc;
+  return peer_signal(p, s);
+}
+
 // One pass of a dist rank: interior pairs overlap the exchange (if `xchg`), then the
 // halo-dependent pairs and the band.
 int dist_pass(fftstencil_plan* p, int t, bool xchg, cudaStream_t s) {
@@ -647,6 +762,13 @@ int run_dist(fftstencil_plan* p, const double* in, double* out, int64_t total_st
       if (e != cudaSuccess) return cuda_fail(e, "copy");
     }
     return FFTSTENCIL_OK;
+  }
+  if (p->peer) {
+    if (!p->peer_connected) {
+      set_error("a peer-transport rank must be connected (fftstencil_peer_connect) before it runs");
+      return FFTSTENCIL_EINVAL;
+    }
+    return run_dist_peer(p, in, out, total_steps, s);
   }
   int rc = dist_begin(p, in, s);
   if (rc) return rc;
@@ -1052,6 +1174,90 @@ int fftstencil_nccl_unique_id(void* out) {
   std::memcpy(out, &id, sizeof id);
   clear_error();
   return FFTSTENCIL_OK;
+}
+
+fftstencil_plan* fftstencil_plan_create_dist_peer(int ndim, const int64_t* extents, const double* weights, int radius,
+                                                  int T, int nranks, int rank) {
+  if (nranks < 2 || rank < 0 || rank >= nranks) { set_error("the peer transport needs nranks >= 2, 0 <= rank < nranks"); return nullptr; }
+  if (!write_value_fn() || !wait_value_fn()) { set_error("stream memory operations unavailable"); return nullptr; }
+  fftstencil_plan* p = new (std::nothrow) fftstencil_plan();
+  if (!p) { set_error("host allocation failed"); return nullptr; }
+  std::string err;
+  int rc = build_host_plan(ndim, extents, weights, radius, T, p->hp, err, nranks, rank, env_algo());
+  if (rc != FFTSTENCIL_OK) { set_error(err); delete p; return nullptr; }
+  p->dist = true;
+  p->peer = true;
+  if (setup_device(p) != FFTSTENCIL_OK) { free_plan(p); return nullptr; }
+  cudaError_t e = cudaMalloc((void**)&p->dFlags, 2 * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaMemset(p->dFlags, 0, 2 * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) { cuda_fail(e, "peer flags"); free_plan(p); return nullptr; }
+  clear_error();
+  return p;
+}
+
+// Handle blob: IPC handles of dE[0], dE[1], dFlags (3 x 64 bytes), then int64 g0, row_lo, row_hi, rank.
+int fftstencil_peer_handle(const fftstencil_plan* p, void* out, int64_t cap) {
+  if (!p || !out || !p->peer) { set_error("a peer-transport plan and an output buffer are required"); return FFTSTENCIL_EINVAL; }
+  if (cap < FFTSTENCIL_PEER_HANDLE_BYTES) { set_error("cap < FFTSTENCIL_PEER_HANDLE_BYTES"); return FFTSTENCIL_EINVAL; }
+  unsigned char* o = static_cast<unsigned char*>(out);
+  std::memset(o, 0, FFTSTENCIL_PEER_HANDLE_BYTES);
+  cudaIpcMemHandle_t hd;
+  void* ptrs[3] = {p->dE[0], p->dE[1], p->dFlags};
+  for (int k = 0; k < 3; ++k) {
+    cudaError_t e = cudaIpcGetMemHandle(&hd, ptrs[k]);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaIpcGetMemHandle");
+    std::memcpy(o + 64 * k, &hd, sizeof hd);
+  }
+  const int64_t geo[4] = {p->hp.g0, p->hp.row_lo, p->hp.row_hi, p->hp.rank};
+  std::memcpy(o + 192, geo, sizeof geo);
+  clear_error();
+  return FFTSTENCIL_OK;
+}
+
+int fftstencil_peer_connect(fftstencil_plan* p, const void* lower, const void* upper) {
+  if (!p || !p->peer) { set_error("a peer-transport plan is required"); return FFTSTENCIL_EINVAL; }
+  const HostPlan& hp = p->hp;
+  if ((hp.rank > 0) != (lower != nullptr) || (hp.rank < hp.nranks - 1) != (upper != nullptr)) {
+    set_error("pass exactly the existing neighbours' handles (lower for rank > 0, upper for rank < nranks - 1)");
+    return FFTSTENCIL_EINVAL;
+  }
+  if (p->peer_connected) { set_error("already connected"); return FFTSTENCIL_EINVAL; }
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (cur != p->device) cudaSetDevice(p->device);
+  const void* hs[2] = {lower, upper};
+  int rc = FFTSTENCIL_OK;
+  for (int side = 0; side < 2 && rc == FFTSTENCIL_OK; ++side) {
+    if (!hs[side]) continue;
+    const unsigned char* h = static_cast<const unsigned char*>(hs[side]);
+    int64_t geo[4];
+    std::memcpy(geo, h + 192, sizeof geo);
+    const int64_t want = side == 0 ? hp.rank - 1 : hp.rank + 1;
+    // the lower neighbour's rows end where ours begin, the upper one's begin where ours end
+    if (geo[3] != want || (side == 0 ? geo[2] != hp.row_lo : geo[1] != hp.row_hi)) {
+      set_error("peer handle of the wrong rank or geometry");
+      rc = FFTSTENCIL_EINVAL;
+      break;
+    }
+    p->pG0[side] = geo[0];
+    void* ptrs[3] = {nullptr, nullptr, nullptr};
+    for (int k = 0; k < 3 && rc == FFTSTENCIL_OK; ++k) {
+      cudaIpcMemHandle_t hd;
+      std::memcpy(&hd, h + 64 * k, sizeof hd);
+      cudaError_t e = cudaIpcOpenMemHandle(&ptrs[k], hd, cudaIpcMemLazyEnablePeerAccess);
+      if (e != cudaSuccess) rc = cuda_fail(e, "cudaIpcOpenMemHandle");
+    }
+    p->pE[side][0] = static_cast<double*>(ptrs[0]);
+    p->pE[side][1] = static_cast<double*>(ptrs[1]);
+    p->pFlags[side] = static_cast<uint32_t*>(ptrs[2]);
+  }
+  if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
+  if (rc == FFTSTENCIL_OK) {
+    p->peer_connected = true;
+    clear_error();
+  }
+  return rc;
 }
 
 int fftstencil_run(fftstencil_plan* p, const double* in, double* out, int64_t total_steps, void* stream) {

@@ -103,3 +103,25 @@ def test_nccl_two_ranks_bitwise(fs, tmp_path):
     assert res.returncode == 0, log[-4000:]
     assert log.count("bitwise OK") == 5, log[-4000:]
     assert "Init COMPLETE" in log or "ncclCommInitRank" in log, "no NCCL communicator was initialised"
+
+
+@pytest.mark.parametrize("nproc", [2, 3])
+def test_peer_transport_processes(fs, tmp_path, nproc):
+    """The peer-memory transport (CUDA IPC halo pushes + stream-memory signal / wait, no NCCL)
+    across `nproc` processes -- on one GPU when only one is visible (IPC within a device), else
+    one GPU per rank -- bitwise equal to one GPU over chained calls (G7)."""
+    import os
+    import socket
+    import subprocess
+    import sys
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    worker = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_peer_worker.py")
+    res = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+                          "--master-addr=127.0.0.1", f"--master-port={port}", worker],
+                         capture_output=True, text=True, timeout=900)
+    log = res.stdout + res.stderr
+    (tmp_path / "peer.log").write_text(log)
+    assert res.returncode == 0, log[-4000:]
+    assert log.count("bitwise OK") == 6, log[-4000:]
