@@ -9,4 +9,4 @@ for w in heat3d box3d27p; do
   python -c "import json;d=json.loads(open('gpurun_out/r02_ring_$w.jsonl').read().strip().splitlines()[-1]);r=d['roofline'];print('$w', round(d['value'],1), 'GSt/s', 'frac', round(r['frac'],3), 'smem', round(r['smem']['frac'],3), 'fused ms', round(r['fused_ms_avg'],3), d['clocks'])" || tail -5 gpurun_out/r02_ring_$w.jsonl
 done
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:fft3d_bf -s 2 -c 1 -o gpurun_out/r02_fft3d_ring python bench.py --workload heat3d --steps 1 --warmup 1 --time-steps 8 --no-e2e --no-cpu-baseline --no-per-config > gpurun_out/r02_ncu3d_ring.log 2>&1; echo ncu rc=$?
-bash tools/r02_ozaki.sh
+bash tools/runs/r02_ozaki.sh

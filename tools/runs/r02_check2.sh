@@ -6,4 +6,4 @@ for w in heat2d heat3d box2d49p; do
   timeout 300 python bench.py --workload $w --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-per-config > gpurun_out/r02_clean_$w.jsonl 2>&1
   python -c "import json;d=json.loads(open('gpurun_out/r02_clean_$w.jsonl').read().strip().splitlines()[-1]);r=d['roofline'];print('$w', round(d['value'],1), 'GSt/s', 'frac', round(r['frac'],3), 'fused ms', round(r['fused_ms_avg'],3), d['clocks'])" || tail -5 gpurun_out/r02_clean_$w.jsonl
 done
-bash tools/r02_ozaki.sh
+bash tools/runs/r02_ozaki.sh
