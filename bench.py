@@ -407,6 +407,42 @@ def exact_cells_of(info, gext):
     return exact
 
 
+TRANSPORT_NOTE = []   # set when the peer transport had to fall back to NCCL (bench line config)
+
+
+def peer_plan(fs, dist, world, rank, gext, w, radius, T):
+    """A connected peer-transport plan, or None on EVERY rank if any rank failed (creation, handle
+    export or mapping a neighbour's memory, e.g. devices without peer access): the group then
+    falls back to NCCL together.  Each step is followed by an all-gather, so no rank is left
+    waiting in a collective the others skipped."""
+    def agree(err):
+        errs = [None] * world
+        dist.all_gather_object(errs, err)
+        return [e for e in errs if e]
+
+    plan, handle, err = None, None, ""
+    try:
+        plan = fs.Plan(gext, w, radius, T, nranks=world, rank=rank, transport="peer")
+        handle = plan.peer_handle()
+    except Exception as e:   # noqa: BLE001 -- reported in the line
+        err = f"rank {rank}: {e}"
+    handles = [None] * world
+    dist.all_gather_object(handles, handle)
+    errs = agree(err)
+    if not errs:
+        try:
+            plan.peer_connect(handles[rank - 1] if rank > 0 else None, handles[rank + 1] if rank < world - 1 else None)
+        except Exception as e:   # noqa: BLE001
+            err = f"rank {rank}: {e}"
+        errs = agree(err)
+    if errs:
+        if plan is not None:
+            plan.close()
+        TRANSPORT_NOTE.append("peer transport unavailable, fell back to NCCL: " + errs[0])
+        return None
+    return plan
+
+
 def max_over_ranks(torch, dist, dev, world, x: float) -> float:
     """Max of a per-rank float over the group (a CPU tensor on a gloo group, CUDA on NCCL)."""
     if world == 1:
@@ -425,9 +461,12 @@ def measure(fs, torch, dist, dev, world, rank, name, T, time_steps, steps, warmu
     w = wk.weights(weights)
     gext = (wk.extents[0] * world,) + tuple(wk.extents[1:])
     cells = int(np.prod(gext))
+    plan = None
     if world > 1 and transport == "peer":
-        plan = fs.Plan(gext, w, wk.radius, T, nranks=world, rank=rank, transport="peer")
-        plan.connect_peers()
+        plan = peer_plan(fs, dist, world, rank, gext, w, wk.radius, T)
+        if plan is None:
+            transport = "nccl"
+    if plan is not None:
         u0 = wl.grid(plan.extents, wk.cfg_id * 1000 + rank)   # this rank's slab, seeded per slab
     elif world > 1:
         obj = [fs.nccl_unique_id() if rank == 0 else None]
@@ -596,7 +635,7 @@ def main(argv=None):
                        "parallelism": "single GPU" if world == 1 else
                        f"outer-axis decomposition over {world} GPUs, r*T halo rows per pass "
                        + ("pushed into the neighbours' buffers (CUDA IPC peer copies, stream-memory signal/wait)"
-                          if args.transport == "peer" else "by NCCL send/recv"),
+                          if args.transport == "peer" and not TRANSPORT_NOTE else "by NCCL send/recv"),
                        "l2": f"inputs {int(np.prod(wk.extents)) * 8 / 1e6:.0f} MB per GPU > 126 MB L2 (no flush needed)"},
             "roofline": main_res["roofline"],
             "cpu_baseline": cpu,
@@ -608,7 +647,9 @@ def main(argv=None):
         if nccl_log:
             line["config"]["nccl"] = nccl_summary(nccl_log)
         if world > 1:
-            line["config"]["transport"] = args.transport
+            line["config"]["transport"] = args.transport if not TRANSPORT_NOTE else "nccl"
+            if TRANSPORT_NOTE:
+                line["config"]["transport_note"] = TRANSPORT_NOTE[0]
         if world > 1 and shared:
             line["shared_gpu"] = "every rank on device 0 (FFTSTENCIL_BENCH_SHARE_GPU=1): a harness test, not a scaling number"
         s = json.dumps(line)

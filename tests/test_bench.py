@@ -4,6 +4,7 @@ bench.py stacks the N=1 workload's rows N times along axis 0 (the global grid th
 decomposes back into per-rank slabs), so the throughput is global cells x time steps / the
 max-over-ranks time -- with no extra factor of the world size (reading Q18).
 """
+import pytest
 import bench
 from synth import workloads as wl
 
@@ -127,3 +128,62 @@ def test_world_size_mismatch_is_an_error(monkeypatch):
     monkeypatch.setenv("RANK", "0")
     with pytest.raises(SystemExit):
         bench.main(["--gpus", "4"])
+
+
+def _peer_plan_worker(rank, port, fail_rank, fail_stage, out):
+    import os
+
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=2)
+
+    class FakePlan:
+        closed = False
+
+        def __init__(self, *a, **k):
+            if rank == fail_rank and fail_stage == "create":
+                raise RuntimeError("no peer access")
+            self.extents = (4, 4)
+
+        def peer_handle(self):
+            return bytes([rank]) * 256
+
+        def peer_connect(self, lower, upper):
+            if rank == fail_rank and fail_stage == "connect":
+                raise RuntimeError("cudaIpcOpenMemHandle failed")
+            assert (lower is None) == (rank == 0) and (upper is None) == (rank == 1)
+
+        def close(self):
+            FakePlan.closed = True
+
+    class FakeFs:
+        Plan = FakePlan
+
+    bench.TRANSPORT_NOTE.clear()
+    plan = bench.peer_plan(FakeFs, dist, 2, rank, (8, 4), None, 1, 2)
+    out.put((rank, plan is not None, list(bench.TRANSPORT_NOTE)))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("fail_rank,fail_stage", [(-1, ""), (1, "create"), (0, "connect")])
+def test_peer_plan_falls_back_together(fail_rank, fail_stage):
+    """bench.peer_plan: either every rank gets a connected peer plan, or -- when any rank fails to
+    create / export / map -- every rank gets None (the group falls back to NCCL together), without
+    a rank stuck in a collective the others skipped (gloo, world size 2, CPU)."""
+    import multiprocessing as mp
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_peer_plan_worker, args=(r, port, fail_rank, fail_stage, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in ps)
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    ok = fail_rank < 0
+    assert all(r[1] == ok for r in res)
+    assert all(bool(r[2]) == (not ok) for r in res)
