@@ -69,7 +69,7 @@ if __name__ == "__main__":
     argv = sys.argv[1:]
     cut = argv.index("--") if "--" in argv else len(argv)
     names, settings = argv[:cut], (argv[cut + 1:] or ["-"])
-    for rep in range(2):
+    for rep in range(int(os.environ.get("ENV_AB_ROUNDS", "2"))):
         for name in names:
             for st in settings:
                 one(name, st)
