@@ -1252,6 +1252,26 @@ int fftstencil_peer_connect(fftstencil_plan* p, const void* lower, const void* u
     p->pE[side][1] = static_cast<double*>(ptrs[1]);
     p->pFlags[side] = static_cast<uint32_t*>(ptrs[2]);
   }
+  if (rc == FFTSTENCIL_OK) {
+    // probe both mechanisms now, so a missing peer path fails here (where callers can still agree
+    // on another transport) and not in the middle of a run: an 8-byte copy into each neighbour's
+    // first halo row (overwritten by the first push before any pass reads it) and a write of this
+    // rank's current epoch into the flag word only this rank writes
+    cudaStream_t ps = nullptr;
+    cudaError_t e = cudaStreamCreateWithFlags(&ps, cudaStreamNonBlocking);
+    for (int side = 0; side < 2 && e == cudaSuccess; ++side) {
+      if (!hs[side]) continue;
+      const int64_t row = side == 0 ? hp.row_lo : hp.row_hi - hp.h;   // its halo row this rank pushes first
+      e = cudaMemcpyAsync(p->pE[side][0] + (size_t)(row - p->pG0[side]) * p->row_cells,
+                          p->dE[0] + (size_t)(row - hp.g0) * p->row_cells, sizeof(double), cudaMemcpyDeviceToDevice, ps);
+      if (e == cudaSuccess &&
+          write_value_fn()((CUstream)ps, (CUdeviceptr)(p->pFlags[side] + (side == 0 ? 1 : 0)), p->epoch, 0) != CUDA_SUCCESS)
+        e = cudaErrorNotSupported;
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(ps);
+    if (ps) cudaStreamDestroy(ps);
+    if (e != cudaSuccess) rc = cuda_fail(e, "peer transport probe (copy / stream write into a neighbour's memory)");
+  }
   if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
   if (rc == FFTSTENCIL_OK) {
     p->peer_connected = true;
