@@ -103,6 +103,8 @@ typedef struct {
                                    copy-run-copy (FFTSTENCIL_E2E_PIPE=0, 1D, small grids, h > S) */
   int last_run_chunks;          /* that run's pipelined schedule: K input / output row chunks   */
   int last_run_depth;           /*   and Q skewed passes at each end (0 / 0 when not pipelined) */
+  int last_run_peer_fused;      /* peer transport: 1 if the last run's boundary rows reached the
+                                   neighbours as the kernels' own stores, 0 (copy pushes / other)  */
 } fftstencil_info;
 
 /* Plan creation flags (fftstencil_plan_create_ex / fftstencil_describe_ex). */
@@ -182,9 +184,11 @@ fftstencil_plan* fftstencil_plan_create_dist(int ndim, const int64_t* extents, c
 
 /* ---- peer-memory transport: the same decomposition without NCCL ----
  * Each rank's two slab buffers and a two-word flag array are shared with its neighbours through
- * CUDA IPC.  After every pass a rank copies its h = radius*T boundary rows straight into the
- * neighbours' halo rows (copy engine over NVLink; a same-device copy when two processes share
- * one GPU) and bumps the neighbours' flag word with a stream memory write; before its
+ * CUDA IPC.  In every pass the kernels that produce a rank's h = radius*T boundary rows (the edge
+ * tile pairs and the band) store those cells straight into the neighbours' halo rows as well
+ * (NVLink stores; same-device stores when processes share one GPU) -- or, for the DMMA engines
+ * and FFTSTENCIL_PEER_FUSED=0, the rows are copied there after the pass -- and the rank then
+ * bumps the neighbours' flag word with a stream memory write; before its
  * halo-dependent tile pairs a rank's stream waits (stream memory wait, no host round trip, no
  * spinning kernel) until both neighbours have signalled as often as it has.  Halo-free pairs
  * run before the wait, so the exchange overlaps them.  Results are bitwise equal to one GPU.

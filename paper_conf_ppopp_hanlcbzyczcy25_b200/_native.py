@@ -63,6 +63,7 @@ class Info(ctypes.Structure):
         ("last_run_pipelined", ctypes.c_int),
         ("last_run_chunks", ctypes.c_int),
         ("last_run_depth", ctypes.c_int),
+        ("last_run_peer_fused", ctypes.c_int),
     ]
 
     def as_dict(self) -> dict:
@@ -83,6 +84,7 @@ class Info(ctypes.Structure):
             "engine": ("dmma", "alu")[self.engine], "alu_ops_per_pass": self.alu_ops_per_pass,
             "last_run_pipelined": bool(self.last_run_pipelined),
             "last_run_chunks": self.last_run_chunks, "last_run_depth": self.last_run_depth,
+            "last_run_peer_fused": bool(self.last_run_peer_fused),
         }
 
 

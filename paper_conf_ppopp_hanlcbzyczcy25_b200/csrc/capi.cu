@@ -87,6 +87,7 @@ struct fftstencil_plan {
   int64_t last_launches = 0;
   bool last_pipelined = false;   // the last run_host took the pipelined schedule
   int last_chunks = 0, last_depth = 0;   // and its K / Q
+  bool last_peer_fused = false;          // the last peer-transport run pushed with the kernels' stores
   // ---- decomposition (dist) ----
   bool dist = false;          // slab plan with halo buffers
   bool loopback = false;      // no communicator: run by fftstencil_run_group
@@ -122,6 +123,9 @@ struct fftstencil_plan {
   uint32_t* pFlags[2] = {nullptr, nullptr};                       // the neighbours' dFlags
   int64_t pG0[2] = {0, 0};      // the neighbours' window starts g0
   uint32_t epoch = 0;           // signals sent so far (both neighbours send the same count)
+  bool peer_fused = true;       // boundary rows stored into the neighbours by the pass's own kernels
+                                // (FFTSTENCIL_PEER_FUSED=0: copy-engine push after the pass)
+  PeerStore peer_store = {nullptr, nullptr, 0, 0, 0, 0};   // set around a pass's edge launches + band
   int ecur = 0;               // index of the buffer holding the current state
   // ---- profiling: event pairs (start, end, kind 0 = fused, 1 = band) recorded by run() ----
   bool profiling = false;
@@ -314,6 +318,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
   const long pe_ = prof_begin(p, 0, s);
   if (hp.ndim == 2) {
     Fft2dArgs a;
+    a.peer = p->peer_store;
     a.src = src;
     a.dst = dst;
     a.n0 = hp.ext[0];
@@ -353,6 +358,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     }
   } else if (hp.ndim == 1) {
     Fft1dArgs a;
+    a.peer = p->peer_store;
     a.src = src;
     a.dst = dst;
     a.n = hp.ext[0];
@@ -386,6 +392,7 @@ int launch_fused(fftstencil_plan* p, const double* src, double* dst, int t, int6
     }
   } else {
     Fft3dArgs a;
+    a.peer = p->peer_store;
     a.src = src;
     a.dst = dst;
     a.n0 = hp.ext[0];
@@ -471,6 +478,7 @@ int band_args(const fftstencil_plan* p, const double* src, double* dst, int t, B
   for (double wv : hp.w) b.ntaps += wv != 0.0;
   b.clip_lo = p->band_clip_lo;
   b.clip_hi = p->band_clip_hi;
+  b.peer = p->peer_store;
   return nb;
 }
 
@@ -666,6 +674,20 @@ int peer_push(fftstencil_plan* p, int b, cudaStream_t s) {
   return e == cudaSuccess ? FFTSTENCIL_OK : cuda_fail(e, "peer halo push");
 }
 
+// As peer_push, from this rank's buffer `from` into the neighbours' buffer `to`.
+int peer_push_from(fftstencil_plan* p, int from, int to, cudaStream_t s) {
+  const HostPlan& hp = p->hp;
+  const size_t rc_ = p->row_cells, bytes = (size_t)hp.h * rc_ * sizeof(double);
+  cudaError_t e = cudaSuccess;
+  if (hp.rank > 0)
+    e = cudaMemcpyAsync(p->pE[0][to] + (size_t)(hp.row_lo - p->pG0[0]) * rc_,
+                        p->dE[from] + (size_t)(hp.row_lo - hp.g0) * rc_, bytes, cudaMemcpyDeviceToDevice, s);
+  if (e == cudaSuccess && hp.rank < hp.nranks - 1)
+    e = cudaMemcpyAsync(p->pE[1][to] + (size_t)(hp.row_hi - hp.h - p->pG0[1]) * rc_,
+                        p->dE[from] + (size_t)(hp.row_hi - hp.h - hp.g0) * rc_, bytes, cudaMemcpyDeviceToDevice, s);
+  return e == cudaSuccess ? FFTSTENCIL_OK : cuda_fail(e, "peer halo push");
+}
+
 // Epoch ++ written into both neighbours' flag words (stream-ordered after the push; the write
 // carries a memory barrier, so the neighbour sees the rows before the flag).
 int peer_signal(fftstencil_plan* p, cudaStream_t s) {
@@ -707,24 +729,42 @@ int peer_wait(fftstencil_plan* p, cudaStream_t s) {
 // for that pass's signal first), and never the owned rows the passes write.
 int run_dist_peer(fftstencil_plan* p, const double* in, double* out, int64_t total_steps, cudaStream_t s) {
   const HostPlan& hp = p->hp;
+  // fused pushes need the ALU kernels' PEER instantiations and the cone band kernel
+  int taps = 1;
+  for (int q = 0; q < hp.ndim; ++q) taps *= 2 * hp.radius + 1;
+  const bool fused = p->peer_fused && hp.algo == 1 && hp.engine == 1 && !p->band_reference && taps <= 512;
+  p->last_peer_fused = fused;
   int rc;
   if ((rc = peer_wait(p, s))) return rc;
   if ((rc = dist_begin(p, in, s))) return rc;
-  if ((rc = peer_push(p, 0, s)) || (rc = peer_signal(p, s))) return rc;
+  // the input's boundary rows into the neighbours' halo rows -- of both buffers when the passes
+  // push fused (their stores cover the computed cells only; the fixed-ring cells of those rows
+  // must already be in place in either buffer)
+  if ((rc = peer_push(p, 0, s)) || (fused && (rc = peer_push_from(p, 0, 1, s))) || (rc = peer_signal(p, s))) return rc;
   const int T = hp.T;
   const int64_t nfull = total_steps / T, P = nfull + (total_steps % T ? 1 : 0);
   for (int64_t i = 0; i < P; ++i) {
     const int t = i < nfull ? T : (int)(total_steps % T);
+    const int db = p->ecur ^ 1;
     const double* src = p->dE[p->ecur];
-    double* dst = p->dE[p->ecur ^ 1];
+    double* dst = p->dE[db];
     if ((rc = launch_fused(p, src, dst, t, hp.ipair_lo, hp.ipair_hi, s))) return rc;
     if ((rc = peer_wait(p, s))) return rc;
-    if ((rc = launch_fused(p, src, dst, t, hp.pair_lo, hp.ipair_lo, s))) return rc;
-    if ((rc = launch_fused(p, src, dst, t, hp.ipair_hi, hp.pair_hi, s))) return rc;
-    if ((rc = launch_band_pass(p, src, dst, t, s))) return rc;
-    if ((rc = band_join(p, s))) return rc;
+    if (fused) {   // the boundary rows' producers store them into the neighbours' buffer db too
+      p->peer_store.lo = hp.rank > 0 ? p->pE[0][db] : nullptr;
+      p->peer_store.lo_end = hp.row_lo + hp.h;
+      p->peer_store.lo_g0 = p->pG0[0];
+      p->peer_store.hi = hp.rank < hp.nranks - 1 ? p->pE[1][db] : nullptr;
+      p->peer_store.hi_begin = hp.row_hi - hp.h;
+      p->peer_store.hi_g0 = p->pG0[1];
+    }
+    rc = launch_fused(p, src, dst, t, hp.pair_lo, hp.ipair_lo, s);
+    if (!rc) rc = launch_fused(p, src, dst, t, hp.ipair_hi, hp.pair_hi, s);
+    if (!rc) rc = launch_band_pass(p, src, dst, t, s);
+    p->peer_store = PeerStore{nullptr, nullptr, 0, 0, 0, 0};
+    if (rc || (rc = band_join(p, s))) return rc;
     p->ecur ^= 1;
-    if (i + 1 < P && ((rc = peer_push(p, p->ecur, s)) || (rc = peer_signal(p, s)))) return rc;
+    if (i + 1 < P && ((!fused && (rc = peer_push(p, p->ecur, s))) || (rc = peer_signal(p, s)))) return rc;
   }
   if ((rc = dist_end(p, out, s))) return rc;
   return peer_signal(p, s);
@@ -906,6 +946,7 @@ int setup_device(fftstencil_plan* p) {
   if (const char* v = std::getenv("FFTSTENCIL_MAX_CTAS")) p->max_ctas = std::max(0, std::atoi(v));
   if (const char* v = std::getenv("FFTSTENCIL_3D_TRAV")) p->trav_blk = std::max(0, std::atoi(v));
   if (const char* v = std::getenv("FFTSTENCIL_ST256")) p->st256 = std::atoi(v) != 0;
+  if (const char* v = std::getenv("FFTSTENCIL_PEER_FUSED")) p->peer_fused = std::atoi(v) != 0;
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
   // 3D: the band (tens of thousands of small blocks) runs before the fused kernel on the run
   // stream -- concurrently, its CTAs hold SMs the register-full fused CTAs then wait for
@@ -1611,6 +1652,7 @@ int fftstencil_plan_info(const fftstencil_plan* p, fftstencil_info* info) {
   info->last_run_pipelined = p->last_pipelined ? 1 : 0;
   info->last_run_chunks = p->last_pipelined ? p->last_chunks : 0;
   info->last_run_depth = p->last_pipelined ? p->last_depth : 0;
+  info->last_run_peer_fused = p->last_peer_fused ? 1 : 0;
   clear_error();
   return FFTSTENCIL_OK;
 }

@@ -349,8 +349,20 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
   const int f0 = fdiv(NTH, O12), f1 = fdiv(NTH - f0 * O12, O2), f2 = NTH - f0 * O12 - f1 * O2;
   double* dst0 = a.dst + ((lo[0] - off[0]) * a.n[1] + (lo[1] - off[1])) * a.n[2] + (lo[2] - off[2]);
   const double* sb0 = b0 + ((lo[0] - rl[0]) * D[1] + (lo[1] - rl[1])) * D[2] + (lo[2] - rl[2]);
+  // peer transport: cells of the rank's boundary rows also go to the neighbour's halo rows
+  const bool peer = (a.peer.lo || a.peer.hi) && !a.reference;
   for (int e = threadIdx.x; e < ovol; e += NTH) {
-    dst0[((int64_t)j0 * a.n[1] + j1) * a.n[2] + j2] = sb0[(j0 * D[1] + j1) * D[2] + j2];
+    const double v = sb0[(j0 * D[1] + j1) * D[2] + j2];
+    dst0[((int64_t)j0 * a.n[1] + j1) * a.n[2] + j2] = v;
+    if (peer) {
+      int64_t c[3] = {lo[0] + j0, lo[1] + j1, lo[2] + j2};
+      const int64_t row = c[a.oax];
+      double* pb = row < a.peer.lo_end ? a.peer.lo : row >= a.peer.hi_begin ? a.peer.hi : nullptr;
+      if (pb) {
+        c[a.oax] = row - (row < a.peer.lo_end ? a.peer.lo_g0 : a.peer.hi_g0);
+        pb[(c[0] * a.n[1] + c[1]) * a.n[2] + c[2]] = v;
+      }
+    }
     j2 += f2;
     j1 += f1;
     j0 += f0;

@@ -155,7 +155,7 @@ __device__ __forceinline__ void twiddle4096(double (&xr)[16], double (&xi)[16], 
   }
 }
 
-template <bool TMA>
+template <bool TMA, bool PEER>
 __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double* sS, const double2* tw64,
                                             const double2* tw4k, const Fft1dArgs& a, const Geom& g, int warp,
                                             int lane, int grp, const CUtensorMap* tm, uint64_t* bar, bool has_next,
@@ -264,10 +264,22 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
       const int l = 16 * j + cc + 64 * (16 * i + rr);   // cell offset a + 64 b within the tile
       if (l >= la0 && l < la1) da[l] = br[i][j];
       if (l >= lb0 && l < lb1) db[l] = bi[i][j];
+      if (PEER) {   // boundary cells of a peer-transport rank: also into the neighbour's halo
+        const int64_t c = g.oa + l, d = g.ob + l;
+        if (l >= la0 && l < la1) {
+          if (c < a.peer.lo_end) a.peer.lo[c - a.peer.lo_g0] = br[i][j];
+          else if (c >= a.peer.hi_begin) a.peer.hi[c - a.peer.hi_g0] = br[i][j];
+        }
+        if (l >= lb0 && l < lb1) {
+          if (d < a.peer.lo_end) a.peer.lo[d - a.peer.lo_g0] = bi[i][j];
+          else if (d >= a.peer.hi_begin) a.peer.hi[d - a.peer.hi_g0] = bi[i][j];
+        }
+      }
     }
 }
 
-template <bool TMA, bool WRAP = false>
+// PEER: boundary cells of a peer-transport rank are also stored into the neighbour (a.peer).
+template <bool TMA, bool WRAP = false, bool PEER = false>
 __global__ void __launch_bounds__(2 * NT, 1) fft1d_bf_kernel(const Fft1dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ unsigned char smem_raw[];
   const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
@@ -319,7 +331,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft1d_bf_kernel(const Fft1dArgs a, 
     }
     const bool has_next = p + stride < p_end;
     const Geom gn = geom(a, has_next ? p + stride : p);
-    tile_passes<TMA>(sR, sI, sS, tw64, tw4k, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn);
+    tile_passes<TMA, PEER>(sR, sI, sS, tw64, tw4k, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn);
   }
 }
 
@@ -334,12 +346,23 @@ cudaError_t fused1d_bf_configure(int* max_blocks) {
   if (e == cudaSuccess) e = cudaFuncSetAttribute(fft1d_bf_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(fft1d_bf_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft1d_bf_kernel<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft1d_bf_kernel<false, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
   if (e != cudaSuccess) return e;
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft1d_bf_kernel<true>, 2 * NT, sm);
 }
 
 cudaError_t launch_fused1d_bf(const Fft1dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s) {
   static const CUtensorMap none = {};
+  if (a.peer.lo || a.peer.hi) {   // boundary cells of a peer-transport rank (never periodic)
+    if (tm)
+      fft1d_bf_kernel<true, false, true><<<grid, 2 * NT, fused1d_bf_smem(), s>>>(a, *tm);
+    else
+      fft1d_bf_kernel<false, false, true><<<grid, 2 * NT, fused1d_bf_smem(), s>>>(a, none);
+    return cudaGetLastError();
+  }
   if (tm)
     fft1d_bf_kernel<true><<<grid, 2 * NT, fused1d_bf_smem(), s>>>(a, *tm);
   else if (a.bd.wrap)

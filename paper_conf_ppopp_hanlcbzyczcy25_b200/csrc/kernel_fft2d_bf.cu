@@ -361,7 +361,7 @@ __device__ __forceinline__ void block_store(double* sR, double* sI, int rr, int 
 // caller waited for them in the first memory phase); releases the buffer (TMA refill of the
 // group's next pair `gn`) after P5's reads, then stores the window.  M / C mark the memory and
 // compute phases of the ping-pong schedule (BF_PINGPONG).
-template <bool TMA>
+template <bool TMA, bool PEER>
 __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double* sS, const double2* tw,
                                             const Fft2dArgs& a, const Geom& g, int warp, int lane, int grp,
                                             const CUtensorMap* tm, uint64_t* bar, bool has_next, const Geom& gn,
@@ -468,10 +468,24 @@ __device__ __forceinline__ void tile_passes(double* sR, double* sI, const double
       if (va[j]) drow[ca + 16 * j] = br[i][j];
       if (vb[j]) drow[cb + 16 * j] = bi[i][j];
     }
+    if (PEER) {   // boundary rows of a peer-transport rank: the same cells into the neighbour's halo row
+      const int64_t c0 = g.o0 + r;
+      double* prow = c0 < a.peer.lo_end ? a.peer.lo + (c0 - a.peer.lo_g0) * a.n1
+                   : c0 >= a.peer.hi_begin ? a.peer.hi + (c0 - a.peer.hi_g0) * a.n1 : nullptr;
+      if (prow) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          if (va[j]) prow[ca + 16 * j] = br[i][j];
+          if (vb[j]) prow[cb + 16 * j] = bi[i][j];
+        }
+      }
+    }
   }
 }
 
-template <bool TMA, bool WRAP = false>
+// PEER: boundary rows of a peer-transport rank are also stored into the neighbour (a.peer,
+// kernels.cuh); a separate instantiation, the single-GPU kernel is unchanged.
+template <bool TMA, bool WRAP = false, bool PEER = false>
 __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ unsigned char smem_raw[];
   const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
@@ -569,7 +583,7 @@ __global__ void __launch_bounds__(2 * NT, 1) fft2d_bf_kernel(const Fft2dArgs a, 
     }
     const bool has_next = p + stride < a.win.p_end;
     const Geom gn = geom(a, has_next ? p + stride : p);
-    tile_passes<TMA>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn, tmem_s, last);
+    tile_passes<TMA, PEER>(sR, sI, sS, tw, a, g, warp, lane, grp, &tm, &bar[grp], has_next, gn, tmem_s, last);
   }
   if (BF_TMEM_S) {
     asm volatile("tcgen05.fence::before_thread_sync;\n");
@@ -590,12 +604,23 @@ cudaError_t fused2d_bf_configure(int* max_blocks) {
   if (e == cudaSuccess) e = cudaFuncSetAttribute(fft2d_bf_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(fft2d_bf_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft2d_bf_kernel<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, st);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft2d_bf_kernel<false, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
   if (e != cudaSuccess) return e;
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft2d_bf_kernel<true>, 2 * NT, st);
 }
 
 cudaError_t launch_fused2d_bf(const Fft2dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s) {
   static const CUtensorMap none = {};
+  if (a.peer.lo || a.peer.hi) {   // boundary rows of a peer-transport rank (never periodic)
+    if (tm)
+      fft2d_bf_kernel<true, false, true><<<grid, 2 * NT, fused2d_bf_smem(true), s>>>(a, *tm);
+    else
+      fft2d_bf_kernel<false, false, true><<<grid, 2 * NT, fused2d_bf_smem(false), s>>>(a, none);
+    return cudaGetLastError();
+  }
   if (tm)
     fft2d_bf_kernel<true><<<grid, 2 * NT, fused2d_bf_smem(true), s>>>(a, *tm);
   else if (a.bd.wrap)

@@ -121,7 +121,10 @@ __device__ __forceinline__ PairGeom pair_geom(const Fft3dArgs& a, int64_t p) {
 // line (t >> 4, t & 15) of every pass, so a warp's P1 rows and P2 lines lie in the same two
 // l0-planes (P1 -> P2 needs only __syncwarp), and likewise P4 -> P5 on the output planes.
 // TMA = false: cp.async loads (periodic wrap-around, or a pitch TMA cannot describe).
-template <bool TMA, bool WRAP = false>
+// PEER: the launch holds boundary rows of a peer-transport rank (a.peer, kernels.cuh): its output
+// rows within h of the slab edge are stored into the neighbour's buffer too (a separate
+// instantiation, so the single-GPU kernel's code and registers are untouched).
+template <bool TMA, bool WRAP = false, bool PEER = false>
 __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, const __grid_constant__ CUtensorMap tm) {
   extern __shared__ unsigned char smem_raw[];
   const uint32_t mis = tma::smem_addr(smem_raw) & (kAlign - 1);
@@ -292,6 +295,21 @@ __global__ void __launch_bounds__(2 * NT, 1) fft3d_bf_kernel(const Fft3dArgs a, 
               if (g.has_b && c2 < a.bd.lim2) drow[c2] = xi[l2];
             }
         }
+        if (PEER) {   // the same cells into the neighbour's halo row (NVLink stores)
+          double* prow = c0 < a.peer.lo_end ? a.peer.lo + ((c0 - a.peer.lo_g0) * a.n1 + c1) * a.n2
+                       : c0 >= a.peer.hi_begin ? a.peer.hi + ((c0 - a.peer.hi_g0) * a.n1 + c1) * a.n2
+                                               : nullptr;
+          if (prow) {
+#pragma unroll
+            for (int l2 = 0; l2 < 16; ++l2)
+              if (l2 >= h && l2 < h + S) {
+                int64_t c2 = g.oa2 + l2;
+                if (c2 < a.bd.lim2) prow[c2] = xr[l2];
+                c2 = g.ob2 + l2;
+                if (g.has_b && c2 < a.bd.lim2) prow[c2] = xi[l2];
+              }
+          }
+        }
       }
     }
   }
@@ -308,12 +326,23 @@ cudaError_t fused3d_bf_configure(int* max_blocks) {
   if (e == cudaSuccess) e = cudaFuncSetAttribute(fft3d_bf_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(fft3d_bf_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft3d_bf_kernel<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, st);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fft3d_bf_kernel<false, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sc);
   if (e != cudaSuccess) return e;
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(max_blocks, fft3d_bf_kernel<true>, 2 * NT, st);
 }
 
 cudaError_t launch_fused3d_bf(const Fft3dArgs& a, const CUtensorMap* tm, int grid, cudaStream_t s) {
   static const CUtensorMap none = {};
+  if (a.peer.lo || a.peer.hi) {   // boundary rows of a peer-transport rank (never periodic)
+    if (tm)
+      fft3d_bf_kernel<true, false, true><<<grid, 2 * NT, fused3d_bf_smem(true), s>>>(a, *tm);
+    else
+      fft3d_bf_kernel<false, false, true><<<grid, 2 * NT, fused3d_bf_smem(false), s>>>(a, none);
+    return cudaGetLastError();
+  }
   if (tm)
     fft3d_bf_kernel<true><<<grid, 2 * NT, fused3d_bf_smem(true), s>>>(a, *tm);
   else if (a.bd.wrap)

@@ -29,6 +29,17 @@ struct Bound {
   int64_t lim0, lim1, lim2;
 };
 
+// Fused halo push of the peer transport (capi.cu run_dist_peer): a launch that produces a rank's
+// boundary rows also stores every cell of global outer-axis row c < lo_end into the lower
+// neighbour's buffer `lo` (an IPC-mapped pointer; its row 0 is global row lo_g0) and of row
+// c >= hi_begin into the upper neighbour's `hi` (row 0 = hi_g0), so the exchange is the pass's own
+// stores over NVLink, tile by tile.  lo / hi null: no such neighbour, or a launch without them.
+struct PeerStore {
+  double* lo;
+  double* hi;
+  int64_t lo_end, lo_g0, hi_begin, hi_g0;
+};
+
 __host__ __device__ __forceinline__ int64_t wrap_index(int64_t x, int64_t n) {
   x %= n;
   return x < 0 ? x + n : x;
@@ -54,6 +65,7 @@ struct Fft2dArgs {
   const double* Sre;     // L x L powered spectrum of this pass, natural row-major
   const double* Sim;
   double* spec;          // unfused ablation only: [pair][re|im][k0][k1] spectrum in HBM
+  PeerStore peer;        // multi-GPU peer transport: boundary rows also stored to the neighbours
 };
 
 // One fused pass of the 1D path: prime-factor 8 x 7 tile (kernel_fft1d.cu) or the
@@ -72,6 +84,7 @@ struct Fft1dArgs {
   const double* Sim;
   const int* crt;        // PFA: 64 tile positions stored at (l1, l2), -1 = padding
   const double* tw;      // factored: w4096^(a c) at [a][c], interleaved (re, im)
+  PeerStore peer;        // multi-GPU peer transport: boundary rows also stored to the neighbours
 };
 
 // One fused pass of the 3D path over every tile pair (kernel_fft3d.cu); 16^3 tiles.
@@ -96,6 +109,7 @@ struct Fft3dArgs {
   // 16-byte store of l2, l2 + 1, for l2 in [h, h + S).  launch_fused sets st32 only when every
   // tile row starts 32-byte aligned (S, n2 multiples of 4, no shift, dst 32-byte aligned).
   int st32, st16;
+  PeerStore peer;        // multi-GPU peer transport: boundary rows also stored to the neighbours
 };
 
 // Direct T-step recomputation of the boundary band (kernel_band.cu).
@@ -114,6 +128,7 @@ struct BandArgs {
   int region_cells;      // host hint: largest block region (cells) at t = T -- sizes the 1D CTA
   int ntaps;             // host hint: nonzero weights (selects a register-tap specialisation)
   int64_t clip_lo, clip_hi;   // only outer-axis rows [clip_lo, clip_hi) are produced (pipelined run_host)
+  PeerStore peer;        // multi-GPU peer transport: boundary rows also stored to the neighbours
 };
 
 // Copy a box (embedded coordinates) from src to dst0 and dst1 (either may be null).

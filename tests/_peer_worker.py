@@ -17,7 +17,8 @@ import paper_conf_ppopp_hanlcbzyczcy25_b200 as fs  # noqa: E402
 from synth import workloads as wl  # noqa: E402
 
 CASES = [((300, 170), "box", 1, 4, (11, 4)), ((257, 129), "star", 3, 2, (9,)), ((60, 40, 50), "box", 1, 2, (5, 2)),
-         ((5000,), "star", 1, 8, (19,)), ((2048, 256), "box", 1, 0, (40, 13)), ((90, 30, 34), "star", 1, 3, (7,))]
+         ((5000,), "star", 1, 8, (19,)), ((2048, 256), "box", 1, 0, (40, 13)), ((90, 30, 34), "star", 1, 3, (7,)),
+         ((300000,), "star", 1, 0, (2100,))]   # 1D factored ALU engine (4096-cell tiles, T = 1024)
 
 
 def main():
@@ -39,6 +40,7 @@ def main():
             p.run(a, b, steps)
             torch.cuda.synchronize()
             a = b
+        fused = p.info()["last_run_peer_fused"]
         slabs = [None] * world
         dist.all_gather_object(slabs, a.cpu().numpy())
         if rank == 0:
@@ -51,8 +53,8 @@ def main():
                 x = y
             torch.cuda.synchronize()
             ok = np.array_equal(got, y.cpu().numpy())
-            print(f"case {ext} r={r} T={inf['T']} ranks={world} devices={min(ndev, world)} runs={runs}: "
-                  f"bitwise {'OK' if ok else 'MISMATCH'}", flush=True)
+            print(f"case {ext} r={r} T={inf['T']} ranks={world} devices={min(ndev, world)} runs={runs} "
+                  f"engine={inf['engine']} fused_push={int(fused)}: bitwise {'OK' if ok else 'MISMATCH'}", flush=True)
             bad += not ok
             q.close()
         dist.barrier()   # every rank done with its plan before any closes its IPC-shared buffers

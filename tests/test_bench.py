@@ -39,7 +39,7 @@ def test_smem_wavefront_model():
 
 
 def _sass_mix(obj):
-    """(DADD, DMUL, DFMA) static counts of the TMA instantiation (<true, false>) in `obj`,
+    """(DADD, DMUL, DFMA) static counts of the TMA instantiation (<true, false[, false]>) in `obj`,
     without the band-folding subroutine (the CALL right before the kernel's final EXIT, up to
     its RET): the mix weights the FP64 peak of the tile passes, which is what bench.py reports."""
     import re
@@ -48,7 +48,8 @@ def _sass_mix(obj):
     lines, inside = [], False
     for ln in out.splitlines():
         if "Function" in ln:
-            inside = "ILb1ELb0E" in ln
+            # the TMA, non-periodic, single-GPU instantiation (not the peer-store one, <1, 0, 1>)
+            inside = "ILb1ELb0E" in ln and "ILb1ELb0ELb1E" not in ln
             continue
         m = re.match(r"\s*/\*([0-9a-f]+)\*/\s+(.*)", ln)
         if inside and m:

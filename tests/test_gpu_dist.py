@@ -105,11 +105,12 @@ def test_nccl_two_ranks_bitwise(fs, tmp_path):
     assert "Init COMPLETE" in log or "ncclCommInitRank" in log, "no NCCL communicator was initialised"
 
 
-@pytest.mark.parametrize("nproc", [2, 3])
-def test_peer_transport_processes(fs, tmp_path, nproc):
-    """The peer-memory transport (CUDA IPC halo pushes + stream-memory signal / wait, no NCCL)
-    across `nproc` processes -- on one GPU when only one is visible (IPC within a device), else
-    one GPU per rank -- bitwise equal to one GPU over chained calls (G7)."""
+@pytest.mark.parametrize("nproc,fused", [(2, 1), (3, 1), (2, 0)])
+def test_peer_transport_processes(fs, tmp_path, nproc, fused):
+    """The peer-memory transport (no NCCL) across `nproc` processes -- on one GPU when only one is
+    visible (IPC within a device), else one GPU per rank -- bitwise equal to one GPU over chained
+    calls (G7).  fused = 1: the boundary rows reach the neighbours as the edge tiles' and the
+    band's own stores (default); 0: a copy-engine push after each pass."""
     import os
     import socket
     import subprocess
@@ -120,8 +121,13 @@ def test_peer_transport_processes(fs, tmp_path, nproc):
     worker = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_peer_worker.py")
     res = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
                           "--master-addr=127.0.0.1", f"--master-port={port}", worker],
-                         capture_output=True, text=True, timeout=900)
+                         capture_output=True, text=True, timeout=900,
+                         env=dict(os.environ, FFTSTENCIL_PEER_FUSED=str(fused)))
     log = res.stdout + res.stderr
     (tmp_path / "peer.log").write_text(log)
     assert res.returncode == 0, log[-4000:]
-    assert log.count("bitwise OK") == 6, log[-4000:]
+    assert log.count("bitwise OK") == 7, log[-4000:]
+    if fused:   # the 1D, 2D and 3D ALU-engine cases push with the kernels' stores
+        assert log.count("fused_push=1") >= 6, log[-4000:]
+    else:
+        assert "fused_push=1" not in log, log[-4000:]
