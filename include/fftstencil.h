@@ -199,7 +199,12 @@ fftstencil_plan* fftstencil_plan_create_dist(int ndim, const int64_t* extents, c
  * channel: torch.distributed, files, ...) and each connects to its neighbours
  * (fftstencil_peer_connect: lower = rank-1's handle or NULL for rank 0, upper = rank+1's or NULL
  * for the last rank).  fftstencil_run before connecting fails with EINVAL.  The devices of
- * neighbouring ranks must be peer capable (NVLink/NVSwitch), or the same device. */
+ * neighbouring ranks must be peer capable (NVLink/NVSwitch), or the same device; connect probes
+ * a peer copy and a stream-memory write and fails (ECUDA) if either does not work, so the caller
+ * can still choose another transport.  Errors: a run that fails midway leaves the ranks out of
+ * lockstep -- destroy the group's plans.  Destroy: every rank's stream work must be finished
+ * (e.g. synchronise, then a host barrier) before any rank destroys its plan, because the
+ * neighbours write into its buffers. */
 #define FFTSTENCIL_PEER_HANDLE_BYTES 256
 fftstencil_plan* fftstencil_plan_create_dist_peer(int ndim, const int64_t* extents, const double* weights,
                                                   int radius, int T, int nranks, int rank);
