@@ -503,13 +503,14 @@ def measure(fs, torch, dist, dev, world, rank, name, T, time_steps, steps, warmu
     prof = plan.profile_read()
     plan.set_profiling(False)
     launches = plan.info()["last_run_launches"]
+    peer_fused = plan.info()["last_run_peer_fused"]
     ms = ev0.elapsed_time(ev1)
     ms_max = max_over_ranks(torch, dist, dev, world, ms)
     passes = steps * -(-time_steps // info["T"])
     res = {"workload": name, "value": gstencils(cells, time_steps * steps, ms_max), "unit": "GStencils/s",
            "ms_per_step": ms_max / steps, "steps": steps, "time_steps_per_step": time_steps,
            "T": info["T"], "tile": info["tile"], "valid": info["valid"], "grid": list(gext),
-           "gpu_launches_per_step": int(launches),
+           "gpu_launches_per_step": int(launches), "peer_fused": bool(peer_fused),
            "roofline": roofline_of(info, prof, passes, exact_cells_of(info, gext), name),
            "fused_share_of_step": prof["fused_ms"] / max(ms, 1e-9)}
     res["roofline"]["fused_share_of_step"] = res["fused_share_of_step"]
@@ -647,7 +648,9 @@ def main(argv=None):
         if nccl_log:
             line["config"]["nccl"] = nccl_summary(nccl_log)
         if world > 1:
-            line["config"]["transport"] = args.transport if not TRANSPORT_NOTE else "nccl"
+            line["config"]["transport"] = (("peer: halo rows stored into the neighbours by the edge tiles' and band's kernels"
+                                            if main_res.get("peer_fused") else "peer: halo rows copied after each pass")
+                                           if args.transport == "peer" and not TRANSPORT_NOTE else "nccl")
             if TRANSPORT_NOTE:
                 line["config"]["transport_note"] = TRANSPORT_NOTE[0]
         if world > 1 and shared:
