@@ -211,6 +211,15 @@ fftstencil_plan* fftstencil_plan_create_dist_peer(int ndim, const int64_t* exten
 int fftstencil_peer_handle(const fftstencil_plan* plan, void* out, int64_t cap);
 int fftstencil_peer_connect(fftstencil_plan* plan, const void* lower, const void* upper);
 
+/* Host-only: the op list a peer-transport run of rank `rank` executes (capi.cu run_dist_peer; the
+ * op codes are in csrc/plan.h build_peer_schedule: WAIT / COPYIN / PUSH / SIGNAL / INTERIOR /
+ * EDGE / COPYOUT), for `total_steps` steps, fused stores or copy pushes, after `epoch0` earlier
+ * signals; 4 int64 per op.  `out` holds `cap` ops (NULL queries the count).  Returns the number
+ * of ops or a negative code.  For CPU replays of the multi-rank protocol (tests/test_dist.py). */
+int64_t fftstencil_peer_schedule(int ndim, const int64_t* extents, const double* weights, int radius,
+                                 int T, int nranks, int rank, int64_t total_steps, int fused,
+                                 int64_t epoch0, int64_t* out, int64_t cap);
+
 /* Writes a new 128-byte ncclUniqueId into `out` (caller-owned, >= 128 bytes; rank 0 of a
  * group).  ENCCL if NCCL cannot create one.  No PAPER.md passage: the paper is single-GPU;
  * the decomposition is SURVEY §8(a) row a10. */

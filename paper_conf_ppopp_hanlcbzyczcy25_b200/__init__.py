@@ -18,7 +18,7 @@ import numpy as np
 from . import _native
 from ._native import FftStencilError, Info, last_error
 
-__all__ = ["Plan", "describe", "describe_dist", "export_aux", "e2e_schedule", "nccl_unique_id", "run_group", "FftStencilError"]
+__all__ = ["Plan", "describe", "describe_dist", "export_aux", "e2e_schedule", "peer_schedule", "nccl_unique_id", "run_group", "FftStencilError"]
 
 
 def _arrays(extents, weights, radius):
@@ -105,6 +105,23 @@ def export_aux(extents, weights, radius: int, T: int, which: int, axis: int = 0,
     out = np.empty(int(n), dtype=np.float64)
     m = L.fftstencil_export_aux(int(ext.size), _i64p(ext), _dp(w), int(radius), int(T), int(which), int(axis),
                                 int(t), _dp(out), int(n))
+    if m < 0:
+        raise FftStencilError(int(m), last_error())
+    return out
+
+
+def peer_schedule(extents, weights, radius: int, T: int, nranks: int, rank: int, total_steps: int,
+                  fused: bool = True, epoch0: int = 0) -> np.ndarray:
+    """Op list of a peer-transport run of one rank, shape (n, 4) int64 (fftstencil_peer_schedule)."""
+    ext, w = _arrays(extents, weights, radius)
+    L = _native.lib()
+    args = (int(ext.size), _i64p(ext), _dp(w), int(radius), int(T), int(nranks), int(rank), int(total_steps),
+            int(bool(fused)), int(epoch0))
+    n = L.fftstencil_peer_schedule(*args, None, 0)
+    if n < 0:
+        raise FftStencilError(int(n), last_error())
+    out = np.zeros((int(n), 4), dtype=np.int64)
+    m = L.fftstencil_peer_schedule(*args, out.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)), int(n))
     if m < 0:
         raise FftStencilError(int(m), last_error())
     return out

@@ -23,7 +23,7 @@ EXPORTS = ("fftstencil_plan_create", "fftstencil_run", "fftstencil_run_host", "f
            "fftstencil_nccl_unique_id", "fftstencil_run_group", "fftstencil_describe_dist",
            "fftstencil_plan_create_ex", "fftstencil_describe_ex", "fftstencil_run_emit",
            "fftstencil_e2e_schedule", "fftstencil_plan_create_dist_peer", "fftstencil_peer_handle",
-           "fftstencil_peer_connect")
+           "fftstencil_peer_connect", "fftstencil_peer_schedule")
 PEER_HANDLE_BYTES = 256   # FFTSTENCIL_PEER_HANDLE_BYTES
 
 
@@ -135,6 +135,10 @@ def lib():
     L.fftstencil_plan_create_dist_peer.restype = vp
     L.fftstencil_peer_handle.argtypes = [vp, vp, ctypes.c_int64]
     L.fftstencil_peer_handle.restype = ctypes.c_int
+    L.fftstencil_peer_schedule.argtypes = [ctypes.c_int, i64p, dp, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                           ctypes.c_int, ctypes.c_int64, ctypes.c_int, ctypes.c_int64, i64p,
+                                           ctypes.c_int64]
+    L.fftstencil_peer_schedule.restype = ctypes.c_int64
     L.fftstencil_peer_connect.argtypes = [vp, vp, vp]
     L.fftstencil_peer_connect.restype = ctypes.c_int
     L.fftstencil_nccl_unique_id.argtypes = [vp]

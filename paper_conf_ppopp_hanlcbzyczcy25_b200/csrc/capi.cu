@@ -661,20 +661,7 @@ int nccl_exchange(fftstencil_plan* p, cudaStream_t s) {
 // row_lo on, at its local row row_lo - g0_lower); rows [row_hi - h, row_hi) to the upper
 // neighbour's (its local rows from 0).  Copy engine over NVLink (same-device copy when the
 // "neighbour" is another process on this GPU), ordered on `s` after the pass that wrote them.
-int peer_push(fftstencil_plan* p, int b, cudaStream_t s) {
-  const HostPlan& hp = p->hp;
-  const size_t rc_ = p->row_cells, bytes = (size_t)hp.h * rc_ * sizeof(double);
-  cudaError_t e = cudaSuccess;
-  if (hp.rank > 0)
-    e = cudaMemcpyAsync(p->pE[0][b] + (size_t)(hp.row_lo - p->pG0[0]) * rc_, p->dE[b] + (size_t)(hp.row_lo - hp.g0) * rc_,
-                        bytes, cudaMemcpyDeviceToDevice, s);
-  if (e == cudaSuccess && hp.rank < hp.nranks - 1)
-    e = cudaMemcpyAsync(p->pE[1][b] + (size_t)(hp.row_hi - hp.h - p->pG0[1]) * rc_,
-                        p->dE[b] + (size_t)(hp.row_hi - hp.h - hp.g0) * rc_, bytes, cudaMemcpyDeviceToDevice, s);
-  return e == cudaSuccess ? FFTSTENCIL_OK : cuda_fail(e, "peer halo push");
-}
-
-// As peer_push, from this rank's buffer `from` into the neighbours' buffer `to`.
+// Here from this rank's buffer `from` into the neighbours' buffer `to`.
 int peer_push_from(fftstencil_plan* p, int from, int to, cudaStream_t s) {
   const HostPlan& hp = p->hp;
   const size_t rc_ = p->row_cells, bytes = (size_t)hp.h * rc_ * sizeof(double);
@@ -690,9 +677,9 @@ int peer_push_from(fftstencil_plan* p, int from, int to, cudaStream_t s) {
 
 // Epoch ++ written into both neighbours' flag words (stream-ordered after the push; the write
 // carries a memory barrier, so the neighbour sees the rows before the flag).
-int peer_signal(fftstencil_plan* p, cudaStream_t s) {
+int peer_signal(fftstencil_plan* p, uint32_t e, cudaStream_t s) {
   const HostPlan& hp = p->hp;
-  ++p->epoch;
+  p->epoch = e;
   CUresult r = CUDA_SUCCESS;
   if (hp.rank > 0) r = write_value_fn()((CUstream)s, (CUdeviceptr)(p->pFlags[0] + 1), p->epoch, 0);
   if (r == CUDA_SUCCESS && hp.rank < hp.nranks - 1)
@@ -705,15 +692,15 @@ int peer_signal(fftstencil_plan* p, cudaStream_t s) {
 }
 
 // `s` waits until both neighbours have signalled as often as this rank.
-int peer_wait(fftstencil_plan* p, cudaStream_t s) {
+int peer_wait(fftstencil_plan* p, uint32_t target, cudaStream_t s) {
   const HostPlan& hp = p->hp;
   // peer copies land in this device's memory before the writer's flag (the write-value carries a
   // memory barrier); no remote-write flush is needed (that flag is for third-party RDMA writers)
   const unsigned flags = CU_STREAM_WAIT_VALUE_GEQ;
   CUresult r = CUDA_SUCCESS;
-  if (hp.rank > 0) r = wait_value_fn()((CUstream)s, (CUdeviceptr)(p->dFlags + 0), p->epoch, flags);
+  if (hp.rank > 0) r = wait_value_fn()((CUstream)s, (CUdeviceptr)(p->dFlags + 0), target, flags);
   if (r == CUDA_SUCCESS && hp.rank < hp.nranks - 1)
-    r = wait_value_fn()((CUstream)s, (CUdeviceptr)(p->dFlags + 1), p->epoch, flags);
+    r = wait_value_fn()((CUstream)s, (CUdeviceptr)(p->dFlags + 1), target, flags);
   if (r != CUDA_SUCCESS) {
     set_error("cuStreamWaitValue32 failed (" + std::to_string((int)r) + ")");
     return FFTSTENCIL_ECUDA;
@@ -734,40 +721,46 @@ int run_dist_peer(fftstencil_plan* p, const double* in, double* out, int64_t tot
   for (int q = 0; q < hp.ndim; ++q) taps *= 2 * hp.radius + 1;
   const bool fused = p->peer_fused && hp.algo == 1 && hp.engine == 1 && !p->band_reference && taps <= 512;
   p->last_peer_fused = fused;
-  int rc;
-  if ((rc = peer_wait(p, s))) return rc;
-  if ((rc = dist_begin(p, in, s))) return rc;
-  // the input's boundary rows into the neighbours' halo rows -- of both buffers when the passes
-  // push fused (their stores cover the computed cells only; the fixed-ring cells of those rows
-  // must already be in place in either buffer)
-  if ((rc = peer_push(p, 0, s)) || (fused && (rc = peer_push_from(p, 0, 1, s))) || (rc = peer_signal(p, s))) return rc;
+  // the schedule (plan.cpp build_peer_schedule; replayed on the CPU by tests/test_dist.py) and
+  // its execution, op by op
+  std::vector<int64_t> ops;
+  int rc = build_peer_schedule(hp, total_steps, fused, p->epoch, ops);
+  if (rc) { set_error("peer schedule"); return rc; }
   const int T = hp.T;
-  const int64_t nfull = total_steps / T, P = nfull + (total_steps % T ? 1 : 0);
-  for (int64_t i = 0; i < P; ++i) {
-    const int t = i < nfull ? T : (int)(total_steps % T);
-    const int db = p->ecur ^ 1;
-    const double* src = p->dE[p->ecur];
-    double* dst = p->dE[db];
-    if ((rc = launch_fused(p, src, dst, t, hp.ipair_lo, hp.ipair_hi, s))) return rc;
-    if ((rc = peer_wait(p, s))) return rc;
-    if (fused) {   // the boundary rows' producers store them into the neighbours' buffer db too
-      p->peer_store.lo = hp.rank > 0 ? p->pE[0][db] : nullptr;
-      p->peer_store.lo_end = hp.row_lo + hp.h;
-      p->peer_store.lo_g0 = p->pG0[0];
-      p->peer_store.hi = hp.rank < hp.nranks - 1 ? p->pE[1][db] : nullptr;
-      p->peer_store.hi_begin = hp.row_hi - hp.h;
-      p->peer_store.hi_g0 = p->pG0[1];
+  const int64_t nfull = total_steps / T;
+  for (size_t i = 0; i < ops.size() && !rc; i += 4) {
+    const int64_t op = ops[i], a = ops[i + 1], b = ops[i + 2], c = ops[i + 3];
+    const int t = a <= nfull ? T : (int)(total_steps % T);
+    switch (op) {
+      case 0: rc = peer_wait(p, (uint32_t)a, s); break;
+      case 1: rc = dist_begin(p, in, s); break;
+      case 2: rc = peer_push_from(p, (int)a, (int)b, s); break;
+      case 3: rc = peer_signal(p, (uint32_t)a, s); break;
+      case 4: rc = launch_fused(p, p->dE[b], p->dE[b ^ 1], t, hp.ipair_lo, hp.ipair_hi, s); break;
+      case 5: {
+        const double* src = p->dE[b];
+        double* dst = p->dE[b ^ 1];
+        if (c) {   // the boundary rows' producers store them into the neighbours' buffer b ^ 1 too
+          p->peer_store.lo = hp.rank > 0 ? p->pE[0][b ^ 1] : nullptr;
+          p->peer_store.lo_end = hp.row_lo + hp.h;
+          p->peer_store.lo_g0 = p->pG0[0];
+          p->peer_store.hi = hp.rank < hp.nranks - 1 ? p->pE[1][b ^ 1] : nullptr;
+          p->peer_store.hi_begin = hp.row_hi - hp.h;
+          p->peer_store.hi_g0 = p->pG0[1];
+        }
+        rc = launch_fused(p, src, dst, t, hp.pair_lo, hp.ipair_lo, s);
+        if (!rc) rc = launch_fused(p, src, dst, t, hp.ipair_hi, hp.pair_hi, s);
+        if (!rc) rc = launch_band_pass(p, src, dst, t, s);
+        p->peer_store = PeerStore{nullptr, nullptr, 0, 0, 0, 0};
+        if (!rc) rc = band_join(p, s);
+        break;
+      }
+      default:
+        p->ecur = (int)a;
+        rc = dist_end(p, out, s);
     }
-    rc = launch_fused(p, src, dst, t, hp.pair_lo, hp.ipair_lo, s);
-    if (!rc) rc = launch_fused(p, src, dst, t, hp.ipair_hi, hp.pair_hi, s);
-    if (!rc) rc = launch_band_pass(p, src, dst, t, s);
-    p->peer_store = PeerStore{nullptr, nullptr, 0, 0, 0, 0};
-    if (rc || (rc = band_join(p, s))) return rc;
-    p->ecur ^= 1;
-    if (i + 1 < P && ((!fused && (rc = peer_push(p, p->ecur, s))) || (rc = peer_signal(p, s)))) return rc;
   }
-  if ((rc = dist_end(p, out, s))) return rc;
-  return peer_signal(p, s);
+  return rc;
 }
 
 // One pass of a dist rank: interior pairs overlap the exchange (if `xchg`), then the
@@ -1034,6 +1027,27 @@ int fftstencil_describe_dist(int ndim, const int64_t* extents, const double* wei
   fill_info(hp, info);
   clear_error();
   return FFTSTENCIL_OK;
+}
+
+int64_t fftstencil_peer_schedule(int ndim, const int64_t* extents, const double* weights, int radius, int T,
+                                 int nranks, int rank, int64_t total_steps, int fused, int64_t epoch0, int64_t* out,
+                                 int64_t cap) {
+  HostPlan hp;
+  std::string err;
+  int rc = build_host_plan(ndim, extents, weights, radius, T, hp, err, nranks, rank, env_algo());
+  if (rc != FFTSTENCIL_OK) { set_error(err); return rc; }
+  std::vector<int64_t> ops;
+  if ((rc = build_peer_schedule(hp, total_steps, fused != 0, epoch0, ops)) != FFTSTENCIL_OK) {
+    set_error("nranks must be >= 2 and total_steps >= 0");
+    return rc;
+  }
+  const int64_t n = (int64_t)ops.size() / 4;
+  if (out) {
+    if (cap < n) { set_error("cap smaller than the number of ops"); return FFTSTENCIL_EINVAL; }
+    std::memcpy(out, ops.data(), ops.size() * sizeof(int64_t));
+  }
+  clear_error();
+  return n;
 }
 
 int64_t fftstencil_e2e_schedule(int ndim, const int64_t* extents, const double* weights, int radius, int T,

@@ -727,4 +727,34 @@ int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std
   return FFTSTENCIL_OK;
 }
 
+int build_peer_schedule(const HostPlan& p, int64_t total_steps, bool fused, int64_t epoch0, std::vector<int64_t>& ops) {
+  ops.clear();
+  if (p.nranks < 2 || total_steps < 0) return FFTSTENCIL_EINVAL;
+  auto push = [&](int64_t op, int64_t a, int64_t b, int64_t c) {
+    ops.push_back(op); ops.push_back(a); ops.push_back(b); ops.push_back(c);
+  };
+  if (total_steps == 0) return FFTSTENCIL_OK;   // a copy, no exchange and no signal (all ranks alike)
+  int64_t e = epoch0;
+  push(0, e, 0, 0);                 // neighbours done with the previous run: their pushes may land
+  push(1, 0, 0, 0);
+  push(2, 0, 0, 0);
+  if (fused) push(2, 0, 1, 0);      // fused stores cover computed cells only: ring cells into both
+  push(3, ++e, 0, 0);
+  const int64_t P = total_steps / p.T + (total_steps % p.T ? 1 : 0);
+  int cur = 0;
+  for (int64_t k = 1; k <= P; ++k) {
+    push(4, k, cur, 0);
+    push(0, e, 0, 0);
+    push(5, k, cur, fused ? 1 : 0);
+    cur ^= 1;
+    if (k < P) {
+      if (!fused) push(2, cur, cur, 0);
+      push(3, ++e, 0, 0);
+    }
+  }
+  push(6, cur, 0, 0);
+  push(3, ++e, 0, 0);
+  return FFTSTENCIL_OK;
+}
+
 }  // namespace fstencil

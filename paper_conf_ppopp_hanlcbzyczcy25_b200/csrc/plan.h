@@ -108,6 +108,20 @@ int build_host_plan(int ndim, const int64_t* extents, const double* weights, int
 int build_e2e_schedule(const HostPlan& p, int64_t total_steps, int K, int Q, std::vector<int64_t>& ops, int Qt = 0,
                        int ramp = 1);
 
+// Peer-transport run of one rank (capi.cu run_dist_peer executes exactly this list): ops of 4
+// int64 {op, a, b, c} in stream order, epochs absolute (the rank has sent `epoch0` signals before):
+//   0 WAIT e        the stream waits until both neighbours have signalled >= e times;
+//   1 COPYIN        the caller's slab -> owned rows of buffer 0 (+ fixed ring into buffer 1);
+//   2 PUSH f, t     own boundary rows of buffer f -> the neighbours' halo rows of their buffer t;
+//   3 SIGNAL e      write e into both neighbours' flag words (this rank's e-th signal);
+//   4 INTERIOR k, s      pass k's halo-free tile pairs: reads owned rows of buffer s, writes rows
+//                        [row_lo + h, row_hi - h) of buffer s ^ 1;
+//   5 EDGE k, s, f       pass k's edge pairs and band: reads rows [g0, g1) of s (halos included),
+//                        writes the owned boundary rows of s ^ 1 and, if f, the same rows into
+//                        the neighbours' buffer s ^ 1 (fused stores);
+//   6 COPYOUT s     owned rows of buffer s -> the caller's slab.
+int build_peer_schedule(const HostPlan& p, int64_t total_steps, bool fused, int64_t epoch0, std::vector<int64_t>& ops);
+
 // Dense-DFT tile cost model (executed FP64 tensor flops per cell-step) used to pick L/T.
 double model_flops_2d(int L, int S, int T);
 // Factored (CT 8 x 8, L = 64) tile: executed FP64 flops per cell-step (DMMA + twiddles + S_T).

@@ -147,3 +147,128 @@ def test_gloo_two_rank_halo_protocol(case):
     assert res[0] == "ok", res
     assert res[1], f"decomposed result differs from the oracle (max abs {res[2]})"
     assert all(p.exitcode == 0 for p in procs)
+
+
+# ---------------------------------------------------------------- peer transport protocol replay
+def _peer_replay(ext, shape, r, T, n, runs, fused, seed):
+    """Replays the op lists the library executes for a peer-transport group (fftstencil_peer_schedule,
+    the same list capi.cu run_dist_peer runs) under one random interleaving of the ranks' streams
+    (a stream blocks only at WAIT).  Row versions are tracked per rank, buffer and outer row:
+    every read must see the previous pass's data (so a neighbour's write that lands before the read
+    it must follow -- a race -- shows up as a wrong version), halo rows must carry the fixed-ring
+    cells (a full-row copy has landed), and the copy-out must see the last pass."""
+    rng = np.random.default_rng(seed)
+    w = wl.seeded_weights(shape, len(ext), r)
+    geo = [fs.describe_dist(ext, w, r, T, n, k) for k in range(n)]
+    h, n0 = geo[0]["halo"], ext[0]
+    lo = [g["row_begin"] for g in geo]
+    hi = [g["row_end"] for g in geo]
+    g0 = [max(0, lo[k] - h) if k > 0 else 0 for k in range(n)]
+    g1 = [min(n0, hi[k] + h) if k < n - 1 else n0 for k in range(n)]
+    ver = np.full((n, 2, n0), -1)      # version = run * 10^6 + pass (0 = the run's input)
+    ring = np.zeros((n, 2, n0), bool)  # full rows (with their fixed-ring cells) in place
+    sig = [0] * n
+    progs, epoch = [], [0] * n
+    plan_T = geo[0]["T"]
+    for k in range(n):
+        ops, e = [], 0
+        for ri, steps in enumerate(runs):
+            sch = fs.peer_schedule(ext, w, r, T, n, k, steps, fused, e)
+            ops += [(ri, tuple(int(x) for x in op)) for op in sch]
+            e = max([e] + [int(op[1]) for op in sch if op[0] == 3])
+        progs.append(ops)
+    pc = [0] * n
+    nbrs = lambda k: [q for q in (k - 1, k + 1) if 0 <= q < n]  # noqa: E731
+    bnd = lambda k: (np.arange(lo[k], lo[k] + h), np.arange(hi[k] - h, hi[k]))  # noqa: E731
+    while True:
+        live = [k for k in range(n) if pc[k] < len(progs[k])]
+        if not live:
+            break
+        ready = [k for k in live if progs[k][pc[k]][1][0] != 0 or all(sig[q] >= progs[k][pc[k]][1][1] for q in nbrs(k))]
+        assert ready, f"deadlock: {[progs[k][pc[k]] for k in live]}"
+        k = int(rng.choice(ready))
+        ri, (op, a, b, c) = progs[k][pc[k]]
+        pc[k] += 1
+        base = ri * 10**6
+        P = -(-runs[ri] // plan_T)
+        if op == 1:        # COPYIN: input into buffer 0, fixed ring into buffer 1 (owned rows)
+            ver[k, 0, lo[k]:hi[k]] = base
+            ring[k, :, lo[k]:hi[k]] = True
+        elif op == 2:      # PUSH a -> b: own boundary rows into the neighbours' halo rows
+            for q in nbrs(k):
+                rows = bnd(k)[0] if q < k else bnd(k)[1]
+                ver[q, b, rows] = ver[k, a, rows]
+                ring[q, b, rows] = True
+        elif op == 3:
+            sig[k] = a
+        elif op == 4:      # INTERIOR: reads owned rows of b, writes [lo + h, hi - h) of b ^ 1
+            assert (ver[k, b, lo[k]:hi[k]] == base + a - 1).all(), f"rank {k} pass {a}: interior read a stale row"
+            ver[k, b ^ 1, lo[k] + h:hi[k] - h] = base + a
+        elif op == 5:      # EDGE: reads [g0, g1) of b, writes the boundary rows (+ the neighbours')
+            rows = slice(g0[k], g1[k])
+            assert (ver[k, b, rows] == base + a - 1).all(), f"rank {k} pass {a}: edge read a stale / overwritten row"
+            assert ring[k, b, rows].all(), f"rank {k} pass {a}: halo row without its fixed-ring cells"
+            for side, rr in zip((0, 1), bnd(k)):
+                ver[k, b ^ 1, rr] = base + a
+                q = k - 1 if side == 0 else k + 1
+                if c and 0 <= q < n:
+                    ver[q, b ^ 1, rr] = base + a
+        elif op == 6:      # COPYOUT
+            assert (ver[k, a, lo[k]:hi[k]] == base + P).all(), f"rank {k} run {ri}: copy-out before the last pass"
+    return progs
+
+
+PEER_CASES = [((300, 170), "box", 1, 4, 3), ((257, 129), "star", 3, 2, 2), ((60, 40, 50), "box", 1, 2, 2),
+              ((5000,), "star", 1, 8, 4), ((2048, 256), "box", 1, 0, 4), ((90, 30, 34), "star", 1, 3, 3)]
+
+
+@pytest.mark.parametrize("fused", [True, False])
+@pytest.mark.parametrize("ext,shape,r,T,n", PEER_CASES)
+def test_peer_schedule_replays_race_free(ext, shape, r, T, n, fused):
+    """50 random interleavings of the ranks' streams, three chained runs (the second a single
+    pass, the last with a remainder pass): every read sees exactly the previous pass."""
+    Tp = fs.describe(ext, wl.seeded_weights(shape, len(ext), r), r, T)["T"]
+    runs = (3 * Tp + 1, Tp, 2 * Tp)
+    for seed in range(50):
+        _peer_replay(ext, shape, r, T, n, runs, fused, seed)
+
+
+def test_peer_replay_catches_a_missing_wait():
+    """Mutation check: dropping the WAIT before a pass's edge work lets a rank read its halo rows
+    before the neighbour's data for that pass arrived -- some interleaving must fail."""
+    orig = fs.peer_schedule
+
+    def no_edge_wait(*a, **k):
+        ops = orig(*a, **k)
+        keep = [i for i in range(len(ops)) if not (ops[i][0] == 0 and i + 1 < len(ops) and ops[i + 1][0] == 5)]
+        return ops[keep]
+
+    fs.peer_schedule = no_edge_wait
+    try:
+        failed = 0
+        for seed in range(200):
+            try:
+                _peer_replay((300, 170), "box", 1, 4, 3, (13,), True, seed)
+            except AssertionError:
+                failed += 1
+        assert failed > 0
+    finally:
+        fs.peer_schedule = orig
+
+
+def test_peer_replay_catches_a_missing_ring_push():
+    """Mutation check: without the begin-of-run push into buffer 1, fused stores leave buffer 1's
+    halo rows without their fixed-ring cells."""
+    orig = fs.peer_schedule
+
+    def no_second_push(*a, **k):
+        ops = orig(*a, **k)
+        keep = [i for i in range(len(ops)) if not (ops[i][0] == 2 and ops[i][2] == 1 and ops[i][1] == 0)]
+        return ops[keep]
+
+    fs.peer_schedule = no_second_push
+    try:
+        with pytest.raises(AssertionError):
+            _peer_replay((300, 170), "box", 1, 4, 2, (13,), True, 0)
+    finally:
+        fs.peer_schedule = orig
