@@ -124,7 +124,9 @@ __device__ __forceinline__ int fdiv(int x, int d) {
 // the fused kernel leaves free (capi.cu), so per-step latency is what counts.
 // NTAPS > 0: the stencil has exactly NTAPS nonzero taps (host-counted); the lean cone loop then
 // keeps offsets and weights in registers, fully unrolled (no shared-memory tap loads, no loop).
-template <int NTH, int NTAPS = 0>
+// PEER: the launch holds boundary rows of a peer-transport rank; their cells are also stored into the
+// neighbour's halo rows (a.peer) -- a separate instantiation, the store loop of the others is unchanged.
+template <int NTH, int NTAPS = 0, bool PEER = false>
 __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(const BandArgs a) {
   extern __shared__ double sb[];
   __shared__ int s_off[kMaxTaps];
@@ -350,11 +352,10 @@ __global__ void __launch_bounds__(NTH, NTH == 256 ? 6 : 1) band_cone_kernel(cons
   double* dst0 = a.dst + ((lo[0] - off[0]) * a.n[1] + (lo[1] - off[1])) * a.n[2] + (lo[2] - off[2]);
   const double* sb0 = b0 + ((lo[0] - rl[0]) * D[1] + (lo[1] - rl[1])) * D[2] + (lo[2] - rl[2]);
   // peer transport: cells of the rank's boundary rows also go to the neighbour's halo rows
-  const bool peer = (a.peer.lo || a.peer.hi) && !a.reference;
   for (int e = threadIdx.x; e < ovol; e += NTH) {
     const double v = sb0[(j0 * D[1] + j1) * D[2] + j2];
     dst0[((int64_t)j0 * a.n[1] + j1) * a.n[2] + j2] = v;
-    if (peer) {
+    if (PEER) {
       int64_t c[3] = {lo[0] + j0, lo[1] + j1, lo[2] + j2};
       const int64_t row = c[a.oax];
       double* pb = row < a.peer.lo_end ? a.peer.lo : row >= a.peer.hi_begin ? a.peer.hi : nullptr;
@@ -415,6 +416,17 @@ cudaError_t band_configure(size_t smem) {
   if ((e = cudaFuncSetAttribute(band_cone_kernel<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
       cudaSuccess)
     return e;
+  if ((e = cudaFuncSetAttribute(band_cone_kernel<256, 5, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)lim1)) != cudaSuccess ||
+      (e = cudaFuncSetAttribute(band_cone_kernel<256, 7, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)lim1)) != cudaSuccess ||
+      (e = cudaFuncSetAttribute(band_cone_kernel<256, 0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)lim1)) != cudaSuccess ||
+      (e = cudaFuncSetAttribute(band_cone_kernel<1024, 0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)lim1)) != cudaSuccess ||
+      (e = cudaFuncSetAttribute(band_cone_kernel<64, 0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)lim1)) != cudaSuccess)
+    return e;
   if ((e = cudaFuncSetAttribute(band_cone_kernel<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lim1)) !=
       cudaSuccess)
     return e;
@@ -424,28 +436,38 @@ cudaError_t band_configure(size_t smem) {
   return smem <= lim0 && smem <= lim1 ? cudaSuccess : cudaErrorInvalidValue;
 }
 
+template <bool PEER>
+void launch_cone(const BandArgs& a, size_t smem, cudaStream_t s, bool one_d) {
+  // 1D: 1024 threads for the long bands of deep-fusion plans (t ~ 1000 sequential steps over
+  // thousands of cells); a 64-thread CTA when the region is small (e.g. configs[0]: 23 cells,
+  // where 32 mostly idle warps spent ~150 issue slots each per step: 15 us vs ~3 us)
+  if (one_d && a.region_cells > 512)
+    band_cone_kernel<1024, 0, PEER><<<a.nblocks, 1024, smem, s>>>(a);
+  else if (one_d)
+    band_cone_kernel<64, 0, PEER><<<a.nblocks, 64, smem, s>>>(a);
+  else
+    // register-resident taps for 5- and 7-point stars (9 taps spill at the 40-register budget
+    // and measured 0.4% slower, profiles/r01_s3_ab_band_tapreg.txt)
+    switch (BAND_LEAN && BAND_TAPREG ? a.ntaps : 0) {
+      case 5: band_cone_kernel<256, 5, PEER><<<a.nblocks, kBandThreads, smem, s>>>(a); break;
+      case 7: band_cone_kernel<256, 7, PEER><<<a.nblocks, kBandThreads, smem, s>>>(a); break;
+      default: band_cone_kernel<256, 0, PEER><<<a.nblocks, kBandThreads, smem, s>>>(a);
+    }
+}
+
 cudaError_t launch_band(const BandArgs& a, size_t smem, cudaStream_t s) {
   if (a.nblocks <= 0) return cudaSuccess;
   int taps = 1;
   for (int q = 0; q < 3; ++q) taps *= a.active[q] ? 2 * a.r + 1 : 1;
   const bool one_d = a.active[0] + a.active[1] + a.active[2] == 1;
-  // 1D: 1024 threads for the long bands of deep-fusion plans (t ~ 1000 sequential steps over
-  // thousands of cells); a 64-thread CTA when the region is small (e.g. configs[0]: 23 cells,
-  // where 32 mostly idle warps spent ~150 issue slots each per step: 15 us vs ~3 us)
-  if (taps <= kMaxTaps && !a.reference && one_d && a.region_cells > 512)
-    band_cone_kernel<1024><<<a.nblocks, 1024, smem, s>>>(a);
-  else if (taps <= kMaxTaps && !a.reference && one_d)
-    band_cone_kernel<64><<<a.nblocks, 64, smem, s>>>(a);
-  else if (taps <= kMaxTaps && !a.reference)
-    // register-resident taps for 5- and 7-point stars (9 taps spill at the 40-register budget
-    // and measured 0.4% slower, profiles/r01_s3_ab_band_tapreg.txt)
-    switch (BAND_LEAN && BAND_TAPREG ? a.ntaps : 0) {
-      case 5: band_cone_kernel<256, 5><<<a.nblocks, kBandThreads, smem, s>>>(a); break;
-      case 7: band_cone_kernel<256, 7><<<a.nblocks, kBandThreads, smem, s>>>(a); break;
-      default: band_cone_kernel<256><<<a.nblocks, kBandThreads, smem, s>>>(a);
-    }
-  else
+  if (taps <= kMaxTaps && !a.reference) {
+    if (a.peer.lo || a.peer.hi)
+      launch_cone<true>(a, smem, s, one_d);
+    else
+      launch_cone<false>(a, smem, s, one_d);
+  } else {
     band_kernel<<<a.nblocks, kBandThreads, smem, s>>>(a);
+  }
   return cudaGetLastError();
 }
 
