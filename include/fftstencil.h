@@ -159,8 +159,10 @@ int fftstencil_run_emit(fftstencil_plan* plan, const double* in, const int64_t* 
  * while the first Q passes advance row-skewed behind it, and the last Q passes finish the
  * result chunk by chunk while earlier chunks are copied out; results are bitwise equal to
  * fftstencil_run.  The copies run on a plan-owned stream ordered after / before `stream`.
- * Environment: FFTSTENCIL_E2E_PIPE=K (default 6, 0 = plain copy-run-copy),
- * FFTSTENCIL_E2E_DEPTH=Q (default 16), FFTSTENCIL_E2E_BAND_SMS (SMs left to the band, 4). */
+ * Environment: FFTSTENCIL_E2E_PIPE=K (default 6..12 by grid size, 0 = plain copy-run-copy),
+ * FFTSTENCIL_E2E_DEPTH=Q (default 16 for 2D, 20 for 3D plans), FFTSTENCIL_E2E_DEPTH_TAIL (tail
+ * depth, default Q), FFTSTENCIL_E2E_RAMP (1), FFTSTENCIL_E2E_BAND_SMS (SMs left to the band, 4);
+ * fftstencil_plan_info reports the K / Q the last call took. */
 int fftstencil_run_host(fftstencil_plan* plan, const double* h_in, double* h_out,
                         int64_t total_steps, void* stream);
 
