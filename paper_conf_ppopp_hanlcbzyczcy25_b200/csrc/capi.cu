@@ -941,11 +941,12 @@ int setup_device(fftstencil_plan* p) {
   if (const char* v = std::getenv("FFTSTENCIL_ST256")) p->st256 = std::atoi(v) != 0;
   if (const char* v = std::getenv("FFTSTENCIL_PEER_FUSED")) p->peer_fused = std::atoi(v) != 0;
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
-  // 3D: the band (tens of thousands of small blocks) runs before the fused kernel on the run
-  // stream -- concurrently, its CTAs hold SMs the register-full fused CTAs then wait for
-  // (Heat-3D 224.1 concurrent vs 228.1 serialised, profiles/r02_band3d.txt); 2D keeps the side
-  // stream (its band is ~45 us and hides in the fused kernel's tail: 1326 vs 1300)
-  if (hp.ndim == 3) p->band_concurrent = false;
+  // The band runs on its side stream, concurrent with the fused kernel, for 2D and 3D plans.  3D
+  // plans serialised it for a while (the slower band's CTAs held SMs the register-full fused CTAs
+  // then waited for: Heat-3D 224.1 concurrent vs 228.1 serialised, profiles/r02_band3d.txt); with
+  // the cp.async / fdiv band the side stream wins again (Heat-3D 432.0 vs 434.4 ms per step, e2e
+  // 503.2 vs 506.2 ms, Box-3D27P +0.4 %, profiles/r02_bandstream2.txt).  FFTSTENCIL_BAND_STREAM=0
+  // serialises it.
   if (const char* v = std::getenv("FFTSTENCIL_BAND_STREAM")) p->band_concurrent = std::atoi(v) != 0;
   if (hp.band_blocks.empty()) p->band_concurrent = false;
   if (p->band_concurrent) {
