@@ -97,6 +97,7 @@ struct fftstencil_plan {
   // ---- the band kernel runs on a side stream, concurrent with the fused kernel (it reads
   // the same source and writes disjoint cells); FFTSTENCIL_BAND_STREAM=0 serialises it ----
   bool band_concurrent = true;
+  bool band_e2e_concurrent = true;   // the pipelined run_host's items run the band on the side stream
   bool small1d = false;       // whole run in one on-chip launch (small 1D PFA plans, kernel_small1d.cu)
   cudaStream_t band_stream = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_band = nullptr;
@@ -941,15 +942,20 @@ int setup_device(fftstencil_plan* p) {
   if (const char* v = std::getenv("FFTSTENCIL_ST256")) p->st256 = std::atoi(v) != 0;
   if (const char* v = std::getenv("FFTSTENCIL_PEER_FUSED")) p->peer_fused = std::atoi(v) != 0;
   if (const char* v = std::getenv("FFTSTENCIL_BAND")) p->band_reference = !std::strcmp(v, "reference");
-  // The band runs on its side stream, concurrent with the fused kernel, for 2D and 3D plans.  3D
-  // plans serialised it for a while (the slower band's CTAs held SMs the register-full fused CTAs
-  // then waited for: Heat-3D 224.1 concurrent vs 228.1 serialised, profiles/r02_band3d.txt); with
-  // the cp.async / fdiv band the side stream wins again (Heat-3D 432.0 vs 434.4 ms per step, e2e
-  // 503.2 vs 506.2 ms, Box-3D27P +0.4 %, profiles/r02_bandstream2.txt).  FFTSTENCIL_BAND_STREAM=0
-  // serialises it.
+  // 2D plans run the band on its side stream, concurrent with the fused kernel.  3D plans run it
+  // before the fused kernel on the run stream in fftstencil_run: concurrent, its CTAs hold SMs the
+  // register-full fused CTAs then wait for (Heat-3D 224.1 vs 228.1 serialised with the round-1
+  // band, profiles/r02_band3d.txt); with the faster cp.async / fdiv band the comparison depends on
+  // the box: +0.55 % concurrent on one, -1.5 % on a power-capped one where the overlap lowers the
+  // SM clock (1935 vs 1950 MHz) (profiles/r02_bandstream2.txt, r02_bandstream3.txt) -- so the device
+  // path stays serialised, while the pipelined run_host, whose many small band launches gain from
+  // overlapping the fused items on both boxes (e2e +0.6 / +0.9 %), runs them concurrently
+  // (band_e2e_concurrent).  FFTSTENCIL_BAND_STREAM=0|1 and FFTSTENCIL_E2E_BAND_STREAM=0|1 override.
+  if (hp.ndim == 3) p->band_concurrent = false;
   if (const char* v = std::getenv("FFTSTENCIL_BAND_STREAM")) p->band_concurrent = std::atoi(v) != 0;
-  if (hp.band_blocks.empty()) p->band_concurrent = false;
-  if (p->band_concurrent) {
+  if (const char* v = std::getenv("FFTSTENCIL_E2E_BAND_STREAM")) p->band_e2e_concurrent = std::atoi(v) != 0;
+  if (hp.band_blocks.empty()) p->band_concurrent = p->band_e2e_concurrent = false;
+  if (p->band_concurrent || p->band_e2e_concurrent) {
     e = cudaStreamCreateWithFlags(&p->band_stream, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->ev_band, cudaEventDisableTiming);
@@ -1495,7 +1501,10 @@ static int run_host_pipelined_ops(fftstencil_plan* p, const double* h_in, double
 static int run_host_pipelined(fftstencil_plan* p, const double* h_in, double* h_out,
                               const std::vector<int64_t>& ops, int64_t total_steps, cudaStream_t caller) {
   cudaStream_t s = caller;
+  const bool conc = p->band_concurrent;
+  p->band_concurrent = conc || p->band_e2e_concurrent;
   const int rc = run_host_pipelined_ops(p, h_in, h_out, ops, total_steps, caller, s);
+  p->band_concurrent = conc;
   if (rc != FFTSTENCIL_OK) {
     const std::string err = g_last_error;
     cudaEvent_t ev;
